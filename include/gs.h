@@ -1,0 +1,224 @@
+/*
+ * gs.h -- C ABI of the B200-native gSampler ECSF sampling hot path.
+ *
+ * The library (libgsb200.so, sources in paper_conf_sosp_gonglmc0lwl23_b200/csrc)
+ * runs every step of the path in hand-written sm_100a CUDA kernels:
+ *   Extract  A[:, frontiers]                      PAPER.md Table 4
+ *   Compute  row/column sums, broadcast divides    Table 4, Fig. 3(b)/(c)
+ *   Select   individual_sample / collective_sample Table 4; walks P:75
+ *   Finalize row()/column(), relabel, compaction   Table 4
+ * ("P:n" = line n of the paper text /root/reference/PAPER.md.)
+ * The paper fixes WHAT is sampled, not HOW; the readings (sampling algorithms,
+ * Philox keying, output order) are listed in DESIGN.md "Readings" (R1..R25).
+ *
+ * Conventions (all entry points):
+ *  - Plain pointers and sizes only.  "device" pointers must be CUDA device (or
+ *    managed) memory of the current device; "host" pointers are CPU memory.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    Calls are stream-ordered: they validate host-side arguments, enqueue
+ *    kernels and return without synchronising unless stated otherwise.
+ *  - Every call returns gs_status; on failure gs_last_error() (thread-local)
+ *    holds a message.  No C++ exception crosses the ABI.
+ *  - Node ids are int32 (N < 2^31); indptr and edge ids are int64.
+ *  - Results depend only on (graph, seeds, batch_size, batch_index_base,
+ *    rng_key, parameters): not on stream, device, launch geometry or the
+ *    number of ranks sharing an epoch.
+ */
+#ifndef GS_H
+#define GS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum gs_status {
+  GS_OK = 0,
+  GS_ERR_INVALID_ARGUMENT = 1,   /* bad pointer / size / mode (host-side check)   */
+  GS_ERR_OUT_OF_MEMORY = 2,      /* allocation through the allocator hook failed  */
+  GS_ERR_CUDA = 3,               /* a CUDA runtime call or kernel launch failed   */
+  GS_ERR_UNSORTED_GRAPH = 4,     /* Node2Vec needs ascending CSC columns          */
+  GS_ERR_INDEX_OUT_OF_RANGE = 5, /* a seed/start id outside [0, N) (device-detected) */
+  GS_ERR_NOT_SUPPORTED = 6,      /* parameter outside the implemented envelope    */
+  GS_ERR_CAPACITY = 7,           /* a device-side output capacity was exceeded    */
+  GS_ERR_INVALID_GRAPH = 8       /* CSC validation failed in gs_graph_create      */
+} gs_status;
+
+const char* gs_last_error(void);
+const char* gs_status_string(gs_status s);
+/* Library version: major*10000 + minor*100 + patch. */
+int gs_version(void);
+
+/* Device-memory hook.  Every device buffer the library owns (graph copies,
+ * blocks, workspaces) is obtained through alloc(bytes, stream, ctx) and
+ * returned through free(ptr, bytes, stream, ctx).  Default (both NULL):
+ * cudaMalloc / cudaFree.  The Python binding installs PyTorch's caching
+ * allocator here, so PyTorch owns the device memory.  Not thread-safe: set it
+ * before creating objects; objects remember the hook they were created with. */
+typedef void* (*gs_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*gs_free_fn)(void* ptr, size_t bytes, void* stream, void* ctx);
+gs_status gs_set_allocator(gs_alloc_fn alloc, gs_free_fn free_fn, void* ctx);
+
+/* ------------------------------------------------------------------------ */
+/* Graph (a0): CSC adjacency, column v = in-neighbours of v.          */
+/* ------------------------------------------------------------------------ */
+typedef struct gs_graph gs_graph;
+
+enum {
+  GS_GRAPH_HOST_PTRS = 1, /* indptr/indices/weights are host pointers (copied to HBM)      */
+  GS_GRAPH_BORROW = 2     /* device pointers are used in place; caller keeps them alive    */
+};                        /* default (0): device pointers, copied into library-owned HBM  */
+
+/* Validates the CSC on the device (indptr[0] == 0, monotone, indptr[N] ==
+ * num_edges, 0 <= indices < N) and records whether every column is sorted
+ * ascending (needed by Node2Vec).  Synchronises `stream` once (one-off).
+ *   indptr  int64[num_nodes + 1], indices int32[num_edges],
+ *   weights fp32[num_edges] or NULL (unweighted: w == 1).
+ * Returns GS_ERR_INVALID_GRAPH if validation fails. */
+gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const float* weights,
+                          int64_t num_nodes, int64_t num_edges, uint32_t flags, void* stream,
+                          gs_graph** out);
+
+typedef struct gs_graph_info {
+  int64_t num_nodes, num_edges;
+  int weighted;       /* weights present */
+  int sorted;         /* every column ascending */
+  int64_t max_in_degree;
+  const int64_t* indptr;   /* device */
+  const int32_t* indices;  /* device */
+  const float* weights;    /* device or NULL */
+} gs_graph_info;
+gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out);
+void gs_graph_destroy(gs_graph* g);
+
+/* ------------------------------------------------------------------------ */
+/* Sample blocks: the result of the sampling calls.                           */
+/* ------------------------------------------------------------------------ */
+/* A gs_blocks object owns device buffers holding, for every (batch, layer),
+ * one sampled sub-matrix of A ("block") over local ids plus its relabel
+ * maps (A.column(), A.row()).  Seeds are cut into batches of
+ * batch_size (the last may be shorter); batch b is independent of every other
+ * (super-batch sampling with per-batch id spaces).
+ *
+ * Reuse: pass `*out == NULL` to create a new object, or a previous result to
+ * reuse its buffers (grown through the allocator when too small; reuse with
+ * unchanged shapes performs no allocation and is CUDA-graph capturable). */
+typedef struct gs_blocks gs_blocks;
+
+typedef struct gs_block_view {
+  int64_t n_cols, n_rows, n_edges;
+  const int32_t* col_map;   /* [n_cols]  local column -> global node (the frontier)      */
+  const int32_t* row_map;   /* [n_rows]  local row -> global node; next layer's frontier */
+  const int64_t* indptr;    /* [n_cols+1] CSC over local ids, indptr[0] == 0             */
+  const int32_t* row_local; /* [n_edges] local row of each edge                           */
+  const int64_t* eid;       /* [n_edges] global edge id (position in indices)            */
+  const float* val;         /* [n_edges] or NULL: LADIES/FastGCN edge value, PASS prob   */
+  const float* row_prob;    /* [n_rows] or NULL: layer-wise p(u) = b(u)/B                */
+} gs_block_view;            /* all pointers are DEVICE pointers into the gs_blocks object */
+
+/* Waits for the stream the blocks were produced on, copies the per-(batch,
+ * layer) counts to the host and reports device-detected errors
+ * (GS_ERR_INDEX_OUT_OF_RANGE, GS_ERR_CAPACITY). */
+gs_status gs_blocks_sync(gs_blocks* b);
+gs_status gs_blocks_shape(const gs_blocks* b, int64_t* num_batches, int* num_layers);
+/* Device pointers of one block; requires a prior gs_blocks_sync. */
+gs_status gs_blocks_view(const gs_blocks* b, int64_t batch, int layer, gs_block_view* out);
+/* Sync-free access: device int64 [num_batches][num_layers][GS_META_FIELDS]:
+ * (n_cols, n_rows, n_edges, col_offset, row_offset, indptr_offset,
+ * edge_offset, 0) -- the offsets locate the block inside the layer-wide
+ * arrays of gs_blocks_layer. */
+enum { GS_META_FIELDS = 8 };
+gs_status gs_blocks_device_meta(const gs_blocks* b, const int64_t** meta);
+
+typedef struct gs_layer_buffers {   /* whole-layer device arrays of one layer */
+  int32_t* col_map;   int64_t col_capacity;
+  int32_t* row_map;   int64_t row_capacity;
+  int64_t* indptr;    int64_t indptr_capacity;
+  int32_t* row_local; int64_t* eid; float* val; int64_t edge_capacity; /* val may be NULL */
+  float* row_prob;    /* [row_capacity] or NULL */
+} gs_layer_buffers;
+gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out);
+void gs_blocks_destroy(gs_blocks* b);
+
+/* ------------------------------------------------------------------------ */
+/* Node-wise sampling (a1 + a3 + a6; + a2 for PASS-style).                    */
+/* ------------------------------------------------------------------------ */
+enum {
+  GS_W_UNIFORM = 0,      /* GraphSAGE: uniform without replacement (Floyd, R5)            */
+  GS_W_EDGE = 1,         /* weighted without replacement, A-Res keys on w_e (R6)          */
+  GS_W_PASS_COLNORM = 2  /* as EDGE, plus val_e = w_e / sum(w over column v): PASS A3 (R11) */
+};
+/* individual_sample, layer by layer:
+ *   seeds   device int32[num_seeds], 0 <= id < N (violations are reported by
+ *           gs_blocks_sync as GS_ERR_INDEX_OUT_OF_RANGE; such columns are empty)
+ *   batch_size > 0; batch b holds seeds [b*batch_size, min(num_seeds, (b+1)*batch_size))
+ *   batch_index_base: global index of batch 0 (keys the RNG; shard invariance)
+ *   fanouts host int32[num_layers], 1 <= fanouts[l] <= 32, fanouts[0] applies to
+ *           the seeds (R15); 1 <= num_layers <= 8
+ *   replace 0: without replacement (GraphSAGE); 1: with replacement (KGCN, R10,
+ *           bias_mode must be GS_W_UNIFORM)
+ *   rng_key Philox key; counters (v, slot, layer|tag<<24, global batch) (R4)
+ * Output per (b, l): col_map = frontier (l = 0: the batch's seeds; l > 0: the
+ * previous layer's row_map, R2), edges in column order then ascending position
+ * (slot order with replacement), row_map in first-occurrence order (R3).
+ * Envelope: batch_size * prod(fanouts[0..l]) <= 2^25 for every l. */
+gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                              int64_t batch_size, int64_t batch_index_base,
+                              const int32_t* fanouts, int num_layers, int replace, int bias_mode,
+                              uint64_t rng_key, void* stream, gs_blocks** out);
+
+/* ShaDow (R12): node-wise sampling as gs_sample_neighbors
+ * (bias_mode UNIFORM or EDGE, no replacement), then for every batch the
+ * subgraph of A induced on U = first-occurrence union of the seeds and all
+ * sampled rows.  One block per batch (num_layers == 1 in the result):
+ * col_map == row_map == U, edges u->v with u, v in U in CSC order. */
+gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                           int64_t batch_size, int64_t batch_index_base, const int32_t* fanouts,
+                           int num_layers, int bias_mode, uint64_t rng_key, void* stream,
+                           gs_blocks** out);
+
+/* ------------------------------------------------------------------------ */
+/* Layer-wise sampling (a1 + a2 + a4 + a6): FastGCN / LADIES.                 */
+/* ------------------------------------------------------------------------ */
+enum {
+  GS_PROB_LADIES = 0, /* b(u) = sum over extracted edges of w^2 (Fig. 2)  */
+  GS_PROB_DEGREE = 1, /* b(u) = in-degree of u (FastGCN)                       */
+  GS_PROB_COUNT = 2   /* b(u) = number of extracted edges of u (node_probs omitted)  */
+};
+/* collective_sample: per (batch, layer) with frontier F, C =
+ * unique rows of A[:, F]; S = all u in C with b(u) > 0 if at most K of them,
+ * else the K smallest A-Res keys (R6/R7); S ascending; block = edges of
+ * A[:, F] whose row is in S (CSC order); row_prob p(u) = b(u)/B with
+ * B = sum of b over C; val_e = a_e / sum_column(a), a_e = w_e / p(u)
+ * (Fig. 3(b) lines 5-7).  Next frontier = S.
+ *   n_per_layer host int32[num_layers], 1 <= K <= 4096. */
+gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                              int64_t batch_size, int64_t batch_index_base,
+                              const int32_t* n_per_layer, int num_layers, int prob_mode,
+                              uint64_t rng_key, void* stream, gs_blocks** out);
+
+/* ------------------------------------------------------------------------ */
+/* Random walks (a5): DeepWalk / Node2Vec.                                   */
+/* ------------------------------------------------------------------------ */
+enum { GS_WALK_FORCE_NODE2VEC = 1 }; /* use the Node2Vec sampler even at p == q == 1 */
+/* One walker per start node.  traces: caller-owned device
+ * int32 [num_walkers][length + 1]; traces[i][0] = starts[i]; a walker at a
+ * node with no in-neighbours stops and the rest of its row is -1 (R13).
+ * p == q == 1 (and no FORCE flag): DeepWalk, uniform in-neighbour per step.
+ * Otherwise Node2Vec with bias 1/p (x == prev), 1 (x in column(prev)), 1/q
+ * (else), by rejection sampling (R14); needs a sorted graph
+ * (GS_ERR_UNSORTED_GRAPH otherwise).  walker_index_base keys the RNG by the
+ * global walker index (R4).  p, q > 0; 0 <= length < 2^24. */
+gs_status gs_random_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
+                         int64_t walker_index_base, int length, float p, float q,
+                         uint64_t rng_key, uint32_t flags, void* stream, int32_t* traces);
+/* Device-detected errors of the last gs_random_walk on this thread's graph
+ * (out-of-range starts); synchronises the stream. */
+gs_status gs_walk_check(const gs_graph* g, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GS_H */

@@ -1,0 +1,185 @@
+// common.cuh -- device primitives of the B200 ECSF path: counter-based RNG,
+// integer draws, A-Res keys, per-(batch, layer) hash tables and warp/block scans.
+// Independent of the CPU oracle (oracle/ shares no code with this directory).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace gsb {
+
+// ---------------------------------------------------------------------------
+// Philox4x32-10 (Salmon et al., SC'11).  Counter layout (R4):
+//   c0 = subject (frontier node / candidate node / walker), c1 = slot,
+//   c2 = layer_or_step | tag << 24, c3 = global batch index; key = rng_key.
+// ---------------------------------------------------------------------------
+struct U4 { uint32_t x, y, z, w; };
+
+__device__ __forceinline__ U4 philox(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,
+                                     uint64_t key) {
+  uint32_t k0 = (uint32_t)key, k1 = (uint32_t)(key >> 32);
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+    uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+    uint32_t n0 = hi1 ^ c1 ^ k0, n2 = hi0 ^ c3 ^ k1;
+    c0 = n0; c1 = lo1; c2 = n2; c3 = lo0;
+    k0 += 0x9E3779B9u; k1 += 0xBB67AE85u;  // the 10th bump is never used
+  }
+  return U4{c0, c1, c2, c3};
+}
+
+enum : uint32_t { TAG_FLOYD = 1, TAG_REPLACE = 2, TAG_ARES_NODE = 3, TAG_ARES_LAYER = 4,
+                  TAG_DEEPWALK = 5, TAG_NODE2VEC = 6 };
+
+__device__ __forceinline__ uint32_t ctr2(int layer, uint32_t tag) {
+  return (uint32_t)layer | (tag << 24);
+}
+
+// floor(r * n / 2^64), r = hi:lo (R23).  Exact 64x64 -> high 64 product.
+__device__ __forceinline__ uint64_t draw_below(uint64_t n, uint32_t lo, uint32_t hi) {
+  uint64_t r = ((uint64_t)hi << 32) | lo;
+  return __umul64hi(r, n);
+}
+
+// -ln((r + 0.5) 2^-32) / bias in fp64 (R6).
+__device__ __forceinline__ double ares_key(uint32_t r, double bias) {
+  double u = ((double)r + 0.5) * 0x1p-32;
+  return -log(u) / bias;
+}
+
+// (key, pos) lexicographic order: smaller key wins, ties -> smaller position.
+__device__ __forceinline__ bool key_less(double ka, int64_t pa, double kb, int64_t pb) {
+  return ka < kb || (ka == kb && pa < pb);
+}
+
+// ---------------------------------------------------------------------------
+// Generation-tagged open-addressing table, one per cluster workspace.
+// Entry = gen(8) | key(31) | val(25).  Entries whose gen differs from the
+// current one are empty, so a table is reused without clearing for 255 uses.
+// For a fixed (gen, key) the entry value is the atomicMin of all inserted
+// vals: the first position at which the key occurs (R3, first occurrence).
+// ---------------------------------------------------------------------------
+constexpr int TAB_VAL_BITS = 25;
+constexpr uint64_t TAB_VAL_MASK = (1ull << TAB_VAL_BITS) - 1;
+
+__device__ __forceinline__ uint32_t tab_hash(uint32_t key, int log_cap) {
+  return (key * 0x9E3779B1u) >> (32 - log_cap);
+}
+__device__ __forceinline__ uint64_t tab_entry(uint32_t gen, uint32_t key, uint32_t val) {
+  return ((uint64_t)gen << 56) | ((uint64_t)key << TAB_VAL_BITS) | (uint64_t)val;
+}
+__device__ __forceinline__ uint32_t tab_gen(uint64_t e) { return (uint32_t)(e >> 56); }
+__device__ __forceinline__ uint32_t tab_key(uint64_t e) {
+  return (uint32_t)((e >> TAB_VAL_BITS) & 0x7FFFFFFFu);
+}
+__device__ __forceinline__ uint32_t tab_val(uint64_t e) { return (uint32_t)(e & TAB_VAL_MASK); }
+
+// Insert key with val; keeps the minimum val per key.  Returns the slot.
+__device__ __forceinline__ uint32_t tab_insert_min(unsigned long long* tab, int log_cap,
+                                                   uint32_t gen, uint32_t key, uint32_t val) {
+  const uint32_t mask = (1u << log_cap) - 1;
+  const unsigned long long mine = tab_entry(gen, key, val);
+  uint32_t h = tab_hash(key, log_cap);
+  while (true) {
+    unsigned long long old = *(volatile unsigned long long*)&tab[h];
+    if (tab_gen(old) != gen) {
+      unsigned long long prev = atomicCAS(&tab[h], old, mine);
+      if (prev == old) return h;
+      old = prev;
+      if (tab_gen(old) != gen) continue;  // raced with a stale-entry writer: retry slot
+    }
+    if (tab_key(old) == key) {
+      if ((uint32_t)tab_val(old) > val) atomicMin(&tab[h], mine);
+      return h;
+    }
+    h = (h + 1) & mask;
+  }
+}
+
+// Insert key if absent (value = val); returns slot and whether it was new.
+__device__ __forceinline__ uint32_t tab_insert_once(unsigned long long* tab, int log_cap,
+                                                    uint32_t gen, uint32_t key, uint32_t val,
+                                                    bool* inserted) {
+  const uint32_t mask = (1u << log_cap) - 1;
+  const unsigned long long mine = tab_entry(gen, key, val);
+  uint32_t h = tab_hash(key, log_cap);
+  while (true) {
+    unsigned long long old = *(volatile unsigned long long*)&tab[h];
+    if (tab_gen(old) != gen) {
+      unsigned long long prev = atomicCAS(&tab[h], old, mine);
+      if (prev == old) { *inserted = true; return h; }
+      old = prev;
+      if (tab_gen(old) != gen) continue;
+    }
+    if (tab_key(old) == key) { *inserted = false; return h; }
+    h = (h + 1) & mask;
+  }
+}
+
+// Lookup: slot of key, or -1.  Call only after the inserting phase is fenced.
+__device__ __forceinline__ int64_t tab_find(const unsigned long long* tab, int log_cap,
+                                            uint32_t gen, uint32_t key) {
+  const uint32_t mask = (1u << log_cap) - 1;
+  uint32_t h = tab_hash(key, log_cap);
+  while (true) {
+    unsigned long long e = tab[h];
+    if (tab_gen(e) != gen) return -1;
+    if (tab_key(e) == key) return (int64_t)h;
+    h = (h + 1) & mask;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Scans
+// ---------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_scan(T v) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    T n = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += n;
+  }
+  return v;
+}
+
+// Block-wide exclusive scan; `total` gets the block sum.  scratch: >= 33 T.
+template <typename T>
+__device__ __forceinline__ T block_exclusive_scan(T v, T* scratch, T* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  T inc = warp_inclusive_scan(v);
+  if (lane == 31) scratch[wid] = inc;
+  __syncthreads();
+  if (wid == 0) {
+    T s = lane < nw ? scratch[lane] : T(0);
+    T si = warp_inclusive_scan(s);
+    if (lane < nw) scratch[lane] = si - s;
+    if (lane == nw - 1) scratch[32] = si;
+  }
+  __syncthreads();
+  T ex = inc - v + scratch[wid];
+  *total = scratch[32];
+  __syncthreads();
+  return ex;
+}
+
+template <typename T>
+__device__ __forceinline__ T block_reduce_sum(T v, T* scratch) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if (lane == 0) scratch[wid] = v;
+  __syncthreads();
+  if (wid == 0) {
+    T s = lane < nw ? scratch[lane] : T(0);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) scratch[32] = s;
+  }
+  __syncthreads();
+  T r = scratch[32];
+  __syncthreads();
+  return r;
+}
+
+}  // namespace gsb

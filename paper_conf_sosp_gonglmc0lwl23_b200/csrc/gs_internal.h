@@ -1,0 +1,82 @@
+// gs_internal.h -- host/device shared structures of libgsb200 (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/gs.h"
+
+namespace gsb {
+
+constexpr int MAX_LAYERS = 8;
+constexpr int MAX_FANOUT = 32;
+constexpr int64_t MAX_SLOTS_PER_BATCH = (1ll << 25);  // table value field (R3 positions)
+
+// ---- error reporting (thread-local message) ----
+void set_error(const char* fmt, ...);
+gs_status fail(gs_status st, const char* fmt, ...);
+gs_status cuda_fail(cudaError_t e, const char* what);
+#define GS_CUDA_TRY(expr)                                   \
+  do {                                                      \
+    cudaError_t _e = (expr);                                \
+    if (_e != cudaSuccess) return ::gsb::cuda_fail(_e, #expr); \
+  } while (0)
+
+// ---- allocator hook ----
+struct Allocator {
+  gs_alloc_fn alloc = nullptr;
+  gs_free_fn free_fn = nullptr;
+  void* ctx = nullptr;
+  void* allocate(size_t bytes, cudaStream_t s) const;
+  void release(void* p, size_t bytes, cudaStream_t s) const;
+};
+Allocator current_allocator();
+
+// A growable device buffer owned through an Allocator.
+struct DevBuf {
+  void* ptr = nullptr;
+  size_t bytes = 0;
+  // Ensures capacity >= need; returns false on allocation failure.
+  bool ensure(const Allocator& al, size_t need, cudaStream_t s, bool zero = false);
+  void reset(const Allocator& al, cudaStream_t s);
+};
+
+// Device error word bits (set by kernels, read by gs_blocks_sync).
+enum : int { ERR_SEED_RANGE = 1, ERR_CAPACITY = 2 };
+
+}  // namespace gsb
+
+struct gs_graph {
+  int64_t num_nodes = 0, num_edges = 0;
+  int64_t* indptr = nullptr;
+  int32_t* indices = nullptr;
+  float* weights = nullptr;
+  bool owns = false;
+  int sorted = 0;
+  int64_t max_in_degree = 0;
+  gsb::Allocator al;
+  gsb::DevBuf b_indptr, b_indices, b_weights, b_err;
+  int* d_err = nullptr;  // walk error word
+};
+
+struct gs_blocks {
+  enum Kind { NODEWISE = 0, LAYERWISE = 1, SHADOW = 2 };
+  gsb::Allocator al;
+  cudaStream_t stream = nullptr;
+  int kind = NODEWISE;
+  int64_t num_batches = 0;
+  int num_layers = 0;
+  gs_layer_buffers layers[gsb::MAX_LAYERS] = {};
+  // owned buffers per layer: col_map (layer 0 / layer-wise), row_map, indptr,
+  // row_local, eid, val, row_prob
+  gsb::DevBuf b_col[gsb::MAX_LAYERS], b_row[gsb::MAX_LAYERS], b_indptr[gsb::MAX_LAYERS],
+      b_rowl[gsb::MAX_LAYERS], b_eid[gsb::MAX_LAYERS], b_val[gsb::MAX_LAYERS],
+      b_rprob[gsb::MAX_LAYERS];
+  gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr;
+  std::vector<int64_t> h_meta;
+  int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
+  int64_t ws_stride_prev = -1; // workspace layout of the previous launch
+  bool synced = false;
+};

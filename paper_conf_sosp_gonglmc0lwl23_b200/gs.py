@@ -1,0 +1,335 @@
+"""Thin Python binding of libgsb200.so (include/gs.h): argument marshalling only.
+
+Every step of the sampling path runs in the library's sm_100a kernels; this
+module converts torch tensors to raw pointers, calls the C ABI and wraps the
+returned device buffers as torch tensors.  There is no CPU fallback: importing
+it without the built library raises.  PyTorch provides the device memory (its
+caching allocator is installed as the library's allocator hook) and streams.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgsb200.so")
+
+GS_OK = 0
+STATUS = {0: "GS_OK", 1: "GS_ERR_INVALID_ARGUMENT", 2: "GS_ERR_OUT_OF_MEMORY", 3: "GS_ERR_CUDA",
+          4: "GS_ERR_UNSORTED_GRAPH", 5: "GS_ERR_INDEX_OUT_OF_RANGE", 6: "GS_ERR_NOT_SUPPORTED",
+          7: "GS_ERR_CAPACITY", 8: "GS_ERR_INVALID_GRAPH"}
+UNIFORM, EDGE, PASS_COLNORM = 0, 1, 2
+LADIES, DEGREE, COUNT = 0, 1, 2
+GRAPH_HOST_PTRS, GRAPH_BORROW = 1, 2
+WALK_FORCE_NODE2VEC = 1
+META_FIELDS = 8
+
+# Every symbol include/gs.h declares (checked by tests/test_capi_symbols.py).
+EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
+           "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
+           "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
+           "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_layerwise",
+           "gs_random_walk", "gs_walk_check"]
+
+
+class GSError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _BlockView(ctypes.Structure):
+    _fields_ = [("n_cols", ctypes.c_int64), ("n_rows", ctypes.c_int64), ("n_edges", ctypes.c_int64),
+                ("col_map", ctypes.c_void_p), ("row_map", ctypes.c_void_p),
+                ("indptr", ctypes.c_void_p), ("row_local", ctypes.c_void_p),
+                ("eid", ctypes.c_void_p), ("val", ctypes.c_void_p), ("row_prob", ctypes.c_void_p)]
+
+
+class _GraphInfo(ctypes.Structure):
+    _fields_ = [("num_nodes", ctypes.c_int64), ("num_edges", ctypes.c_int64),
+                ("weighted", ctypes.c_int), ("sorted", ctypes.c_int),
+                ("max_in_degree", ctypes.c_int64), ("indptr", ctypes.c_void_p),
+                ("indices", ctypes.c_void_p), ("weights", ctypes.c_void_p)]
+
+
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_lib = None
+_hooks = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Loads the C ABI (raises if the CUDA library has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = ctypes.CDLL(path)
+    vp, i64, i32, u64, u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_uint64, ctypes.c_uint32
+    L.gs_last_error.restype = ctypes.c_char_p
+    L.gs_status_string.restype = ctypes.c_char_p
+    L.gs_status_string.argtypes = [i32]
+    L.gs_set_allocator.argtypes = [_ALLOC_FN, _FREE_FN, vp]
+    L.gs_graph_create.argtypes = [vp, vp, vp, i64, i64, u32, vp, ctypes.POINTER(vp)]
+    L.gs_graph_get_info.argtypes = [vp, ctypes.POINTER(_GraphInfo)]
+    L.gs_graph_destroy.argtypes = [vp]
+    L.gs_graph_destroy.restype = None
+    L.gs_sample_neighbors.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, u64, vp,
+                                      ctypes.POINTER(vp)]
+    L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
+    L.gs_sample_layerwise.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp,
+                                      ctypes.POINTER(vp)]
+    L.gs_random_walk.argtypes = [vp, vp, i64, i64, i32, ctypes.c_float, ctypes.c_float, u64, u32,
+                                 vp, vp]
+    L.gs_walk_check.argtypes = [vp, vp]
+    L.gs_blocks_sync.argtypes = [vp]
+    L.gs_blocks_shape.argtypes = [vp, ctypes.POINTER(i64), ctypes.POINTER(i32)]
+    L.gs_blocks_view.argtypes = [vp, i64, i32, ctypes.POINTER(_BlockView)]
+    L.gs_blocks_device_meta.argtypes = [vp, ctypes.POINTER(vp)]
+    L.gs_blocks_destroy.argtypes = [vp]
+    L.gs_blocks_destroy.restype = None
+    _lib = L
+    return L
+
+
+def _check(st, where=""):
+    if st != GS_OK:
+        msg = _lib.gs_last_error().decode(errors="replace")
+        raise GSError(st, f"{where}: {msg}" if where else msg)
+
+
+def use_torch_allocator():
+    """Routes every library-owned device allocation through PyTorch's caching allocator."""
+    global _hooks
+    L = load_library()
+
+    def _alloc(nbytes, stream, ctx):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), torch.cuda.current_device(),
+                                                      stream or 0)
+        except Exception:  # reported to C as NULL -> GS_ERR_OUT_OF_MEMORY
+            return None
+
+    def _free(ptr, nbytes, stream, ctx):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    _hooks = (_ALLOC_FN(_alloc), _FREE_FN(_free))
+    _check(L.gs_set_allocator(_hooks[0], _hooks[1], None), "gs_set_allocator")
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+class _CudaArray:
+    """__cuda_array_interface__ wrapper so torch can view library-owned memory."""
+
+    def __init__(self, ptr, n, typestr, owner):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": typestr,
+                                         "data": (int(ptr or 0), False), "version": 3,
+                                         "strides": None}
+        self._owner = owner
+
+
+def _dev_tensor(ptr, n, dtype, owner):
+    if n == 0 or not ptr:
+        return torch.empty(0, dtype=dtype, device="cuda")
+    ts = {torch.int32: "<i4", torch.int64: "<i8", torch.float32: "<f4"}[dtype]
+    return torch.as_tensor(_CudaArray(ptr, n, ts, owner), device="cuda")
+
+
+class Graph:
+    """gs_graph: validated CSC in HBM (a0)."""
+
+    def __init__(self, indptr: torch.Tensor, indices: torch.Tensor, weights=None, borrow=False,
+                 stream=None):
+        L = load_library()
+        indptr = indptr.to(torch.int64).contiguous()
+        indices = indices.to(torch.int32).contiguous()
+        if weights is not None:
+            weights = weights.to(torch.float32).contiguous()
+        flags = 0
+        if indptr.device.type == "cpu":
+            flags |= GRAPH_HOST_PTRS
+        elif borrow:
+            flags |= GRAPH_BORROW
+            self._keep = (indptr, indices, weights)
+        h = ctypes.c_void_p()
+        _check(L.gs_graph_create(_ptr(indptr), _ptr(indices), _ptr(weights), indptr.numel() - 1,
+                                 indices.numel(), flags, _stream_ptr(stream), ctypes.byref(h)),
+               "gs_graph_create")
+        self._h = h
+        info = _GraphInfo()
+        _check(L.gs_graph_get_info(h, ctypes.byref(info)))
+        self.num_nodes = info.num_nodes
+        self.num_edges = info.num_edges
+        self.weighted = bool(info.weighted)
+        self.sorted = bool(info.sorted)
+        self.max_in_degree = info.max_in_degree
+
+    @property
+    def handle(self):
+        return self._h
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.gs_graph_destroy(self._h)
+            self._h = None
+
+
+class Blocks:
+    """gs_blocks: per-(batch, layer) sampled blocks in HBM."""
+
+    def __init__(self):
+        self._h = ctypes.c_void_p()
+        self.synced = False
+
+    def sync(self):
+        _check(_lib.gs_blocks_sync(self._h), "gs_blocks_sync")
+        nb, nl = ctypes.c_int64(), ctypes.c_int()
+        _check(_lib.gs_blocks_shape(self._h, ctypes.byref(nb), ctypes.byref(nl)))
+        self.num_batches, self.num_layers = nb.value, nl.value
+        self.synced = True
+        return self
+
+    def view(self, batch: int, layer: int) -> dict:
+        if not self.synced:
+            self.sync()
+        v = _BlockView()
+        _check(_lib.gs_blocks_view(self._h, batch, layer, ctypes.byref(v)), "gs_blocks_view")
+        o = self
+        return {
+            "col_map": _dev_tensor(v.col_map, v.n_cols, torch.int32, o),
+            "row_map": _dev_tensor(v.row_map, v.n_rows, torch.int32, o),
+            "indptr": _dev_tensor(v.indptr, v.n_cols + 1, torch.int64, o),
+            "row_local": _dev_tensor(v.row_local, v.n_edges, torch.int32, o),
+            "eid": _dev_tensor(v.eid, v.n_edges, torch.int64, o),
+            "val": None if not v.val else _dev_tensor(v.val, v.n_edges, torch.float32, o),
+            "row_prob": None if not v.row_prob else _dev_tensor(v.row_prob, v.n_rows, torch.float32, o),
+        }
+
+    def device_meta(self) -> torch.Tensor:
+        """int64 [num_batches, num_layers, 8] on the device (no sync)."""
+        p = ctypes.c_void_p()
+        _check(_lib.gs_blocks_device_meta(self._h, ctypes.byref(p)))
+        nb, nl = ctypes.c_int64(), ctypes.c_int()
+        _check(_lib.gs_blocks_shape(self._h, ctypes.byref(nb), ctypes.byref(nl)))
+        t = _dev_tensor(p.value, nb.value * nl.value * META_FIELDS, torch.int64, self)
+        return t.view(nb.value, nl.value, META_FIELDS)
+
+    def to_host(self) -> list:
+        """blocks[batch][layer] -> dict of numpy arrays (tests / e2e)."""
+        if not self.synced:
+            self.sync()
+        out = []
+        for b in range(self.num_batches):
+            layers = []
+            for l in range(self.num_layers):
+                v = self.view(b, l)
+                layers.append({k: (None if x is None else x.cpu().numpy()) for k, x in v.items()})
+            out.append(layers)
+        return out
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.gs_blocks_destroy(self._h)
+            self._h = None
+
+
+def _host_i32(xs):
+    arr = (ctypes.c_int * len(xs))(*[int(x) for x in xs])
+    return arr
+
+
+def sample_neighbors(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch_index_base=0,
+                     replace=False, bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None):
+    """GraphSAGE / KGCN / weighted A-Res / PASS-style node-wise sampling (gs_sample_neighbors)."""
+    L = load_library()
+    seeds = seeds.to(torch.int32).contiguous()
+    bs = int(batch_size or max(1, seeds.numel()))
+    out = out or Blocks()
+    f = _host_i32(fanouts)
+    _check(L.gs_sample_neighbors(g.handle, _ptr(seeds), seeds.numel(), bs, int(batch_index_base),
+                                 f, len(fanouts), int(replace), int(bias_mode),
+                                 ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                                 ctypes.byref(out._h)), "gs_sample_neighbors")
+    out.synced = False
+    out._seeds = seeds
+    return out
+
+
+def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch_index_base=0,
+                  bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None, retry=True):
+    L = load_library()
+    seeds = seeds.to(torch.int32).contiguous()
+    bs = int(batch_size or max(1, seeds.numel()))
+    out = out or Blocks()
+    f = _host_i32(fanouts)
+    for attempt in range(3):
+        _check(L.gs_sample_shadow(g.handle, _ptr(seeds), seeds.numel(), bs, int(batch_index_base),
+                                  f, len(fanouts), int(bias_mode), ctypes.c_uint64(rng_key),
+                                  _stream_ptr(stream), ctypes.byref(out._h)), "gs_sample_shadow")
+        out.synced = False
+        if not retry:
+            break
+        try:
+            out.sync()
+            break
+        except GSError as e:
+            if e.status != 7 or attempt == 2:
+                raise
+    out._seeds = seeds
+    return out
+
+
+def sample_layerwise(g: Graph, seeds: torch.Tensor, n_per_layer, batch_size=None,
+                     batch_index_base=0, prob_mode=LADIES, rng_key=0, stream=None,
+                     out: Blocks = None, retry=True):
+    L = load_library()
+    seeds = seeds.to(torch.int32).contiguous()
+    bs = int(batch_size or max(1, seeds.numel()))
+    out = out or Blocks()
+    f = _host_i32(n_per_layer)
+    for attempt in range(3):
+        _check(L.gs_sample_layerwise(g.handle, _ptr(seeds), seeds.numel(), bs,
+                                     int(batch_index_base), f, len(n_per_layer), int(prob_mode),
+                                     ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                                     ctypes.byref(out._h)), "gs_sample_layerwise")
+        out.synced = False
+        if not retry:
+            break
+        try:
+            out.sync()
+            break
+        except GSError as e:
+            if e.status != 7 or attempt == 2:
+                raise
+    out._seeds = seeds
+    return out
+
+
+def random_walk(g: Graph, starts: torch.Tensor, length: int, p=1.0, q=1.0, walker_index_base=0,
+                rng_key=0, force_node2vec=False, stream=None, out: torch.Tensor = None):
+    """DeepWalk / Node2Vec; returns int32 traces [num_walkers, length + 1] on the device."""
+    L = load_library()
+    starts = starts.to(torch.int32).contiguous()
+    if out is None:
+        out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)
+    _check(L.gs_random_walk(g.handle, _ptr(starts), starts.numel(), int(walker_index_base),
+                            int(length), float(p), float(q), ctypes.c_uint64(rng_key),
+                            WALK_FORCE_NODE2VEC if force_node2vec else 0, _stream_ptr(stream),
+                            _ptr(out)), "gs_random_walk")
+    return out
+
+
+def walk_check(g: Graph, stream=None):
+    _check(load_library().gs_walk_check(g.handle, _stream_ptr(stream)), "gs_walk_check")
