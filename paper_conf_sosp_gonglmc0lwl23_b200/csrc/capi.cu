@@ -379,15 +379,23 @@ gs_status gs_blocks_sync(gs_blocks* b) {
     GS_CUDA_TRY(cudaMemcpy(b->h_meta.data(), b->b_meta.ptr, b->h_meta.size() * 8,
                            cudaMemcpyDeviceToHost));
   int err[4] = {0};
-  unsigned long long ctr = 0;
+  unsigned long long ctr[MAX_LAYERS + 2] = {0};
   GS_CUDA_TRY(cudaMemcpy(err, b->b_err.ptr, 16, cudaMemcpyDeviceToHost));
-  GS_CUDA_TRY(cudaMemcpy(&ctr, b->b_ctr.ptr, 8, cudaMemcpyDeviceToHost));
+  GS_CUDA_TRY(cudaMemcpy(ctr, b->b_ctr.ptr, std::min<size_t>(sizeof(ctr), b->b_ctr.bytes),
+                         cudaMemcpyDeviceToHost));
   b->synced = true;
+  if (err[0] & ERR_INTERNAL) return fail(GS_ERR_CUDA, "internal consistency check failed in a sampling kernel");
   if (err[0] & ERR_SEED_RANGE) return fail(GS_ERR_INDEX_OUT_OF_RANGE, "a seed id is outside [0, N)");
   if (err[0] & ERR_CAPACITY) {
-    b->sh_edge_hint = (int64_t)(ctr + ctr / 4 + 1024);
-    return fail(GS_ERR_CAPACITY, "edge capacity exceeded (needed %llu); call again with this gs_blocks to grow",
-                (unsigned long long)ctr);
+    if (b->kind == gs_blocks::SHADOW) {
+      b->sh_edge_hint = (int64_t)(ctr[0] + ctr[0] / 4 + 1024);
+    } else {
+      for (int l = 0; l < b->num_layers; ++l)
+        b->lw_edge_hint[l] = std::max<int64_t>(b->lw_edge_hint[l], (int64_t)(ctr[l] + ctr[l] / 4 + 1024));
+      b->lw_tab_hint = std::max<int64_t>(b->lw_tab_hint, (int64_t)ctr[MAX_LAYERS]);
+    }
+    return fail(GS_ERR_CAPACITY,
+                "a device-side capacity was exceeded; call again with this gs_blocks (it has grown)");
   }
   return GS_OK;
 }

@@ -81,7 +81,7 @@ __device__ __forceinline__ uint32_t tab_insert_min(unsigned long long* tab, int 
   const unsigned long long mine = tab_entry(gen, key, val);
   uint32_t h = tab_hash(key, log_cap);
   while (true) {
-    unsigned long long old = *(volatile unsigned long long*)&tab[h];
+    unsigned long long old = __ldcg(&tab[h]);
     if (tab_gen(old) != gen) {
       unsigned long long prev = atomicCAS(&tab[h], old, mine);
       if (prev == old) return h;
@@ -104,7 +104,7 @@ __device__ __forceinline__ uint32_t tab_insert_once(unsigned long long* tab, int
   const unsigned long long mine = tab_entry(gen, key, val);
   uint32_t h = tab_hash(key, log_cap);
   while (true) {
-    unsigned long long old = *(volatile unsigned long long*)&tab[h];
+    unsigned long long old = __ldcg(&tab[h]);
     if (tab_gen(old) != gen) {
       unsigned long long prev = atomicCAS(&tab[h], old, mine);
       if (prev == old) { *inserted = true; return h; }
@@ -117,12 +117,13 @@ __device__ __forceinline__ uint32_t tab_insert_once(unsigned long long* tab, int
 }
 
 // Lookup: slot of key, or -1.  Call only after the inserting phase is fenced.
+// Loads bypass L1 (ld.global.cg): L1 is not coherent with other SMs' atomics.
 __device__ __forceinline__ int64_t tab_find(const unsigned long long* tab, int log_cap,
                                             uint32_t gen, uint32_t key) {
   const uint32_t mask = (1u << log_cap) - 1;
   uint32_t h = tab_hash(key, log_cap);
   while (true) {
-    unsigned long long e = tab[h];
+    unsigned long long e = __ldcg(&tab[h]);
     if (tab_gen(e) != gen) return -1;
     if (tab_key(e) == key) return (int64_t)h;
     h = (h + 1) & mask;

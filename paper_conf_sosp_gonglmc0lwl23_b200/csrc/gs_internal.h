@@ -44,7 +44,7 @@ struct DevBuf {
 };
 
 // Device error word bits (set by kernels, read by gs_blocks_sync).
-enum : int { ERR_SEED_RANGE = 1, ERR_CAPACITY = 2 };
+enum : int { ERR_SEED_RANGE = 1, ERR_CAPACITY = 2, ERR_INTERNAL = 4 };
 
 }  // namespace gsb
 
@@ -78,5 +78,7 @@ struct gs_blocks {
   std::vector<int64_t> h_meta;
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch
+  int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
+  int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;
 };

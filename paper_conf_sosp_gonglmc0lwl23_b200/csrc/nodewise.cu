@@ -171,7 +171,7 @@ __device__ void nw_select(const NWParams& P, Ws& W, int l, int log_cap, uint32_t
         }
         if (need) {
           pos = x;
-          slot = rnk;
+          slot = s < k ? rnk : k;  // lanes beyond k (G > k) hold nothing
         }
       }
     } else {
@@ -332,7 +332,7 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
     const uint32_t u = zval(z);
     const int64_t h = tab_find(W.tab, log_cap, gen, u);
     if (tab_val(__ldcg(W.tab + h)) == (uint32_t)z) {
-      const int64_t lid = s_base_r[crank] + W.lid[z];
+      const int64_t lid = s_base_r[crank] + __ldcg(W.lid + z);
       P.sh_nodes[ubase + lid] = (int32_t)u;
       W.tab[h] = tab_entry(gen, u, (uint32_t)lid);
     }
@@ -351,16 +351,16 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
       cnt += tab_find(W.tab, log_cap, gen, u) >= 0 ? 1 : 0;
     }
     cnt = __reduce_add_sync(0xffffffffu, (unsigned)cnt);
-    if (lane == 0) W.cnt[c - u0] = cnt;
+    if (lane == 0) W.cnt[c] = cnt;
   }
   __syncthreads();
   carry = 0;
   for (int64_t ct = u0; ct < u1; ct += blockDim.x) {
     const int64_t c = ct + threadIdx.x;
-    const unsigned long long cv = c < u1 ? (unsigned long long)W.cnt[c - u0] : 0ull;
+    const unsigned long long cv = c < u1 ? (unsigned long long)__ldcg(W.cnt + c) : 0ull;
     unsigned long long tot;
     const unsigned long long ex = block_exclusive_scan(cv, s_scan, &tot) + carry;
-    if (c < u1) W.eoff[c - u0] = (int32_t)ex;
+    if (c < u1) W.eoff[c] = (int32_t)ex;
     carry += tot;
   }
   if (threadIdx.x == 0) *s_tot = carry;
@@ -385,7 +385,7 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
   for (int64_t c = u0 + warp; c < u1; c += nwarps) {
     const int32_t v = __ldcg(P.sh_nodes + ubase + c);
     const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
-    int64_t e = s_base_e[crank] + W.eoff[c - u0];
+    int64_t e = s_base_e[crank] + __ldcg(W.eoff + c);
     if (lane == 0) P.sh_indptr[uibase + c] = e;
     if (!fits) continue;
     for (int64_t i0 = 0; i0 < d; i0 += 32) {
@@ -482,9 +482,10 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
           s = (int)(p - j * k);
           valid = s < __ldcg(W.cnt + j);
           if (valid) {
-            const uint32_t u = (uint32_t)W.u[p];
+            const uint32_t u = (uint32_t)__ldcg(W.u + p);
             const int64_t h = tab_find(W.tab, log_cap, gen, u);
-            const uint32_t p0 = tab_val(__ldcg(W.tab + h));
+            if (h < 0) atomicOr(P.err, ERR_INTERNAL);
+            const uint32_t p0 = h < 0 ? 0xffffffffu : tab_val(__ldcg(W.tab + h));
             W.p0[p] = (int32_t)p0;
             first = (p0 == (uint32_t)p);
           }
@@ -529,24 +530,24 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
         const int64_t j = p / k;
         const int s = (int)(p - j * k);
         if (s == 0) {
-          if (indptr_out) indptr_out[ibase + j] = baseE + W.eoff[j];
+          if (indptr_out) indptr_out[ibase + j] = baseE + __ldcg(W.eoff + j);
           if (l == 0 && P.col0) P.col0[bstart + j] = F[j];
         }
-        if (s >= W.cnt[j]) continue;
-        const int32_t p0 = W.p0[p];
+        if (s >= __ldcg(W.cnt + j)) continue;
+        const int32_t p0 = __ldcg(W.p0 + p);
         int64_t lid;
         if (p0 == (int32_t)p) {
-          lid = baseR + W.lid[p];
-          row_map[rbase + lid] = W.u[p];
+          lid = baseR + __ldcg(W.lid + p);
+          row_map[rbase + lid] = __ldcg(W.u + p);
         } else {
           const int64_t j0 = p0 / k;
           const int r0 = (int)(j0 / chunk);
           lid = s_base_r[r0] + __ldcg(W.lid + p0);
         }
-        const int64_t e = rbase + baseE + W.eidx[p];
+        const int64_t e = rbase + baseE + __ldcg(W.eidx + p);
         if (row_local) row_local[e] = (int32_t)lid;
-        if (eid_out) eid_out[e] = W.e[p];
-        if (val_out) val_out[e] = W.val[p];
+        if (eid_out) eid_out[e] = __ldcg(W.e + p);
+        if (val_out) val_out[e] = __ldcg(W.val + p);
       }
       if (crank == 0 && threadIdx.x == 0) {
         if (indptr_out) indptr_out[ibase + T] = totE;

@@ -8,8 +8,10 @@ caching allocator is installed as the library's allocator hook) and streams.
 """
 from __future__ import annotations
 
+import atexit
 import ctypes
 import os
+import sys
 
 import torch
 
@@ -58,6 +60,30 @@ _ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, 
 _FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 _lib = None
 _hooks = None
+_exiting = False
+
+
+@atexit.register
+def _at_exit():
+    # objects still alive at interpreter exit are leaked on purpose: the CUDA
+    # context and PyTorch's allocator may already be torn down.
+    global _exiting
+    _exiting = True
+
+
+def _alive():
+    return _lib is not None and not _exiting and not sys.is_finalizing()
+
+
+# Handles released by the garbage collector are destroyed at the next API call
+# (never from inside __del__: a GC pass can run while PyTorch's allocator is busy).
+_pending = []
+
+
+def _drain():
+    while _pending and _alive():
+        kind, h = _pending.pop()
+        (_lib.gs_blocks_destroy if kind == "b" else _lib.gs_graph_destroy)(h)
 
 
 def load_library(path: str = LIB_PATH):
@@ -105,6 +131,8 @@ def use_torch_allocator():
     """Routes every library-owned device allocation through PyTorch's caching allocator."""
     global _hooks
     L = load_library()
+    if _hooks is not None:  # idempotent: objects keep pointers to these thunks forever
+        return
 
     def _alloc(nbytes, stream, ctx):
         try:
@@ -153,6 +181,7 @@ class Graph:
     def __init__(self, indptr: torch.Tensor, indices: torch.Tensor, weights=None, borrow=False,
                  stream=None):
         L = load_library()
+        _drain()
         indptr = indptr.to(torch.int64).contiguous()
         indices = indices.to(torch.int32).contiguous()
         if weights is not None:
@@ -181,8 +210,8 @@ class Graph:
         return self._h
 
     def __del__(self):
-        if getattr(self, "_h", None) and _lib is not None:
-            _lib.gs_graph_destroy(self._h)
+        if getattr(self, "_h", None) and _alive():
+            _pending.append(("g", self._h))
             self._h = None
 
 
@@ -240,8 +269,8 @@ class Blocks:
         return out
 
     def __del__(self):
-        if getattr(self, "_h", None) and self._h.value and _lib is not None:
-            _lib.gs_blocks_destroy(self._h)
+        if getattr(self, "_h", None) and self._h.value and _alive():
+            _pending.append(("b", self._h))
             self._h = None
 
 
@@ -254,6 +283,7 @@ def sample_neighbors(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, ba
                      replace=False, bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None):
     """GraphSAGE / KGCN / weighted A-Res / PASS-style node-wise sampling (gs_sample_neighbors)."""
     L = load_library()
+    _drain()
     seeds = seeds.to(torch.int32).contiguous()
     bs = int(batch_size or max(1, seeds.numel()))
     out = out or Blocks()
@@ -270,6 +300,7 @@ def sample_neighbors(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, ba
 def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch_index_base=0,
                   bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None, retry=True):
     L = load_library()
+    _drain()
     seeds = seeds.to(torch.int32).contiguous()
     bs = int(batch_size or max(1, seeds.numel()))
     out = out or Blocks()
@@ -295,6 +326,7 @@ def sample_layerwise(g: Graph, seeds: torch.Tensor, n_per_layer, batch_size=None
                      batch_index_base=0, prob_mode=LADIES, rng_key=0, stream=None,
                      out: Blocks = None, retry=True):
     L = load_library()
+    _drain()
     seeds = seeds.to(torch.int32).contiguous()
     bs = int(batch_size or max(1, seeds.numel()))
     out = out or Blocks()
@@ -321,6 +353,7 @@ def random_walk(g: Graph, starts: torch.Tensor, length: int, p=1.0, q=1.0, walke
                 rng_key=0, force_node2vec=False, stream=None, out: torch.Tensor = None):
     """DeepWalk / Node2Vec; returns int32 traces [num_walkers, length + 1] on the device."""
     L = load_library()
+    _drain()
     starts = starts.to(torch.int32).contiguous()
     if out is None:
         out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)

@@ -1,0 +1,83 @@
+"""GPU parity: layer-wise path (LADIES / FastGCN / COUNT) vs the oracle.
+Integers (row_map = S, indptr, row_local, eid) bit-exact; val and row_prob
+within 1e-5 relative (north_star)."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from tests.graphs_small import B, E, fig1_graph
+from tests.parity import compare_all, host_graph
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def gs():
+    from paper_conf_sosp_gonglmc0lwl23_b200 import gs as _gs
+    _gs.load_library()
+    _gs.use_torch_allocator()
+    return _gs
+
+
+@pytest.fixture(scope="module")
+def ljlike(gs, oracle_lib):
+    # LiveJournal-shaped (directed, GCN-normalised weights) at reduced size
+    g = synth.small_graph(300_000, 4_300_000, undirected=False, weights="gcn", seed=17,
+                          device="cuda")
+    return g, gs.Graph(g["indptr"], g["indices"], g["weights"]), oracle_lib.Graph(*host_graph(g))
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
+def test_layerwise_parity(gs, oracle_lib, ljlike, mode):
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 8), 4000)
+    out = gs.sample_layerwise(G, seeds.cuda(), [512, 512, 512], batch_size=512, prob_mode=mode,
+                              rng_key=33, batch_index_base=2).to_host()
+    ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [512, 512, 512], batch_size=512,
+                                      prob_mode=mode, rng_key=33, batch_index_base=2)
+    compare_all(out, ref, f"layerwise mode {mode}")
+
+
+@pytest.mark.parametrize("K", [1, 7, 64, 4096])
+def test_layerwise_K(gs, oracle_lib, ljlike, K):
+    g, G, O = ljlike
+    seeds = torch.arange(0, 300_000, 997, dtype=torch.int32)
+    out = gs.sample_layerwise(G, seeds.cuda(), [K, K], batch_size=100, prob_mode=0,
+                              rng_key=4).to_host()
+    ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [K, K], batch_size=100, prob_mode=0,
+                                      rng_key=4)
+    compare_all(out, ref, f"layerwise K={K}")
+
+
+def test_fig1_toy(gs, oracle_lib):
+    ip, ix, w = fig1_graph()
+    G = gs.Graph(torch.from_numpy(ip).cuda(), torch.from_numpy(ix).cuda(), torch.from_numpy(w).cuda())
+    O = oracle_lib.Graph(ip, ix, w)
+    seeds = np.array([B, E] * 50, np.int32)
+    for K in [2, 4, 5]:
+        out = gs.sample_layerwise(G, torch.from_numpy(seeds).cuda(), [K], batch_size=2,
+                                  rng_key=K).to_host()
+        ref = oracle_lib.sample_layerwise(O, seeds, [K], batch_size=2, rng_key=K)
+        compare_all(out, ref, f"fig1 K={K}")
+        if K == 5:  # B_f = 0.58; p(f) = 0.58 / 2.08
+            assert out[0][0]["row_prob"][2] == pytest.approx(0.58 / 2.08, rel=1e-6)
+
+
+def test_unit_weights_count_identity(gs, ljlike):
+    g, G, O = ljlike
+    G1 = gs.Graph(g["indptr"], g["indices"], torch.ones_like(g["weights"]))
+    seeds = torch.arange(0, 300_000, 211, dtype=torch.int32, device="cuda")
+    a = gs.sample_layerwise(G1, seeds, [256, 256], batch_size=300, prob_mode=0, rng_key=5).to_host()
+    b = gs.sample_layerwise(G1, seeds, [256, 256], batch_size=300, prob_mode=2, rng_key=5).to_host()
+    compare_all(a, b, "ladies(w=1) == count")
+
+
+def test_capacity_retry(gs, oracle_lib, ljlike):
+    """A tiny initial edge capacity overflows; the binding grows it and re-runs."""
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 9), 2048)
+    out = gs.sample_layerwise(G, seeds.cuda(), [2048], batch_size=2048, prob_mode=1, rng_key=1)
+    ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [2048], batch_size=2048, prob_mode=1,
+                                      rng_key=1)
+    compare_all(out.to_host(), ref, "fastgcn big")
