@@ -131,29 +131,15 @@ def dist_env():
 
 
 def make_graph_dist(name, world, rank, device):
-    """Rank 0 generates the graph; NCCL broadcasts it to the other ranks."""
+    """Rank 0 generates the graph; NCCL broadcasts it to the other ranks (load time)."""
     import synth
+    from paper_conf_sosp_gonglmc0lwl23_b200 import dist as gdist
     spec = synth.CONFIGS[name]
     if world == 1:
         return synth.make_graph(spec, device=device)
-    import torch.distributed as dist
-    if rank == 0:
-        g = synth.make_graph(spec, device=device)
-        sizes = torch.tensor([g["indptr"].numel(), g["indices"].numel(),
-                              0 if g["weights"] is None else g["weights"].numel()],
-                             dtype=torch.int64, device=device)
-    else:
-        sizes = torch.zeros(3, dtype=torch.int64, device=device)
-    dist.broadcast(sizes, 0)
-    if rank != 0:
-        g = {"indptr": torch.empty(int(sizes[0]), dtype=torch.int64, device=device),
-             "indices": torch.empty(int(sizes[1]), dtype=torch.int32, device=device),
-             "weights": None if int(sizes[2]) == 0 else
-             torch.empty(int(sizes[2]), dtype=torch.float32, device=device), "spec": spec}
-    dist.broadcast(g["indptr"], 0)
-    dist.broadcast(g["indices"], 0)
-    if g["weights"] is not None:
-        dist.broadcast(g["weights"], 0)
+    g = synth.make_graph(spec, device=device) if rank == 0 else None
+    g = gdist.broadcast_graph(g, device)
+    g["spec"] = spec
     return g
 
 
@@ -292,6 +278,7 @@ def run_reference(args, wl):
 # ---------------------------------------------------------------------------
 def run_nodewise(args, wl, world, rank, device):
     import synth
+    from paper_conf_sosp_gonglmc0lwl23_b200 import dist as gdist
     from paper_conf_sosp_gonglmc0lwl23_b200 import gs
     import torch.distributed as dist
     gs.use_torch_allocator()
@@ -309,7 +296,7 @@ def run_nodewise(args, wl, world, rank, device):
     base_key = 0x5EED
 
     def step(i, blocks):
-        return gs.sample_neighbors(G, seeds, fan, batch_size=bs, batch_index_base=rank * nb,
+        return gs.sample_neighbors(G, seeds, fan, batch_size=bs, batch_index_base=gdist.weak_batch_base(rank, nb),
                                    replace=wl["replace"], bias_mode=wl["bias"],
                                    rng_key=base_key + 7919 * i, stream=stream, out=blocks)
 
@@ -354,7 +341,7 @@ def run_nodewise(args, wl, world, rank, device):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         dev_seeds.copy_(host_seeds, non_blocking=True)
-        gs.sample_neighbors(G, dev_seeds, fan, batch_size=bs, batch_index_base=rank * nb,
+        gs.sample_neighbors(G, dev_seeds, fan, batch_size=bs, batch_index_base=gdist.weak_batch_base(rank, nb),
                             replace=wl["replace"], bias_mode=wl["bias"], rng_key=base_key + i,
                             stream=stream, out=out)
         meta_h.copy_(out.device_meta(), non_blocking=True)

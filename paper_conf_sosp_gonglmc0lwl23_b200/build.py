@@ -13,8 +13,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libgsb200.so")
-SOURCES = ["capi.cu", "nodewise.cu", "layerwise.cu", "walk.cu"]
-HEADERS = ["common.cuh", "gs_internal.h"]
+SOURCES = ["capi.cu", "nodewise.cu", "nodewise_pq.cu", "layerwise.cu", "walk.cu"]
+HEADERS = ["common.cuh", "gs_internal.h", "nodewise_common.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-fmad=false",
          "-std=c++17", "-Xcompiler", "-fPIC", "-I", os.path.join(ROOT, "include")]

@@ -131,6 +131,53 @@ __device__ __forceinline__ int64_t tab_find(const unsigned long long* tab, int l
 }
 
 // ---------------------------------------------------------------------------
+// Ordered open-addressing table (node-wise kernel).  Entry =
+// tag(8) | key(31) | val(25) with tag = 255 - gen: entries of older
+// generations (and the cleared value ~0) compare LARGER than every entry of
+// the current generation, so one atomicMin both claims a stale slot and, for
+// an equal key, keeps the minimum val (the first occurrence, R3).  When the
+// atomicMin displaces a larger entry of another key, the displaced entry is
+// carried on and re-inserted further along the probe sequence (ordered linear
+// probing): no load-then-CAS round trip, one atomic per probe step.  Lookups
+// scan from the hash until the key or a stale slot.  Between clears the
+// generation must increase; a table is cleared to ~0 every 255 uses.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t otag(uint32_t gen) { return 255u - gen; }
+
+// Continues an insertion whose first atomicMin at slot h returned `old`.
+__device__ __forceinline__ void otab_finish(unsigned long long* tab, uint32_t mask, uint32_t tag,
+                                            uint32_t h, unsigned long long carry,
+                                            unsigned long long old) {
+  while (true) {
+    if (tab_gen(old) != tag) return;               // stale slot: carry placed
+    if (tab_key(old) == tab_key(carry)) return;    // same key: min kept
+    if (old > carry) carry = old;                  // displaced: carry it on
+    h = (h + 1) & mask;
+    old = atomicMin(&tab[h], carry);
+  }
+}
+
+__device__ __forceinline__ void otab_insert_min(unsigned long long* tab, int log_cap, uint32_t tag,
+                                                uint32_t key, uint32_t val) {
+  const unsigned long long e = tab_entry(tag, key, val);
+  const uint32_t h = tab_hash(key, log_cap);
+  otab_finish(tab, (1u << log_cap) - 1u, tag, h, e, atomicMin(&tab[h], e));
+}
+
+// Slot of key (current generation) or -1.
+__device__ __forceinline__ int64_t otab_find(const unsigned long long* tab, int log_cap,
+                                             uint32_t tag, uint32_t key) {
+  const uint32_t mask = (1u << log_cap) - 1u;
+  uint32_t h = tab_hash(key, log_cap);
+  while (true) {
+    const unsigned long long e = __ldcg(&tab[h]);
+    if (tab_gen(e) != tag) return -1;
+    if (tab_key(e) == key) return (int64_t)h;
+    h = (h + 1) & mask;
+  }
+}
+
+// ---------------------------------------------------------------------------
 // Scans
 // ---------------------------------------------------------------------------
 template <typename T>

@@ -74,10 +74,11 @@ struct gs_blocks {
   gsb::DevBuf b_col[gsb::MAX_LAYERS], b_row[gsb::MAX_LAYERS], b_indptr[gsb::MAX_LAYERS],
       b_rowl[gsb::MAX_LAYERS], b_eid[gsb::MAX_LAYERS], b_val[gsb::MAX_LAYERS],
       b_rprob[gsb::MAX_LAYERS];
-  gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr;
+  gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr, b_sched;
   std::vector<int64_t> h_meta;
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch
+  int ws_kind_prev = 0;        // 1 node-wise (tables cleared to ~0), 2 layer-wise (cleared to 0)
   int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;

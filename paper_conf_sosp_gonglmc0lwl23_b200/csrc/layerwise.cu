@@ -487,11 +487,12 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
   const bool grow = blk->b_ws.bytes < ws_bytes;
   if (!blk->b_ws.ensure(al, ws_bytes, stream, true) || !blk->b_gen.ensure(al, 4096 * 4, stream, true))
     return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (layer-wise workspace)");
-  if (grow || blk->ws_stride_prev != P.ws_stride) {
-    if (!grow) GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, blk->b_ws.bytes, stream));
+  if (grow || blk->ws_stride_prev != P.ws_stride || blk->ws_kind_prev != 2) {
+    GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, blk->b_ws.bytes, stream));
     GS_CUDA_TRY(cudaMemsetAsync(blk->b_gen.ptr, 0, 4096 * 4, stream));
   }
   blk->ws_stride_prev = P.ws_stride;
+  blk->ws_kind_prev = 2;
   P.ws = (char*)blk->b_ws.ptr;
   P.gen = (uint32_t*)blk->b_gen.ptr;
   P.col0 = (int32_t*)blk->b_col[0].ptr;

@@ -1,24 +1,29 @@
 // nodewise.cu -- node-wise ECSF sampling (GraphSAGE, KGCN, weighted A-Res,
 // PASS-style A3 probabilities) and the ShaDow induced subgraph, as ONE
-// persistent thread-block-cluster kernel per call.
+// persistent thread-block-cluster kernel per call (one launch per epoch).
 //
-// Design:
-//   * one cluster (CS CTAs) owns one mini-batch at a time (super-batch):
-//     every hop of the batch -- Extract, Select and
-//     Finalize -- runs inside the cluster, separated by cluster
-//     barriers, so per-batch state (hash table, slot staging) stays in L2 and
-//     the epoch needs no host synchronisation and one launch;
-//   * P1 select: a group of G = pow2ceil(k) lanes per frontier column
-//     (Extract-Select fusion): gather the indptr pair, draw positions
-//     (Floyd / with replacement / A-Res top-k), gather the sampled rows, stage
-//     (u, eid) in padded slots [T][k] and insert (u, slot) into a
-//     generation-tagged hash keeping the minimum slot (first occurrence);
-//   * P2 finalize-1, slot-parallel: first-occurrence flag, CTA scan of
-//     (valid, first) -> CTA-local edge index and local row id;
-//   * P3 finalize-2, slot-parallel: cluster offsets from DSMEM totals,
-//     relabel, compaction into the block (CSC indptr + COO row_local/eid) and
-//     row_map (A.row(), next frontier).
+// Design ("K-nodewise"):
+//   * one cluster (8 CTAs x 1024 threads, one CTA per SM) owns one mini-batch
+//     at a time (super-batch) and runs every hop of it -- Extract
+//     (P:180), Select, Finalize -- with the
+//     phases separated by cluster barriers, so a batch's hash table and slot
+//     staging (~3 MB) stay in L2 and no host synchronisation is needed;
+//   * every warp owns a contiguous range of frontier columns and works on
+//     chunks of 32 columns (one per lane) with batched independent loads
+//     (memory-level parallelism instead of per-column latency chains):
+//       P1  Extract + Select: indptr pairs, positions (Floyd / replacement /
+//           A-Res top-k) into shared memory, a flattened gather of the sampled
+//           rows (NW_ILP loads in flight per lane), staging of (u, position)
+//           and an ordered-hash atomicMin insert of (u, slot) -- Extract-Select
+//           fusion;
+//       P2  Finalize-1: first-occurrence bitmap over the batch's padded slots
+//           (slot p is first iff the table holds p for its row) and per-word
+//           prefix counts;
+//       P3  Finalize-2: local id of every edge = rank of its row's first slot
+//           (bitmap popcount), compaction into the block (CSC indptr + COO
+//           row_local/eid) and row_map (A.row(), the next frontier).
 #include <cooperative_groups.h>
+
 #include <algorithm>
 #include <cuda_runtime.h>
 #include <math.h>
@@ -26,10 +31,16 @@
 
 #include "common.cuh"
 #include "gs_internal.h"
+#include "nodewise_common.cuh"
 
 namespace cg = cooperative_groups;
 
 namespace gsb {
+
+constexpr int NW_CS = 8;          // CTAs per cluster (= SMs per mini-batch)
+constexpr int NW_THREADS = 1024;  // one CTA per SM
+constexpr int NW_WARPS = NW_THREADS / 32;
+constexpr int MAX_CLUSTERS = 4096;
 
 struct NWParams {
   const int64_t* indptr;
@@ -56,7 +67,7 @@ struct NWParams {
   // per-cluster workspace
   char* ws;
   int64_t ws_stride;
-  int64_t o_u, o_e, o_p0, o_lid, o_eidx, o_val, o_cnt, o_eoff, o_tab;
+  int64_t o_u, o_pos, o_val, o_coff, o_ccnt, o_ceoff, o_bits, o_wpre, o_tab;
   int log_tab_cap;
   uint32_t* gen;
   // ShaDow: induced subgraph on U
@@ -71,197 +82,45 @@ struct NWParams {
 };
 
 struct Ws {
-  int32_t* u;
-  int64_t* e;
-  int32_t* p0;
-  int32_t* lid;
-  int32_t* eidx;
-  float* val;
-  int32_t* cnt;
-  int32_t* eoff;
+  int32_t* u;      // [slot] sampled row
+  uint32_t* pos;   // [slot] position inside the column (ShaDow: local id)
+  float* val;      // [slot] PASS prob (or NULL)
+  int64_t* coff;   // [col] indptr[v]
+  int32_t* ccnt;   // [col] sampled edges of the column
+  int32_t* ceoff;  // [col] CTA-local edge offset
+  uint32_t* bits;  // [slot/32] first-occurrence bitmap
+  int32_t* wpre;   // [slot/32] CTA-local count of first slots before the word
   unsigned long long* tab;
 };
 
-__device__ __forceinline__ int pow2ceil_int(int k) { return k <= 1 ? 1 : 1 << (32 - __clz(k - 1)); }
-
-__device__ __forceinline__ int log2_pow2ceil64(int64_t x) {
-  int l = 0;
-  while ((1ll << l) < x) ++l;
-  return l;
-}
-
+// shared memory of one CTA (dynamic, ~150 KB)
+struct NWSmem {
+  WarpChunk wc[NW_WARPS];
+  unsigned long long scan[33];
+  long long wtot[NW_WARPS];
+  unsigned long long tot;                   // this CTA: (edges << 32) | rows
+  long long base_e[NW_CS + 1], base_r[NW_CS + 1];
+  long long misc[4];
+};
 // next generation tag 1..255; returns true when the table must be cleared.
 __device__ __forceinline__ bool next_gen(uint32_t& gen) {
-  bool wrap = (gen == 255u);
+  const bool wrap = (gen == 255u);
   gen = (gen % 255u) + 1u;
   return wrap;
 }
 
-template <int CS>
 __device__ void clear_table(const NWParams& P, Ws& W, int crank) {
   const int64_t cap = 1ll << P.log_tab_cap;
-  for (int64_t i = (int64_t)crank * blockDim.x + threadIdx.x; i < cap; i += (int64_t)CS * blockDim.x)
-    W.tab[i] = 0ull;
+  for (int64_t i = (int64_t)crank * blockDim.x + threadIdx.x; i < cap;
+       i += (int64_t)NW_CS * blockDim.x)
+    W.tab[i] = ~0ull;
 }
 
-__device__ __forceinline__ uint32_t sel_word(const U4& r, int i) {
-  return i == 0 ? r.x : (i == 1 ? r.y : (i == 2 ? r.z : r.w));
-}
-
-// ---------------------------------------------------------------------------
-// P1: select for the columns [c0, c1) of frontier F (batch-local indices).
-// ---------------------------------------------------------------------------
-__device__ void nw_select(const NWParams& P, Ws& W, int l, int log_cap, uint32_t gen,
-                          const int32_t* F, int64_t c0, int64_t c1, uint32_t gb) {
-  const int k = P.k[l];
-  const int G = pow2ceil_int(k);
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-  const int s = lane & (G - 1), gbase = lane & ~(G - 1);
-  const uint32_t gbits = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << gbase);
-  const int gpw = 32 / G;
-  const uint32_t FULL = 0xffffffffu;
-  const int64_t N = P.N;
-  const bool weighted_sel = !P.replace && P.bias != GS_W_UNIFORM;
-
-  for (int64_t jb = c0 + (int64_t)warp * gpw; jb < c1; jb += (int64_t)nwarps * gpw) {
-    const int64_t j = jb + lane / G;
-    const bool active = j < c1;
-    int32_t v = active ? __ldcg(F + j) : 0;
-    const bool valid = active && v >= 0 && (int64_t)v < N;
-    if (active && !valid && s == 0) atomicOr(P.err, ERR_SEED_RANGE);
-    int64_t off = 0, d = 0;
-    if (valid) {
-      off = __ldg(P.indptr + v);
-      d = __ldg(P.indptr + v + 1) - off;
-    }
-    int cnt = 0;
-    int64_t pos = 0;
-    int slot = s;
-    float pval = 0.f;
-
-    if (P.replace) {
-      // KGCN (R10): k i.i.d. uniform positions, slot order.
-      cnt = d > 0 ? k : 0;
-      if (s < cnt) {
-        U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.key);
-        pos = (int64_t)draw_below((uint64_t)d, r.x, r.y);
-      }
-    } else if (!weighted_sel) {
-      // GraphSAGE (R5): d <= k -> all positions; else Floyd, positions ascending.
-      const bool need = valid && d > k;
-      cnt = (int)(d < k ? d : k);
-      pos = s;
-      if (__ballot_sync(FULL, need)) {
-        const int64_t m = d - k + s;
-        int64_t t = 0;
-        if (need && s < k) {
-          U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.key);
-          t = (int64_t)draw_below((uint64_t)(m + 1), r.x, r.y);
-        }
-        int64_t x = -1;
-        for (int i = 0; i < k; ++i) {
-          const int64_t ti = __shfl_sync(FULL, t, gbase + i);
-          const uint32_t b = __ballot_sync(FULL, s < i && x == ti) & gbits;
-          if (s == i) x = b ? m : t;
-        }
-        int rnk = 0;
-        for (int i = 0; i < k; ++i) {
-          const int64_t xi = __shfl_sync(FULL, x, gbase + i);
-          rnk += (xi < x) ? 1 : 0;
-        }
-        if (need) {
-          pos = x;
-          slot = s < k ? rnk : k;  // lanes beyond k (G > k) hold nothing
-        }
-      }
-    } else {
-      // Weighted without replacement (R6): the k smallest A-Res keys over the
-      // eligible positions (w > 0), ties -> smaller position.
-      double bk = INFINITY;
-      int64_t bp = INT64_MAX;
-      double mk = INFINITY;
-      int64_t mp = INT64_MAX;
-      int ml = 0;
-      double csum = 0.0;
-      int rounds = valid ? (int)((d + G - 1) / G) : 0;
-      rounds = __reduce_max_sync(FULL, (unsigned)rounds);
-      for (int rd = 0; rd < rounds; ++rd) {
-        const int64_t i = (int64_t)rd * G + s;
-        const bool in = valid && i < d;
-        const float w = in ? (P.weights ? __ldg(P.weights + off + i) : 1.0f) : 0.0f;
-        csum += in ? (double)w : 0.0;
-        const bool elig = in && w > 0.0f;
-        double kk = INFINITY;
-        if (elig) {
-          U4 r = philox((uint32_t)v, (uint32_t)(i >> 2), ctr2(l, TAG_ARES_NODE), gb, P.key);
-          kk = ares_key(sel_word(r, (int)(i & 3)), (double)w);
-        }
-        uint32_t cand = __ballot_sync(FULL, elig && key_less(kk, i, mk, mp)) & gbits;
-        while (__any_sync(FULL, cand != 0u)) {
-          const int c = cand ? (__ffs(cand) - 1) : 0;
-          const double ck = __shfl_sync(FULL, kk, c);
-          const int64_t cp = __shfl_sync(FULL, i, c);
-          const bool ins = cand != 0u && key_less(ck, cp, mk, mp);
-          if (ins && s == ml) {
-            bk = ck;
-            bp = cp;
-          }
-          if (cand) cand &= cand - 1u;
-          // new group maximum over the k held entries: (key, pos, lane) lexicographic
-          double tk = (s < k) ? bk : -INFINITY;
-          int64_t tp = (s < k) ? bp : -1;
-          int tl = s;
-          for (int o = G >> 1; o > 0; o >>= 1) {
-            const double ok = __shfl_xor_sync(FULL, tk, o);
-            const int64_t op = __shfl_xor_sync(FULL, tp, o);
-            const int ol = __shfl_xor_sync(FULL, tl, o);
-            const bool other_bigger = key_less(tk, tp, ok, op) || (tk == ok && tp == op && ol > tl);
-            if (other_bigger) {
-              tk = ok;
-              tp = op;
-              tl = ol;
-            }
-          }
-          if (ins) {
-            mk = tk;
-            mp = tp;
-            ml = tl;
-          }
-        }
-      }
-      const bool sel = s < k && bp != INT64_MAX;
-      const uint32_t selb = __ballot_sync(FULL, sel) & gbits;
-      cnt = __popc(selb);
-      int rnk = 0;
-      for (int i = 0; i < G; ++i) {
-        const int64_t pi = __shfl_sync(FULL, bp, gbase + i);
-        const bool si = (selb >> (gbase + i)) & 1u;
-        rnk += (si && pi < bp) ? 1 : 0;
-      }
-      pos = bp;
-      slot = rnk;
-      if (P.bias == GS_W_PASS_COLNORM) {
-        for (int o = G >> 1; o > 0; o >>= 1) csum += __shfl_xor_sync(FULL, csum, o);
-        if (sel) {
-          const float w = P.weights ? __ldg(P.weights + off + bp) : 1.0f;
-          pval = w / (float)csum;
-        }
-      }
-      if (!sel) slot = k;  // not taken
-    }
-
-    // Stage the sampled edges and insert their rows (first slot wins).
-    if (valid && slot < cnt) {
-      const int64_t e = off + pos;
-      const int32_t u = __ldg(P.indices + e);
-      const int64_t p = j * k + slot;
-      W.u[p] = u;
-      W.e[p] = e;
-      if (W.val) W.val[p] = pval;
-      tab_insert_min(W.tab, log_cap, gen, (uint32_t)u, (uint32_t)p);
-    }
-    if (active && s == 0) W.cnt[j] = valid ? cnt : 0;
-  }
+// Range of warp `w` inside [c0, c1) (contiguous split).
+__device__ __forceinline__ void warp_range(int64_t c0, int64_t c1, int w, int64_t* a, int64_t* b) {
+  const int64_t n = c1 - c0, per = (n + NW_WARPS - 1) / NW_WARPS;
+  *a = min(c1, c0 + (int64_t)w * per);
+  *b = min(c1, *a + per);
 }
 
 // ---------------------------------------------------------------------------
@@ -272,13 +131,9 @@ __device__ void nw_select(const NWParams& P, Ws& W, int l, int log_cap, uint32_t
 //   S3 write U and replace each entry's value by the local id;
 //   S4 warp-per-column count of in-U rows + CTA scan;  S5 emit.
 // ---------------------------------------------------------------------------
-template <int CS>
-__device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& cluster, int crank,
-                              int64_t b, int64_t bstart, int64_t nb, const int64_t* rows_l,
-                              uint32_t gen, unsigned long long* s_scan, unsigned long long* s_tot,
-                              long long* s_base_e, long long* s_base_r) {
-  __shared__ long long s_ebase;
-  // segment starts of Z
+__device__ void shadow_induce(const NWParams& P, Ws& W, NWSmem& S, cg::cluster_group& cluster,
+                              int crank, int64_t b, int64_t bstart, int64_t nb,
+                              const int64_t* rows_l, uint32_t tag) {
   int64_t seg_start[MAX_LAYERS + 2];
   seg_start[0] = 0;
   seg_start[1] = nb;
@@ -292,14 +147,15 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
   };
   int log_cap = log2_pow2ceil64((Zn * 4) / 3 + 64);
   if (log_cap > P.log_tab_cap) log_cap = P.log_tab_cap;
-  const int64_t zchunk = (Zn + CS - 1) / CS;
+  const int64_t zchunk = (Zn + NW_CS - 1) / NW_CS;
   const int64_t z0 = min(Zn, (int64_t)crank * zchunk), z1 = min(Zn, z0 + zchunk);
   const int64_t ubase = bstart * P.sh_stride;
   const int64_t uibase = ubase + b;
+  uint32_t* lidz = W.pos;  // reuse: local id of first occurrences
 
   // S1
   for (int64_t z = z0 + threadIdx.x; z < z1; z += blockDim.x)
-    tab_insert_min(W.tab, log_cap, gen, zval(z), (uint32_t)z);
+    otab_insert_min(W.tab, log_cap, tag, zval(z), (uint32_t)z);
   cluster.sync();
   // S2
   unsigned long long carry = 0;
@@ -307,95 +163,92 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
     const int64_t z = zt + threadIdx.x;
     bool first = false;
     if (z < z1) {
-      const int64_t h = tab_find(W.tab, log_cap, gen, zval(z));
-      first = tab_val(__ldcg(W.tab + h)) == (uint32_t)z;
+      const int64_t h = otab_find(W.tab, log_cap, tag, zval(z));
+      first = h >= 0 && tab_val(__ldcg(W.tab + h)) == (uint32_t)z;
     }
     unsigned long long tot;
-    const unsigned long long ex = block_exclusive_scan((unsigned long long)(first ? 1 : 0), s_scan, &tot) + carry;
-    if (first) W.lid[z] = (int32_t)ex;
+    const unsigned long long ex =
+        block_exclusive_scan((unsigned long long)(first ? 1 : 0), S.scan, &tot) + carry;
+    if (first) lidz[z] = (uint32_t)ex;
     carry += tot;
   }
-  if (threadIdx.x == 0) *s_tot = carry;
+  if (threadIdx.x == 0) S.tot = carry;
   cluster.sync();
   if (threadIdx.x == 0) {
     long long a = 0;
-    for (int r = 0; r < CS; ++r) {
-      s_base_r[r] = a;
-      a += (long long)*cluster.map_shared_rank(s_tot, r);
+    for (int r = 0; r < NW_CS; ++r) {
+      S.base_r[r] = a;
+      a += (long long)cluster.map_shared_rank(&S, r)->tot;
     }
-    s_base_r[CS] = a;
+    S.base_r[NW_CS] = a;
   }
   __syncthreads();
-  const int64_t nU = s_base_r[CS];
+  const int64_t nU = S.base_r[NW_CS];
   // S3
   for (int64_t z = z0 + threadIdx.x; z < z1; z += blockDim.x) {
     const uint32_t u = zval(z);
-    const int64_t h = tab_find(W.tab, log_cap, gen, u);
-    if (tab_val(__ldcg(W.tab + h)) == (uint32_t)z) {
-      const int64_t lid = s_base_r[crank] + __ldcg(W.lid + z);
+    const int64_t h = otab_find(W.tab, log_cap, tag, u);
+    if (h >= 0 && tab_val(__ldcg(W.tab + h)) == (uint32_t)z) {
+      const int64_t lid = S.base_r[crank] + __ldcg(lidz + z);
       P.sh_nodes[ubase + lid] = (int32_t)u;
-      W.tab[h] = tab_entry(gen, u, (uint32_t)lid);
+      W.tab[h] = tab_entry(tag, u, (uint32_t)lid);
     }
   }
   cluster.sync();
   // S4: count in-U rows of every column of U (warp per column)
-  const int64_t uchunk = (nU + CS - 1) / CS;
+  const int64_t uchunk = (nU + NW_CS - 1) / NW_CS;
   const int64_t u0 = min(nU, (int64_t)crank * uchunk), u1 = min(nU, u0 + uchunk);
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-  for (int64_t c = u0 + warp; c < u1; c += nwarps) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int64_t c = u0 + warp; c < u1; c += NW_WARPS) {
     const int32_t v = __ldcg(P.sh_nodes + ubase + c);
     const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
     int cnt = 0;
     for (int64_t i = lane; i < d; i += 32) {
       const uint32_t u = (uint32_t)__ldg(P.indices + off + i);
-      cnt += tab_find(W.tab, log_cap, gen, u) >= 0 ? 1 : 0;
+      cnt += otab_find(W.tab, log_cap, tag, u) >= 0 ? 1 : 0;
     }
-    cnt = __reduce_add_sync(0xffffffffu, (unsigned)cnt);
-    if (lane == 0) W.cnt[c] = cnt;
+    cnt = (int)__reduce_add_sync(0xffffffffu, (unsigned)cnt);
+    if (lane == 0) W.ccnt[c] = cnt;
   }
   __syncthreads();
   carry = 0;
   for (int64_t ct = u0; ct < u1; ct += blockDim.x) {
     const int64_t c = ct + threadIdx.x;
-    const unsigned long long cv = c < u1 ? (unsigned long long)__ldcg(W.cnt + c) : 0ull;
+    const unsigned long long cv = c < u1 ? (unsigned long long)__ldcg(W.ccnt + c) : 0ull;
     unsigned long long tot;
-    const unsigned long long ex = block_exclusive_scan(cv, s_scan, &tot) + carry;
-    if (c < u1) W.eoff[c] = (int32_t)ex;
+    const unsigned long long ex = block_exclusive_scan(cv, S.scan, &tot) + carry;
+    if (c < u1) W.ceoff[c] = (int32_t)ex;
     carry += tot;
   }
-  if (threadIdx.x == 0) *s_tot = carry;
+  if (threadIdx.x == 0) S.tot = carry;
   cluster.sync();
   if (threadIdx.x == 0) {
     long long a = 0;
-    for (int r = 0; r < CS; ++r) {
-      s_base_e[r] = a;
-      a += (long long)*cluster.map_shared_rank(s_tot, r);
+    for (int r = 0; r < NW_CS; ++r) {
+      S.base_e[r] = a;
+      a += (long long)cluster.map_shared_rank(&S, r)->tot;
     }
-    s_base_e[CS] = a;
-    if (crank == 0) s_ebase = (long long)atomicAdd(P.sh_edge_ctr, (unsigned long long)a);
+    S.base_e[NW_CS] = a;
+    if (crank == 0) S.misc[0] = (long long)atomicAdd(P.sh_edge_ctr, (unsigned long long)a);
   }
   cluster.sync();
-  if (threadIdx.x == 0) s_ebase = *cluster.map_shared_rank(&s_ebase, 0);
+  if (threadIdx.x == 0) S.misc[1] = cluster.map_shared_rank(&S, 0)->misc[0];
   __syncthreads();
-  const int64_t nE = s_base_e[CS];
-  const int64_t ebase = s_ebase;
+  const int64_t nE = S.base_e[NW_CS];
+  const int64_t ebase = S.misc[1];
   const bool fits = ebase + nE <= P.sh_edge_cap;
   if (!fits && crank == 0 && threadIdx.x == 0) atomicOr(P.err, ERR_CAPACITY);
   // S5: emit (warp per column, ballot compaction keeps CSC order)
-  for (int64_t c = u0 + warp; c < u1; c += nwarps) {
+  for (int64_t c = u0 + warp; c < u1; c += NW_WARPS) {
     const int32_t v = __ldcg(P.sh_nodes + ubase + c);
     const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
-    int64_t e = s_base_e[crank] + __ldcg(W.eoff + c);
+    int64_t e = S.base_e[crank] + __ldcg(W.ceoff + c);
     if (lane == 0) P.sh_indptr[uibase + c] = e;
     if (!fits) continue;
     for (int64_t i0 = 0; i0 < d; i0 += 32) {
       const int64_t i = i0 + lane;
       int64_t h = -1;
-      uint32_t u = 0;
-      if (i < d) {
-        u = (uint32_t)__ldg(P.indices + off + i);
-        h = tab_find(W.tab, log_cap, gen, u);
-      }
+      if (i < d) h = otab_find(W.tab, log_cap, tag, (uint32_t)__ldg(P.indices + off + i));
       const uint32_t m = __ballot_sync(0xffffffffu, h >= 0);
       if (h >= 0) {
         const int64_t o = ebase + e + __popc(m & ((1u << lane) - 1u));
@@ -417,30 +270,45 @@ __device__ void shadow_induce(const NWParams& P, Ws& W, cg::cluster_group& clust
 // ---------------------------------------------------------------------------
 // The kernel: one cluster per batch, all hops (and the ShaDow induce) inside.
 // ---------------------------------------------------------------------------
-template <int CS>
-__global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
+__global__ void __cluster_dims__(NW_CS, 1, 1) __launch_bounds__(NW_THREADS, 1)
+    nodewise_kernel(NWParams P) {
   cg::cluster_group cluster = cg::this_cluster();
   const int crank = (int)cluster.block_rank();
-  const int64_t cid = blockIdx.x / CS;
-  const int64_t nclusters = gridDim.x / CS;
-
-  __shared__ unsigned long long s_scan[33];
-  __shared__ unsigned long long s_tot;        // this CTA: (edges << 32) | rows
-  __shared__ long long s_base_e[CS + 1], s_base_r[CS + 1];
+  const int64_t cid = blockIdx.x / NW_CS;
+  const int64_t nclusters = gridDim.x / NW_CS;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  NWSmem& S = *reinterpret_cast<NWSmem*>(smem_raw);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
 
   Ws W;
   char* base = P.ws + cid * P.ws_stride;
   W.u = (int32_t*)(base + P.o_u);
-  W.e = (int64_t*)(base + P.o_e);
-  W.p0 = (int32_t*)(base + P.o_p0);
-  W.lid = (int32_t*)(base + P.o_lid);
-  W.eidx = (int32_t*)(base + P.o_eidx);
+  W.pos = (uint32_t*)(base + P.o_pos);
   W.val = P.o_val >= 0 ? (float*)(base + P.o_val) : nullptr;
-  W.cnt = (int32_t*)(base + P.o_cnt);
-  W.eoff = (int32_t*)(base + P.o_eoff);
+  W.coff = (int64_t*)(base + P.o_coff);
+  W.ccnt = (int32_t*)(base + P.o_ccnt);
+  W.ceoff = (int32_t*)(base + P.o_ceoff);
+  W.bits = (uint32_t*)(base + P.o_bits);
+  W.wpre = (int32_t*)(base + P.o_wpre);
   W.tab = (unsigned long long*)(base + P.o_tab);
 
   uint32_t gen = P.gen[cid];
+  NWCore core;
+  core.indptr = P.indptr;
+  core.indices = P.indices;
+  core.weights = P.weights;
+  core.N = P.N;
+  core.err = P.err;
+  core.replace = P.replace;
+  core.bias = P.bias;
+  core.key = P.key;
+  NWStage stage;
+  stage.u = W.u;
+  stage.pos = W.pos;
+  stage.val = W.val;
+  stage.coff = W.coff;
+  stage.ccnt = W.ccnt;
+  stage.tab = W.tab;
 
   for (int64_t b = cid; b < P.num_batches; b += nclusters) {
     const int64_t bstart = b * P.batch_size;
@@ -448,7 +316,7 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
     const uint32_t gb = (uint32_t)(P.batch_base + b);
     const int32_t* F = P.seeds + bstart;
     int64_t T = nb;
-    int64_t colbase = bstart;      // region of this layer's columns
+    int64_t colbase = bstart;
     int64_t rows_l[MAX_LAYERS];
 
     for (int l = 0; l < P.L; ++l) {
@@ -456,101 +324,192 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
       const int64_t rbase = bstart * P.K[l];
       const int64_t ibase = colbase + b;
       if (next_gen(gen)) {
-        clear_table<CS>(P, W, crank);
+        clear_table(P, W, crank);
         cluster.sync();
       }
-      int64_t want = (T * k * 4) / 3 + 64;
-      int log_cap = log2_pow2ceil64(want);
+      const uint32_t tag = otag(gen);
+      int log_cap = log2_pow2ceil64((T * k * 4) / 3 + 64);
       if (log_cap > P.log_tab_cap) log_cap = P.log_tab_cap;
-      const int64_t chunk = (T + CS - 1) / CS;
+      const int64_t chunk = (T + NW_CS - 1) / NW_CS;
       const int64_t c0 = min(T, (int64_t)crank * chunk), c1 = min(T, c0 + chunk);
+      int64_t wa, wb;
+      warp_range(c0, c1, warp, &wa, &wb);
 
-      // ---- P1: select + insert ----
-      nw_select(P, W, l, log_cap, gen, F, c0, c1, gb);
-      cluster.sync();
-
-      // ---- P2: first-occurrence flags, CTA scan over slots ----
-      unsigned long long carry = 0;
-      const int64_t p_lo = c0 * k, p_hi = c1 * k;
-      for (int64_t pt = p_lo; pt < p_hi; pt += blockDim.x) {
-        const int64_t p = pt + threadIdx.x;
-        bool valid = false, first = false;
-        int64_t j = 0;
-        int s = 0;
-        if (p < p_hi) {
-          j = p / k;
-          s = (int)(p - j * k);
-          valid = s < __ldcg(W.cnt + j);
-          if (valid) {
-            const uint32_t u = (uint32_t)__ldcg(W.u + p);
-            const int64_t h = tab_find(W.tab, log_cap, gen, u);
-            if (h < 0) atomicOr(P.err, ERR_INTERNAL);
-            const uint32_t p0 = h < 0 ? 0xffffffffu : tab_val(__ldcg(W.tab + h));
-            W.p0[p] = (int32_t)p0;
-            first = (p0 == (uint32_t)p);
-          }
-        }
-        const unsigned long long packed = ((unsigned long long)(valid ? 1 : 0) << 32) | (first ? 1ull : 0ull);
-        unsigned long long tot;
-        const unsigned long long ex = block_exclusive_scan(packed, s_scan, &tot) + carry;
-        if (p < p_hi) {
-          if (s == 0) W.eoff[j] = (int32_t)(ex >> 32);
-          if (valid) W.eidx[p] = (int32_t)(ex >> 32);
-          if (first) W.lid[p] = (int32_t)(ex & 0xffffffffu);
-        }
-        carry += tot;
+      // ---- P1: Extract + Select + stage + insert ----
+      int wedges = 0;
+      for (int64_t jb = wa; jb < wb; jb += 32)
+        wedges += select_chunk(core, stage, S.wc[warp], l, k, log_cap, tag, F, jb, wb, gb);
+      if (lane == 0) S.wtot[warp] = wedges;
+      __syncthreads();
+      if (warp == 0) {  // exclusive scan of the warp totals
+        const int t = lane < NW_WARPS ? (int)S.wtot[lane] : 0;
+        int tot;
+        const int ex = warp_excl(t, &tot);
+        if (lane < NW_WARPS) S.wtot[lane] = ex;
+        if (lane == 0) S.misc[2] = tot;
       }
-      if (threadIdx.x == 0) s_tot = carry;
+      __syncthreads();
+      {  // CTA-local edge offset of every column of this warp
+        long long run = S.wtot[warp];
+        for (int64_t jb = wa; jb < wb; jb += 32) {
+          const int64_t j = jb + lane;
+          const int c = j < wb ? __ldcg(W.ccnt + j) : 0;
+          int tot;
+          const int ex = warp_excl(c, &tot);
+          if (j < wb) W.ceoff[j] = (int32_t)(run + ex);
+          run += tot;
+        }
+      }
+      const long long cta_edges = S.misc[2];
       cluster.sync();
 
-      // ---- P3: cluster offsets, relabel, compaction ----
+      // ---- P2: first-occurrence bitmap over the batch's padded slots ----
+      const int64_t PT = T * k;
+      const int64_t NWD = (PT + 31) >> 5;
+      const int64_t wchunk = (NWD + NW_CS - 1) / NW_CS;
+      const int64_t w0 = min(NWD, (int64_t)crank * wchunk), w1 = min(NWD, w0 + wchunk);
+      int64_t xa, xb;
+      warp_range(w0, w1, warp, &xa, &xb);
+      int wrows = 0;
+      for (int64_t wd0 = xa; wd0 < xb; wd0 += NW_ILP) {
+        uint32_t uu[NW_ILP];
+        bool vv[NW_ILP];
+        int64_t hh[NW_ILP];
+#pragma unroll
+        for (int i = 0; i < NW_ILP; ++i) {
+          const int64_t wd = wd0 + i;
+          const int64_t p = wd * 32 + lane;
+          vv[i] = false;
+          if (wd < xb && p < PT) {
+            const int64_t j = p / k;
+            vv[i] = (p - j * k) < __ldcg(W.ccnt + j);
+          }
+          uu[i] = vv[i] ? (uint32_t)__ldcg(W.u + p) : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < NW_ILP; ++i)
+          hh[i] = vv[i] ? otab_find(W.tab, log_cap, tag, uu[i]) : -1;
+#pragma unroll
+        for (int i = 0; i < NW_ILP; ++i) {
+          const int64_t wd = wd0 + i;
+          const int64_t p = wd * 32 + lane;
+          bool first = false;
+          if (vv[i]) {
+            if (hh[i] < 0) atomicOr(P.err, ERR_INTERNAL);
+            else first = tab_val(__ldcg(W.tab + hh[i])) == (uint32_t)p;
+          }
+          const uint32_t word = __ballot_sync(0xffffffffu, first);
+          if (wd < xb && lane == 0) W.bits[wd] = word;
+          wrows += __popc(word);
+        }
+      }
+      if (lane == 0) S.wtot[warp] = wrows;
+      __syncthreads();
+      if (warp == 0) {
+        const int t = lane < NW_WARPS ? (int)S.wtot[lane] : 0;
+        int tot;
+        const int ex = warp_excl(t, &tot);
+        if (lane < NW_WARPS) S.wtot[lane] = ex;
+        if (lane == 0) S.tot = ((unsigned long long)cta_edges << 32) | (unsigned)tot;
+      }
+      __syncthreads();
+      {  // CTA-local count of first slots before every word of this warp
+        long long run = S.wtot[warp];
+        for (int64_t wd0 = xa; wd0 < xb; wd0 += 32) {
+          const int64_t wd = wd0 + lane;
+          const int c = wd < xb ? __popc(__ldcg(W.bits + wd)) : 0;
+          int tot;
+          const int ex = warp_excl(c, &tot);
+          if (wd < xb) W.wpre[wd] = (int32_t)(run + ex);
+          run += tot;
+        }
+      }
+      cluster.sync();
+
+      // ---- P3: relabel + compaction ----
       if (threadIdx.x == 0) {
         long long ae = 0, ar = 0;
-        for (int r = 0; r < CS; ++r) {
-          s_base_e[r] = ae;
-          s_base_r[r] = ar;
-          const unsigned long long t = *cluster.map_shared_rank(&s_tot, r);
+        for (int r = 0; r < NW_CS; ++r) {
+          S.base_e[r] = ae;
+          S.base_r[r] = ar;
+          const unsigned long long t = cluster.map_shared_rank(&S, r)->tot;
           ae += (long long)(t >> 32);
           ar += (long long)(t & 0xffffffffu);
         }
-        s_base_e[CS] = ae;
-        s_base_r[CS] = ar;
+        S.base_e[NW_CS] = ae;
+        S.base_r[NW_CS] = ar;
       }
       __syncthreads();
-      const int64_t baseE = s_base_e[crank], baseR = s_base_r[crank];
-      const int64_t totE = s_base_e[CS], totR = s_base_r[CS];
-      int32_t* row_map = P.row_map[l];
-      int32_t* row_local = P.row_local[l];
-      int64_t* eid_out = P.eid[l];
-      float* val_out = P.val[l];
-      int64_t* indptr_out = P.indptr_out[l];
-      for (int64_t pt = p_lo; pt < p_hi; pt += blockDim.x) {
-        const int64_t p = pt + threadIdx.x;
-        if (p >= p_hi) continue;
-        const int64_t j = p / k;
-        const int s = (int)(p - j * k);
-        if (s == 0) {
-          if (indptr_out) indptr_out[ibase + j] = baseE + __ldcg(W.eoff + j);
-          if (l == 0 && P.col0) P.col0[bstart + j] = F[j];
+      const int64_t baseE = S.base_e[crank];
+      const int64_t totE = S.base_e[NW_CS], totR = S.base_r[NW_CS];
+      int32_t* row_map = P.row_map[l] + rbase;
+      int32_t* row_local = P.row_local[l] ? P.row_local[l] + rbase : nullptr;
+      int64_t* eid_out = P.eid[l] ? P.eid[l] + rbase : nullptr;
+      float* val_out = P.val[l] ? P.val[l] + rbase : nullptr;
+      int64_t* indptr_out = P.indptr_out[l] ? P.indptr_out[l] + ibase : nullptr;
+      for (int64_t jb = wa; jb < wb; jb += 32) {
+        const int64_t j = jb + lane;
+        const bool act = j < wb;
+        const int cnt = act ? __ldcg(W.ccnt + j) : 0;
+        const int eo = act ? __ldcg(W.ceoff + j) : 0;
+        const int64_t off = act ? __ldcg(W.coff + j) : 0;
+        int total;
+        const int pre = warp_excl(cnt, &total);
+        S.wc[warp].pre[lane] = pre;
+        S.wc[warp].coff[lane] = off;
+        S.wc[warp].cnt_all[lane] = eo;  // P3: CTA-local edge offset of the column
+        if (act) {
+          if (indptr_out) indptr_out[j] = baseE + eo;
+          if (l == 0 && P.col0) P.col0[bstart + j] = __ldcg(F + j);
         }
-        if (s >= __ldcg(W.cnt + j)) continue;
-        const int32_t p0 = __ldcg(W.p0 + p);
-        int64_t lid;
-        if (p0 == (int32_t)p) {
-          lid = baseR + __ldcg(W.lid + p);
-          row_map[rbase + lid] = __ldcg(W.u + p);
-        } else {
-          const int64_t j0 = p0 / k;
-          const int r0 = (int)(j0 / chunk);
-          lid = s_base_r[r0] + __ldcg(W.lid + p0);
+        __syncwarp();
+        for (int f0 = 0; f0 < total; f0 += 32 * NW_ILP) {
+          int64_t p[NW_ILP], e[NW_ILP], hh[NW_ILP];
+          uint32_t uu[NW_ILP], ps[NW_ILP];
+          int cc[NW_ILP];
+          bool ok[NW_ILP];
+#pragma unroll
+          for (int i = 0; i < NW_ILP; ++i) {
+            const int f = f0 + i * 32 + lane;
+            ok[i] = f < total;
+            cc[i] = 0;
+            if (ok[i]) {
+              const int c = chunk_col(S.wc[warp].pre, f);
+              const int s = f - S.wc[warp].pre[c];
+              p[i] = (jb + c) * k + s;
+              e[i] = baseE + S.wc[warp].cnt_all[c] + s;
+              uu[i] = (uint32_t)__ldcg(W.u + p[i]);
+              ps[i] = __ldcg(W.pos + p[i]);
+              cc[i] = c;
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < NW_ILP; ++i) {
+            hh[i] = -1;
+            if (ok[i]) {
+              if (eid_out) eid_out[e[i]] = S.wc[warp].coff[cc[i]] + ps[i];
+              if (val_out) val_out[e[i]] = __ldcg(W.val + p[i]);
+              hh[i] = otab_find(W.tab, log_cap, tag, uu[i]);
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < NW_ILP; ++i) {
+            if (ok[i]) {
+              const uint32_t p0 = hh[i] >= 0 ? tab_val(__ldcg(W.tab + hh[i])) : 0u;
+              const int64_t wd = p0 >> 5;
+              const int r0 = (int)(wd / wchunk);
+              const uint32_t bw = __ldcg(W.bits + wd);
+              const int64_t lid = S.base_r[r0] + __ldcg(W.wpre + wd) +
+                                  __popc(bw & ((1u << (p0 & 31)) - 1u));
+              if (row_local) row_local[e[i]] = (int32_t)lid;
+              if (p0 == (uint32_t)p[i]) row_map[lid] = (int32_t)uu[i];
+            }
+          }
         }
-        const int64_t e = rbase + baseE + __ldcg(W.eidx + p);
-        if (row_local) row_local[e] = (int32_t)lid;
-        if (eid_out) eid_out[e] = __ldcg(W.e + p);
-        if (val_out) val_out[e] = __ldcg(W.val + p);
+        __syncwarp();
       }
       if (crank == 0 && threadIdx.x == 0) {
-        if (indptr_out) indptr_out[ibase + T] = totE;
+        if (indptr_out) indptr_out[T] = totE;
         if (!P.shadow) {
           long long* m = (long long*)(P.meta + (b * P.meta_layers + l) * 8);
           m[0] = T; m[1] = totR; m[2] = totE; m[3] = colbase; m[4] = rbase; m[5] = ibase;
@@ -558,7 +517,7 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
         }
       }
       cluster.sync();
-      F = row_map + rbase;
+      F = P.row_map[l] + rbase;
       T = totR;
       colbase = rbase;
       rows_l[l] = totR;
@@ -566,55 +525,40 @@ __global__ void __launch_bounds__(512, 2) nodewise_kernel(NWParams P) {
 
     if (P.shadow) {
       if (next_gen(gen)) {
-        clear_table<CS>(P, W, crank);
+        clear_table(P, W, crank);
         cluster.sync();
       }
-      shadow_induce<CS>(P, W, cluster, crank, b, bstart, nb, rows_l, gen, s_scan, &s_tot,
-                        s_base_e, s_base_r);
+      shadow_induce(P, W, S, cluster, crank, b, bstart, nb, rows_l, otag(gen));
     }
   }
   if (crank == 0 && threadIdx.x == 0) P.gen[cid] = gen;
 }
 
-}  // namespace gsb
-
 // ---------------------------------------------------------------------------
 // Host side
 // ---------------------------------------------------------------------------
-namespace gsb {
-
 static int64_t align256(int64_t x) { return (x + 255) & ~int64_t(255); }
 
-template <int CS>
-static int max_active_clusters(int threads) {
+static int max_active_clusters() {
   static int cached = -1;
   if (cached > 0) return cached;
+  cudaFuncSetAttribute(nodewise_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)sizeof(NWSmem));
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(CS * 1024);
-  cfg.blockDim = dim3(threads);
-  cfg.dynamicSmemBytes = 0;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = CS;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.gridDim = dim3(NW_CS * 1024);
+  cfg.blockDim = dim3(NW_THREADS);
+  cfg.dynamicSmemBytes = sizeof(NWSmem);
   int n = 0;
-  if (cudaOccupancyMaxActiveClusters(&n, nodewise_kernel<CS>, &cfg) != cudaSuccess || n <= 0) {
+  if (cudaOccupancyMaxActiveClusters(&n, nodewise_kernel, &cfg) != cudaSuccess || n <= 0) {
     cudaGetLastError();
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    n = sms / CS;
+    n = sms / NW_CS;
   }
   cached = n;
   return n;
 }
-
-constexpr int NW_CS = 8;
-constexpr int NW_THREADS = 512;
-constexpr int MAX_CLUSTERS = 4096;
 
 gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                        int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
@@ -636,7 +580,7 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
   P.bias = bias;
   P.key = key;
   int64_t prod = 1, sum_K = 0;
-  int64_t slot_cap = 1, col_cap = 1;
+  int64_t slot_cap = 32, col_cap = 32;
   for (int l = 0; l < L; ++l) {
     P.k[l] = fanouts[l];
     col_cap = std::max(col_cap, batch_size * prod);
@@ -651,6 +595,8 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
     slot_cap = std::max(slot_cap, batch_size * P.sh_stride);
     col_cap = std::max(col_cap, batch_size * P.sh_stride);
   }
+  col_cap += 32;
+  slot_cap += 64;
   const int64_t nbatch = P.num_batches;
   blk->kind = shadow ? gs_blocks::SHADOW : gs_blocks::NODEWISE;
   blk->num_batches = nbatch;
@@ -676,52 +622,52 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
   int64_t sh_nodes = 0, sh_edges = 0;
   if (shadow && ok) {
     sh_nodes = num_seeds * P.sh_stride;
-    sh_edges = std::max<int64_t>(std::max<int64_t>(int64_t(1) << 20, blk->sh_edge_hint), sh_nodes * 4);
+    sh_edges = std::max<int64_t>(std::max<int64_t>(int64_t(1) << 20, blk->sh_edge_hint),
+                                 sh_nodes * 4);
     ok = need(blk->b_col[1], sh_nodes * 4) && need(blk->b_indptr[0], (sh_nodes + nbatch) * 8) &&
          need(blk->b_rowl[0], sh_edges * 4) && need(blk->b_eid[0], sh_edges * 8);
     sh_edges = (int64_t)std::min(blk->b_rowl[0].bytes / 4, blk->b_eid[0].bytes / 8);
   }
   const int meta_layers = shadow ? 1 : L;
   ok = ok && need(blk->b_meta, nbatch * meta_layers * 8 * 8) && need(blk->b_err, 16) &&
-       need(blk->b_ctr, 16);
+       need(blk->b_ctr, 8 * (MAX_LAYERS + 2));
   if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (blocks buffers)");
 
   // ---- workspace (per cluster) ----
   int log_tab = 6;
   while ((int64_t(1) << log_tab) < (slot_cap * 4) / 3 + 64) ++log_tab;
+  const int64_t words = (slot_cap + 31) / 32 + 2;
   int64_t o = 0;
   P.o_u = o; o = align256(o + slot_cap * 4);
-  P.o_e = o; o = align256(o + slot_cap * 8);
-  P.o_p0 = o; o = align256(o + slot_cap * 4);
-  P.o_lid = o; o = align256(o + slot_cap * 4);
-  P.o_eidx = o; o = align256(o + slot_cap * 4);
+  P.o_pos = o; o = align256(o + slot_cap * 4);
   if (bias == GS_W_PASS_COLNORM && !shadow) {
     P.o_val = o;
     o = align256(o + slot_cap * 4);
   } else {
     P.o_val = -1;
   }
-  P.o_cnt = o; o = align256(o + col_cap * 4);
-  P.o_eoff = o; o = align256(o + col_cap * 4);
+  P.o_coff = o; o = align256(o + col_cap * 8);
+  P.o_ccnt = o; o = align256(o + col_cap * 4);
+  P.o_ceoff = o; o = align256(o + col_cap * 4);
+  P.o_bits = o; o = align256(o + words * 4);
+  P.o_wpre = o; o = align256(o + words * 4);
   P.o_tab = o; o = align256(o + (int64_t(8) << log_tab));
   P.ws_stride = o;
   P.log_tab_cap = log_tab;
   const int nclusters =
-      (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, max_active_clusters<NW_CS>(NW_THREADS)));
+      (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, max_active_clusters()));
   const size_t ws_bytes = (size_t)P.ws_stride * nclusters;
-  const bool grow = blk->b_ws.bytes < ws_bytes;
-  if (!blk->b_ws.ensure(al, ws_bytes, stream, true) ||
-      !blk->b_gen.ensure(al, MAX_CLUSTERS * 4, stream, true))
+  const bool fresh = blk->b_ws.bytes < ws_bytes || blk->ws_stride_prev != P.ws_stride ||
+                     blk->ws_kind_prev != 1;
+  if (!blk->b_ws.ensure(al, ws_bytes, stream) || !blk->b_gen.ensure(al, MAX_CLUSTERS * 4, stream))
     return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (workspace)");
-  if (grow) {
-    // a regrown workspace starts with an all-empty table: restart the tags
-    GS_CUDA_TRY(cudaMemsetAsync(blk->b_gen.ptr, 0, MAX_CLUSTERS * 4, stream));
-  } else if (blk->ws_stride_prev != P.ws_stride) {
-    // the layout moved: old tags could alias inside the new table region
-    GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, blk->b_ws.bytes, stream));
+  if (fresh) {
+    // tables start cleared (~0 = the oldest generation), tags restart at 1
+    GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0xFF, blk->b_ws.bytes, stream));
     GS_CUDA_TRY(cudaMemsetAsync(blk->b_gen.ptr, 0, MAX_CLUSTERS * 4, stream));
   }
   blk->ws_stride_prev = P.ws_stride;
+  blk->ws_kind_prev = 1;
   P.ws = (char*)blk->b_ws.ptr;
   P.gen = (uint32_t*)blk->b_gen.ptr;
 
@@ -771,22 +717,15 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
   P.meta_layers = meta_layers;
   P.err = (int*)blk->b_err.ptr;
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
-  GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 16, stream));
+  GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
 
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(nclusters * NW_CS));
   cfg.blockDim = dim3(NW_THREADS);
-  cfg.dynamicSmemBytes = 0;
+  cfg.dynamicSmemBytes = sizeof(NWSmem);
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = NW_CS;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, nodewise_kernel<NW_CS>, P));
+  GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, nodewise_kernel, P));
   return GS_OK;
 }
 
