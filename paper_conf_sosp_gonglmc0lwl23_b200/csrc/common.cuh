@@ -178,6 +178,40 @@ __device__ __forceinline__ int64_t otab_find(const unsigned long long* tab, int 
 }
 
 // ---------------------------------------------------------------------------
+// Fixed-position table for concurrent insert + lookup (stream kernel).
+// Entry = key(31) << 25 | val(25); EMPTY = ~0 (the table is reset to EMPTY
+// after every use).  A key, once placed, never moves; its val only decreases
+// (atomicMin), so lookups may run while later slots are still inserting.
+// ---------------------------------------------------------------------------
+constexpr unsigned long long CT_EMPTY = ~0ull;
+__device__ __forceinline__ unsigned long long ct_entry(uint32_t key, uint32_t val) {
+  return ((unsigned long long)key << TAB_VAL_BITS) | (unsigned long long)val;
+}
+// Continues an insertion whose first CAS(EMPTY -> mine) at slot h returned old.
+__device__ __forceinline__ void ct_finish(unsigned long long* tab, uint32_t mask, uint32_t h,
+                                          unsigned long long mine, unsigned long long old) {
+  while (true) {
+    if (old == CT_EMPTY) return;                                   // placed
+    if ((old >> TAB_VAL_BITS) == (mine >> TAB_VAL_BITS)) {          // same key
+      if (old > mine) atomicMin(&tab[h], mine);
+      return;
+    }
+    h = (h + 1) & mask;
+    old = atomicCAS(&tab[h], CT_EMPTY, mine);
+  }
+}
+__device__ __forceinline__ int64_t ct_find(const unsigned long long* tab, int log_cap, uint32_t key) {
+  const uint32_t mask = (1u << log_cap) - 1u;
+  uint32_t h = tab_hash(key, log_cap);
+  while (true) {
+    const unsigned long long e = __ldcg(&tab[h]);
+    if (e == CT_EMPTY) return -1;
+    if ((uint32_t)(e >> TAB_VAL_BITS) == key) return (int64_t)h;
+    h = (h + 1) & mask;
+  }
+}
+
+// ---------------------------------------------------------------------------
 // Scans
 // ---------------------------------------------------------------------------
 template <typename T>

@@ -78,6 +78,7 @@ struct gs_blocks {
   std::vector<int64_t> h_meta;
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch
+  unsigned int launch_id = 0;  // per-call tag for device-side flags
   int ws_kind_prev = 0;        // 1 node-wise (tables cleared to ~0), 2 layer-wise (cleared to 0)
   int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow

@@ -168,8 +168,10 @@ __device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t
 // Select for one warp chunk of up to 32 columns [jb, min(jb + 32, jend)) of
 // frontier F (batch-local column j -> padded slots j*k .. j*k+k-1), stage the
 // sampled edges and insert every (u, slot) into the ordered hash (first
-// occurrence = minimum slot).  Returns the chunk's edge count (warp-uniform);
+// occurrence = minimum slot; kFixed: fixed-position CAS table, safe for
+// lookups concurrent with later inserts).  Returns the chunk's edge count (warp-uniform);
 // C.pre / C.cnt_all describe the chunk afterwards.
+template <bool kFixed = false>
 __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk& C, int l, int k,
                                    int log_cap, uint32_t tag, const int32_t* F, int64_t jb,
                                    int64_t jend, uint32_t gb) {
@@ -271,14 +273,22 @@ __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk&
           const float w = P.weights ? __ldg(P.weights + C.coff[cc[i]] + ps[i]) : 1.0f;
           W.val[p[i]] = w / C.csum[cc[i]];
         }
-        carry[i] = tab_entry(tag, (uint32_t)u[i], (uint32_t)p[i]);
         h[i] = tab_hash((uint32_t)u[i], log_cap);
-        old[i] = atomicMin(&W.tab[h[i]], carry[i]);
+        if (kFixed) {
+          carry[i] = ct_entry((uint32_t)u[i], (uint32_t)p[i]);
+          old[i] = atomicCAS(&W.tab[h[i]], CT_EMPTY, carry[i]);
+        } else {
+          carry[i] = tab_entry(tag, (uint32_t)u[i], (uint32_t)p[i]);
+          old[i] = atomicMin(&W.tab[h[i]], carry[i]);
+        }
       }
     }
 #pragma unroll
-    for (int i = 0; i < NW_ILP; ++i)
-      if (ok[i]) otab_finish(W.tab, mask, tag, h[i], carry[i], old[i]);
+    for (int i = 0; i < NW_ILP; ++i) {
+      if (!ok[i]) continue;
+      if (kFixed) ct_finish(W.tab, mask, h[i], carry[i], old[i]);
+      else otab_finish(W.tab, mask, tag, h[i], carry[i], old[i]);
+    }
   }
   __syncwarp();
   return total;
