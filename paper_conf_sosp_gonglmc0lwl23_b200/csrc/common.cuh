@@ -178,6 +178,80 @@ __device__ __forceinline__ int64_t otab_find(const unsigned long long* tab, int 
 }
 
 // ---------------------------------------------------------------------------
+// L2 eviction-priority hints (createpolicy + .L2::cache_hint).  The graph
+// gathers and the block outputs are streams (evict_first); the per-batch
+// workspace (tables, staging) is reused within microseconds (evict_last), so
+// it stays resident in the 126 MB L2 instead of being written back to HBM.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t pol_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t pol_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ int32_t ldh(const int32_t* a, uint64_t p) {
+  int32_t v;
+  asm volatile("ld.global.cg.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint32_t ldh(const uint32_t* a, uint64_t p) {
+  uint32_t v;
+  asm volatile("ld.global.cg.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ int64_t ldh(const int64_t* a, uint64_t p) {
+  int64_t v;
+  asm volatile("ld.global.cg.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ unsigned long long ldh(const unsigned long long* a, uint64_t p) {
+  unsigned long long v;
+  asm volatile("ld.global.cg.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ float ldh(const float* a, uint64_t p) {
+  float v;
+  asm volatile("ld.global.cg.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(a), "l"(p));
+  return v;
+}
+// read-only graph data through the non-coherent path with a hint
+__device__ __forceinline__ int32_t ldg_h(const int32_t* a, uint64_t p) {
+  int32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ float ldg_h(const float* a, uint64_t p) {
+  float v;
+  asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(a), "l"(p));
+  return v;
+}
+__device__ __forceinline__ void sth(int32_t* a, int32_t v, uint64_t p) {
+  asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(p) : "memory");
+}
+__device__ __forceinline__ void sth(uint32_t* a, uint32_t v, uint64_t p) {
+  asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(p) : "memory");
+}
+__device__ __forceinline__ void sth(int64_t* a, int64_t v, uint64_t p) {
+  asm volatile("st.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(a), "l"(v), "l"(p) : "memory");
+}
+__device__ __forceinline__ void sth(unsigned long long* a, unsigned long long v, uint64_t p) {
+  asm volatile("st.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(a), "l"(v), "l"(p) : "memory");
+}
+__device__ __forceinline__ void sth(float* a, float v, uint64_t p) {
+  asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" ::"l"(a), "f"(v), "l"(p) : "memory");
+}
+__device__ __forceinline__ unsigned long long atom_cas_h(unsigned long long* a, unsigned long long cmp,
+                                                         unsigned long long v, uint64_t) {
+  // atom.cas takes no .L2::cache_hint; the table lines get their evict_last
+  // priority from the hinted clears / loads
+  return atomicCAS(a, cmp, v);
+}
+
+// ---------------------------------------------------------------------------
 // Fixed-position table for concurrent insert + lookup (stream kernel).
 // Entry = key(31) << 25 | val(25); EMPTY = ~0 (the table is reset to EMPTY
 // after every use).  A key, once placed, never moves; its val only decreases
@@ -189,7 +263,8 @@ __device__ __forceinline__ unsigned long long ct_entry(uint32_t key, uint32_t va
 }
 // Continues an insertion whose first CAS(EMPTY -> mine) at slot h returned old.
 __device__ __forceinline__ void ct_finish(unsigned long long* tab, uint32_t mask, uint32_t h,
-                                          unsigned long long mine, unsigned long long old) {
+                                          unsigned long long mine, unsigned long long old,
+                                          uint64_t pol) {
   while (true) {
     if (old == CT_EMPTY) return;                                   // placed
     if ((old >> TAB_VAL_BITS) == (mine >> TAB_VAL_BITS)) {          // same key
@@ -197,16 +272,17 @@ __device__ __forceinline__ void ct_finish(unsigned long long* tab, uint32_t mask
       return;
     }
     h = (h + 1) & mask;
-    old = atomicCAS(&tab[h], CT_EMPTY, mine);
+    old = atom_cas_h(&tab[h], CT_EMPTY, mine, pol);
   }
 }
-__device__ __forceinline__ int64_t ct_find(const unsigned long long* tab, int log_cap, uint32_t key) {
+// Entry of key (its val = first slot) or CT_EMPTY when absent.
+__device__ __forceinline__ unsigned long long ct_get(const unsigned long long* tab, int log_cap,
+                                                     uint32_t key, uint64_t pol) {
   const uint32_t mask = (1u << log_cap) - 1u;
   uint32_t h = tab_hash(key, log_cap);
   while (true) {
-    const unsigned long long e = __ldcg(&tab[h]);
-    if (e == CT_EMPTY) return -1;
-    if ((uint32_t)(e >> TAB_VAL_BITS) == key) return (int64_t)h;
+    const unsigned long long e = ldh(&tab[h], pol);
+    if (e == CT_EMPTY || (uint32_t)(e >> TAB_VAL_BITS) == key) return e;
     h = (h + 1) & mask;
   }
 }

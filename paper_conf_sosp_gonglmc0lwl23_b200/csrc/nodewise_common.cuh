@@ -85,8 +85,9 @@ __device__ __forceinline__ int chunk_col(const int32_t* pre, int f) {
 // stream a column's weights, keep the k smallest (key, position), and write
 // the selected positions (ascending) into list[.][c] and the count into
 // cnt_all[c]; csum[c] = fp32(sum_fp64 w over the whole column) (PASS A3).
-__device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t gb, int k,
-                                  int32_t my_v, bool my_valid, int64_t my_off, int64_t my_d) {
+template <typename Out>
+__device__ inline void ares_chunk_t(const NWCore& P, Out out, int l, uint32_t gb, int k,
+                                    int32_t my_v, bool my_valid, int64_t my_off, int64_t my_d) {
   const int G = pow2ceil_int(k);
   const int lane = threadIdx.x & 31;
   const int s = lane & (G - 1), gbase = lane & ~(G - 1);
@@ -156,13 +157,23 @@ __device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t
       rnk += (((selb >> (gbase + i)) & 1u) && pi < bp) ? 1 : 0;
     }
     for (int o = G >> 1; o > 0; o >>= 1) csum += __shfl_xor_sync(FULL, csum, o);
-    if (sel) C.list[rnk][c] = (uint32_t)bp;
-    if (s == 0) {
-      C.cnt_all[c] = __popc(selb);
-      C.csum[c] = (float)csum;
-    }
+    if (sel) out.pos(c, rnk, (uint32_t)bp);
+    if (s == 0) out.col(c, __popc(selb), (float)csum);
   }
   __syncwarp();
+}
+
+struct ChunkOut {
+  WarpChunk* C;
+  __device__ void pos(int c, int r, uint32_t v) const { C->list[r][c] = v; }
+  __device__ void col(int c, int cnt, float cs) const {
+    C->cnt_all[c] = cnt;
+    C->csum[c] = cs;
+  }
+};
+__device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t gb, int k,
+                                  int32_t my_v, bool my_valid, int64_t my_off, int64_t my_d) {
+  ares_chunk_t(P, ChunkOut{&C}, l, gb, k, my_v, my_valid, my_off, my_d);
 }
 
 // Select for one warp chunk of up to 32 columns [jb, min(jb + 32, jend)) of
@@ -174,11 +185,12 @@ __device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t
 template <bool kFixed = false>
 __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk& C, int l, int k,
                                    int log_cap, uint32_t tag, const int32_t* F, int64_t jb,
-                                   int64_t jend, uint32_t gb) {
+                                   int64_t jend, uint32_t gb, unsigned long long* dbg = nullptr) {
   const int lane = threadIdx.x & 31;
+  const uint64_t pf = pol_first(), pl = pol_last();
   const int64_t j = jb + lane;
   const bool active = j < jend;
-  const int32_t v = active ? __ldcg(F + j) : -1;
+  const int32_t v = active ? (kFixed ? ldh(F + j, pl) : __ldcg(F + j)) : -1;
   const bool valid = active && v >= 0 && (int64_t)v < P.N;
   if (active && !valid) atomicOr(P.err, ERR_SEED_RANGE);
   int64_t off = 0, d = 0;
@@ -189,6 +201,11 @@ __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk&
   int cnt = 0;
   bool all = false;
   const bool weighted = !P.replace && P.bias != GS_W_UNIFORM;
+  if (dbg && lane == 0) {
+    unsigned long long tt;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
+    dbg[0] = tt + (unsigned long long)(d & 0);
+  }
   if (weighted) {
     ares_chunk(P, C, l, gb, k, v, valid, off, d);
     cnt = C.cnt_all[lane];
@@ -229,12 +246,22 @@ __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk&
   }
   int total;
   const int pre = warp_excl(cnt, &total);
+  if (dbg && lane == 0) {
+    unsigned long long tt;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
+    dbg[1] = tt;
+  }
   C.coff[lane] = off;
   C.pre[lane] = pre;
   if (!weighted) C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
   if (active) {
-    W.coff[j] = off;
-    W.ccnt[j] = cnt;
+    if (kFixed) {
+      sth(W.coff + j, off, pl);
+      sth(W.ccnt + j, cnt, pl);
+    } else {
+      W.coff[j] = off;
+      W.ccnt[j] = cnt;
+    }
   }
   __syncwarp();
   // Flattened gather + stage + insert: flat slot f of the chunk -> column c, rank s.
@@ -258,7 +285,8 @@ __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk&
         const int s = f - C.pre[c];
         ps[i] = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)s : C.list[s][c];
         p[i] = (jb + c) * k + s;
-        u[i] = __ldg(P.indices + C.coff[c] + ps[i]);
+        u[i] = kFixed ? ldg_h(P.indices + C.coff[c] + ps[i], pf)
+                      : __ldg(P.indices + C.coff[c] + ps[i]);
         cc[i] = c;
       }
     }
@@ -266,31 +294,65 @@ __device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk&
     uint32_t h[NW_ILP];
 #pragma unroll
     for (int i = 0; i < NW_ILP; ++i) {
+      h[i] = 0;
+      carry[i] = 0;
       if (ok[i]) {
-        W.u[p[i]] = u[i];
-        W.pos[p[i]] = ps[i];
+        if (kFixed) {
+          sth(W.u + p[i], u[i], pl);
+          sth(W.pos + p[i], ps[i], pl);
+        } else {
+          W.u[p[i]] = u[i];
+          W.pos[p[i]] = ps[i];
+        }
         if (W.val) {
           const float w = P.weights ? __ldg(P.weights + C.coff[cc[i]] + ps[i]) : 1.0f;
           W.val[p[i]] = w / C.csum[cc[i]];
         }
         h[i] = tab_hash((uint32_t)u[i], log_cap);
-        if (kFixed) {
-          carry[i] = ct_entry((uint32_t)u[i], (uint32_t)p[i]);
-          old[i] = atomicCAS(&W.tab[h[i]], CT_EMPTY, carry[i]);
-        } else {
-          carry[i] = tab_entry(tag, (uint32_t)u[i], (uint32_t)p[i]);
-          old[i] = atomicMin(&W.tab[h[i]], carry[i]);
-        }
+        carry[i] = kFixed ? ct_entry((uint32_t)u[i], (uint32_t)p[i])
+                          : tab_entry(tag, (uint32_t)u[i], (uint32_t)p[i]);
       }
     }
+    if (kFixed) {
+      // Hot rows (hubs) recur in many columns: a CAS per occurrence would
+      // serialise on one L2 address.  Only the first occurrence inside the
+      // warp (lowest lane = smallest slot) proceeds, and it first reads the
+      // home slot: a row already holding a smaller slot needs no atomic.
+      bool go[NW_ILP];
 #pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) {
-      if (!ok[i]) continue;
-      if (kFixed) ct_finish(W.tab, mask, h[i], carry[i], old[i]);
-      else otab_finish(W.tab, mask, tag, h[i], carry[i], old[i]);
+      for (int i = 0; i < NW_ILP; ++i) {
+        const uint32_t peers = __match_any_sync(0xffffffffu, ok[i] ? (uint32_t)u[i] : 0xFFFFFFFFu);
+        go[i] = ok[i] && (__ffs(peers) - 1) == lane;
+        old[i] = go[i] ? ldh(&W.tab[h[i]], pl) : 0ull;
+      }
+#pragma unroll
+      for (int i = 0; i < NW_ILP; ++i) {
+        if (!go[i]) continue;
+        if (old[i] != CT_EMPTY && (old[i] >> TAB_VAL_BITS) == (carry[i] >> TAB_VAL_BITS) &&
+            old[i] <= carry[i]) {
+          go[i] = false;  // present with an earlier slot
+          continue;
+        }
+        old[i] = atom_cas_h(&W.tab[h[i]], CT_EMPTY, carry[i], pl);
+      }
+#pragma unroll
+      for (int i = 0; i < NW_ILP; ++i)
+        if (go[i]) ct_finish(W.tab, mask, h[i], carry[i], old[i], pl);
+    } else {
+#pragma unroll
+      for (int i = 0; i < NW_ILP; ++i)
+        if (ok[i]) old[i] = atomicMin(&W.tab[h[i]], carry[i]);
+#pragma unroll
+      for (int i = 0; i < NW_ILP; ++i)
+        if (ok[i]) otab_finish(W.tab, mask, tag, h[i], carry[i], old[i]);
     }
   }
   __syncwarp();
+  if (dbg && lane == 0) {
+    unsigned long long tt;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
+    dbg[2] = tt;
+  }
   return total;
 }
 

@@ -22,6 +22,9 @@
 // The CTA completing the last tile of a hop writes the block's meta, clears
 // the table and releases the next hop (or the batch) -- all on the device.
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -39,10 +42,17 @@ constexpr int NS_MAXW = 512;            // bitmap words per tile (NS_COLS * MAX_
 
 struct NSBatch {                  // per mini-batch (device), zeroed per launch
   long long T[MAX_LAYERS];        // frontier columns of every hop
-  unsigned int ready[MAX_LAYERS]; // hop l may start (T[l] valid, table clear)
-  unsigned int cnt[MAX_LAYERS];   // tiles of hop l finished (including empty ones)
+  unsigned int ready[MAX_LAYERS]; // unused (kept for layout)
+  unsigned int cnt[MAX_LAYERS];   // tiles of hop l finished
   unsigned int done;              // every hop finished: the window slot is free
   unsigned int pad;
+};
+
+// A hop job: hop l of batch b, ntiles tiles, occupying tickets [start, start + nt).
+struct NSJob {
+  long long start;
+  int b, l, nt;
+  unsigned int ready;
 };
 
 struct NSParams {
@@ -52,11 +62,8 @@ struct NSParams {
   int L;
   int k[MAX_LAYERS];
   int64_t K[MAX_LAYERS];
-  int maxtiles[MAX_LAYERS];  // tile budget of hop l (bound on its frontier / NS_COLS)
-  int tile_off[MAX_LAYERS];  // position of hop l's tiles inside a step (deepest first)
-  int tps;                   // tickets per step
-  int64_t nsteps;
-  int win;                   // window slots (> (L-1) * NS_LAG)
+  int maxtiles[MAX_LAYERS];  // bound on the tiles of hop l (frontier bound / NS_COLS)
+  int win;                   // window slots = mini-batches in flight
   int32_t* col0;
   int32_t* row_map[MAX_LAYERS];
   int64_t* indptr_out[MAX_LAYERS];
@@ -65,13 +72,18 @@ struct NSParams {
   float* val[MAX_LAYERS];
   int64_t* meta;
   NSBatch* bs;
-  unsigned long long* ticket;
+  unsigned long long* ticket;   // [0] head (claimed tickets), [1] tail (jobs << 40 | tickets),
+                                // [2] finished batches
+  NSJob* jobs;
   char* ws;
   int64_t ws_stride;
   int64_t o_u, o_pos, o_val, o_coff, o_ccnt, o_ceoff, o_bits, o_wpre, o_tab;
   int64_t o_sel, o_agg, o_rx;  // per (hop, tile) look-back state
+  int64_t o_first;             // direct first-slot array [N]
   int max_tiles_all;           // max over l of maxtiles[l]
   unsigned int launch;         // per-call id (tags of the look-back state)
+  unsigned long long* trace;   // optional: [tickets][8] globaltimer checkpoints (GS_TRACE)
+  unsigned long long* trace2;  // optional: [tickets][4] select sub-steps of warp 0
   int log_tab_cap;
 };
 
@@ -80,6 +92,7 @@ struct NSSlot {
   int32_t* ceoff;
   uint32_t* bits;
   int32_t* wpre;
+  uint32_t* first;          // [N] first slot of every row in the current hop (~0 = none)
   unsigned long long* sel;  // [L][maxt] = batch + 1 once the tile's inserts are done
   unsigned long long* lbs;  // [L][maxt] look-back status word
   unsigned long long* lba;  // [L][maxt] aggregate (edges, rows)
@@ -99,6 +112,7 @@ __device__ __forceinline__ NSSlot ns_slot(const NSParams& P, int64_t b) {
   s.ceoff = (int32_t*)(base + P.o_ceoff);
   s.bits = (uint32_t*)(base + P.o_bits);
   s.wpre = (int32_t*)(base + P.o_wpre);
+  s.first = (uint32_t*)(base + P.o_first);
   s.sel = (unsigned long long*)(base + P.o_sel);
   s.lbs = (unsigned long long*)(base + P.o_agg);
   s.lba = s.lbs + (int64_t)P.L * P.max_tiles_all;
@@ -121,11 +135,22 @@ __device__ __forceinline__ unsigned long long lb_pack(int64_t e, int64_t r) {
 __device__ __forceinline__ int64_t lb_e(unsigned long long v) { return (int64_t)(v >> 32); }
 __device__ __forceinline__ int64_t lb_r(unsigned long long v) { return (int64_t)(v & 0xFFFFFFFFull); }
 
+constexpr int NS_SLOTS = 6144;            // slots of one tile kept in shared memory
+constexpr int NS_SROW = NS_SLOTS + 512;   // padded rows (odd stride) of the tile's slots
+
 struct NSSmem {
-  WarpChunk wc[NS_WARPS];
+  uint32_t su[NS_SROW];     // sampled row of tile slot q = column * ks + rank
+  uint32_t spos[NS_SROW];   // position inside the column
+  uint32_t sp0[NS_SROW];    // first slot (batch-hop slot id) of the slot's row
+  int64_t scoff[NS_COLS];   // indptr[v] of the tile's columns
+  int32_t scnt[NS_COLS];    // sampled edges per column
+  int32_t sceo[NS_COLS];    // tile-local edge offset per column
+  float scsum[NS_COLS];     // PASS column sums
+  uint32_t sbits[NS_MAXW];  // first-occurrence bitmap of the tile's words
+  int32_t swpre[NS_MAXW];   // tile-local count of first slots before each word
+  int32_t spre[NS_WARPS][32];
   int wtot[NS_WARPS];
-  int wcnt[NS_MAXW];
-  long long x[4];   // exclusive edges / rows of this tile, totals
+  long long x[4];
   long long job[4];
   int flag;
 };
@@ -147,175 +172,314 @@ __device__ __forceinline__ void st_rel_u64(unsigned long long* p, unsigned long 
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+// Polling with exponential backoff: spinning threads must not turn a flag's
+// L2 slice into a hot spot that every other request queues behind.
+struct Backoff {
+  unsigned int ns = 64;
+  __device__ __forceinline__ void wait() {
+    __nanosleep(ns);
+    ns = ns < 4096u ? ns * 2u : 4096u;
+  }
+};
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+struct NSSmem;
+__device__ void ns_hop_done(const NSParams& P, NSSmem& sm, int64_t b, int l, int64_t T, int64_t E, int64_t R);
+
+// Tile geometry of a hop with fanout k: rows of the shared-memory slot arrays
+// have an odd stride ks (conflict-free per-lane rows), and a tile has as many
+// 32-column chunks as fit NS_SLOTS slots (at most NS_COLS columns).
+__device__ __forceinline__ int ns_ks(int k) { return k | 1; }
+__device__ __forceinline__ int ns_tile_cols(int k) {
+  const int chunks = NS_SLOTS / (ns_ks(k) * 32);
+  return min(NS_COLS, max(1, chunks) * 32);
+}
+
 __device__ __forceinline__ int ns_log_cap(const NSParams& P, int64_t T, int k) {
   const int lc = log2_pow2ceil64((T * k * 4) / 3 + 64);
   return lc > P.log_tab_cap ? P.log_tab_cap : lc;
 }
 
+struct RowOut {  // A-Res output into the tile's shared-memory rows
+  uint32_t* spos;
+  int32_t* scnt;
+  float* scsum;
+  int base, ks;
+  __device__ void pos(int c, int r, uint32_t v) const { spos[(base + c) * ks + r] = v; }
+  __device__ void col(int c, int cnt, float cs) const {
+    scnt[base + c] = cnt;
+    scsum[base + c] = cs;
+  }
+};
+
 // The tile: (batch b, hop l, tile t).  All threads of the CTA.
-__device__ void ns_tile(const NSParams& P, NSSmem& sm, int64_t b, int l, int t) {
+__device__ void ns_tile(const NSParams& P, NSSmem& sm, int64_t b, int l, int t, unsigned long long tk) {
+  unsigned long long* trc = P.trace ? P.trace + tk * 8 : nullptr;
+  if (trc && threadIdx.x == 0) { trc[0] = gtimer(); trc[7] = ((unsigned long long)b << 16) | ((unsigned long long)l << 12) | (unsigned long long)t; }
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t bstart = b * P.batch_size;
   NSBatch& B = P.bs[b];
-  // ---- 0. wait for the inputs of this hop ----
-  if (threadIdx.x == 0) {
-    if (l == 0) {
-      if (b >= P.win) {  // the window slot must be free
-        while (ld_acq_u32(&P.bs[b - P.win].done) == 0u) __nanosleep(64);
-      }
-    } else {
-      while (ld_acq_u32(&B.ready[l]) == 0u) __nanosleep(64);
-    }
-  }
-  __syncthreads();
-  const int64_t T = l == 0 ? min(P.batch_size, P.num_seeds - bstart) : __ldcg(&B.T[l]);
+  if (trc && threadIdx.x == 0) trc[1] = gtimer();
+  // the job was appended only once its inputs were complete: no waiting here
+  const int64_t T = __ldcg(&B.T[l]);
   const int k = P.k[l];
-  const int ntiles = (int)((T + NS_COLS - 1) / NS_COLS);
+  const int ks = ns_ks(k);
+  const int TC = ns_tile_cols(k);
+  const int ntiles = (int)((T + TC - 1) / TC);
   const NSSlot S = ns_slot(P, b);
-  const int log_cap = ns_log_cap(P, T, k);
-  const uint32_t tag = 0u;  // tables are cleared after every hop
+  const uint64_t pf = pol_first(), pl = pol_last();
   // (launch, batch) tag of the per-tile flags: stale values from earlier
   // batches in this window slot or from earlier launches never match
   const unsigned long long btag = ((unsigned long long)P.launch << 32) | (unsigned long long)(b + 1);
-  if (t < ntiles) {
-    const uint32_t gb = (uint32_t)(P.batch_base + b);
-    const int32_t* F = l == 0 ? P.seeds + bstart : P.row_map[l - 1] + bstart * P.K[l - 1];
-    const int64_t tend = min(T, (int64_t)(t + 1) * NS_COLS);
-    const int64_t jb = (int64_t)t * NS_COLS + warp * 32;
-    // ---- 1. Extract + Select + stage + insert ----
-    int e = 0, pre = 0;
-    if (jb < tend) {
-      e = select_chunk<true>(P.core, S.stg, sm.wc[warp], l, k, log_cap, tag, F, jb, tend, gb);
-      pre = sm.wc[warp].pre[lane];
+  const uint32_t gb = (uint32_t)(P.batch_base + b);
+  const int32_t* F = l == 0 ? P.seeds + bstart : P.row_map[l - 1] + bstart * P.K[l - 1];
+  const int64_t c0 = (int64_t)t * TC;                 // first column of the tile
+  const int ncols = (int)min((int64_t)TC, T - c0);    // columns of this tile
+  const int64_t p_base = c0 * k;                      // first batch-hop slot of the tile
+  const int nslots = ncols * k;
+  const int nwords = (nslots + 31) >> 5;
+  const bool weighted = !P.core.replace && P.core.bias != GS_W_UNIFORM;
+
+  // ---- 1. Extract + Select: positions into shared memory rows ----
+  const int nchunks = (ncols + 31) >> 5;
+  for (int ch = warp; ch < nchunks; ch += NS_WARPS) {
+    const int jl = ch * 32 + lane;
+    const bool active = jl < ncols;
+    const int32_t v = active ? ldh(F + c0 + jl, pl) : -1;
+    const bool valid = active && v >= 0 && (int64_t)v < P.core.N;
+    if (active && !valid) atomicOr(P.core.err, ERR_SEED_RANGE);
+    int64_t off = 0, d = 0;
+    if (valid) {
+      off = __ldg(P.core.indptr + v);
+      d = __ldg(P.core.indptr + v + 1) - off;
     }
-    if (lane == 0) sm.wtot[warp] = e;
-    __syncthreads();
-    if (warp == 0) {
-      const int v = lane < NS_WARPS ? sm.wtot[lane] : 0;
-      int tot;
-      const int ex = warp_excl(v, &tot);
-      if (lane < NS_WARPS) sm.wtot[lane] = ex;
-      if (lane == 0) sm.x[2] = tot;  // tile edges
-    }
-    __syncthreads();
-    if (jb + lane < tend) S.ceoff[jb + lane] = sm.wtot[warp] + pre;
-    __syncthreads();
-    const int maxt = P.max_tiles_all;
-    unsigned long long* sel = S.sel + (int64_t)l * maxt;
-    unsigned long long* lbs = S.lbs + (int64_t)l * maxt;
-    unsigned long long* lba = S.lba + (int64_t)l * maxt;
-    unsigned long long* lbp = S.lbp + (int64_t)l * maxt;
-    long long* rx = S.rx + (int64_t)l * maxt;
-    if (threadIdx.x == 0) {
-      __threadfence();
-      st_rel_u64(&sel[t], btag);
-    }
-    // ---- 2. wait for the inserts of every earlier tile ----
-    if (warp == 0) {
-      for (int t0 = lane; t0 < t; t0 += 32)
-        while (ld_acq_u64(&sel[t0]) != btag) __nanosleep(32);
+    uint32_t* row = &sm.spos[jl * ks];
+    int cnt = 0;
+    if (weighted) {
+      ares_chunk_t(P.core, RowOut{sm.spos, sm.scnt, sm.scsum, ch * 32, ks}, l, gb, k, v, valid,
+                   off, d);
       __syncwarp();
-    }
-    __syncthreads();
-    // ---- 3. first-occurrence bitmap of this tile's slots ----
-    const int64_t PT = T * k;
-    const int64_t wbase = ((int64_t)t * NS_COLS * k) >> 5;   // first word of the tile
-    const int64_t wend = min((PT + 31) >> 5, wbase + (int64_t)NS_COLS * k / 32);
-    const int wpw = k;                                        // words per warp
-    const int64_t w0 = wbase + (int64_t)warp * wpw;
-    int wrun = 0;
-    for (int i0 = 0; i0 < wpw; i0 += NW_ILP) {
-      uint32_t uu[NW_ILP];
-      bool vv[NW_ILP];
-      int64_t hh[NW_ILP];
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i) {
-        const int64_t wd = w0 + i0 + i;
-        const int64_t p = wd * 32 + lane;
-        vv[i] = false;
-        if (i0 + i < wpw && wd < wend && p < PT) {
-          const int64_t j = p / k;
-          vv[i] = (p - j * k) < __ldcg(S.stg.ccnt + j);
-        }
-        uu[i] = vv[i] ? (uint32_t)__ldcg(S.stg.u + p) : 0u;
+      cnt = active ? sm.scnt[jl] : 0;
+    } else if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
+      cnt = d > 0 ? k : 0;
+      for (int s = 0; s < cnt; ++s) {
+        const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
+        row[s] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
       }
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i)
-        hh[i] = vv[i] ? ct_find(S.stg.tab, log_cap, uu[i]) : -1;
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i) {
-        const int64_t wd = w0 + i0 + i;
-        const int64_t p = wd * 32 + lane;
-        bool first = false;
-        if (vv[i]) {
-          if (hh[i] < 0) atomicOr(P.core.err, ERR_INTERNAL);
-          else first = tab_val(__ldcg(S.stg.tab + hh[i])) == (uint32_t)p;
+    } else if (d <= k) {  // GraphSAGE, d <= k: every neighbour (R5)
+      cnt = (int)d;
+      for (int s = 0; s < cnt; ++s) row[s] = (uint32_t)s;
+    } else {  // GraphSAGE (R5): Floyd, the row kept sorted (m is always appended)
+      cnt = k;
+      int nn = 0;
+      for (int s = 0; s < k; ++s) {
+        const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.core.key);
+        const uint32_t m = (uint32_t)(d - k + s);
+        const uint32_t tt = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
+        int lo = 0, hi = nn;
+        while (lo < hi) {
+          const int mid = (lo + hi) >> 1;
+          if (row[mid] < tt) lo = mid + 1;
+          else hi = mid;
         }
-        const uint32_t word = __ballot_sync(0xffffffffu, first);
-        if (i0 + i < wpw) {
-          if (wd < wend && lane == 0) S.bits[wd] = word;
-          if (lane == 0) sm.wcnt[warp * wpw + i0 + i] = __popc(word);
-          wrun += __popc(word);
+        if (lo < nn && row[lo] == tt) {
+          row[nn] = m;
+        } else {
+          for (int q = nn; q > lo; --q) row[q] = row[q - 1];
+          row[lo] = tt;
         }
+        ++nn;
       }
     }
-    if (lane == 0) sm.wtot[warp] = wrun;
-    __syncthreads();
-    if (warp == 0) {
-      const int v = lane < NS_WARPS ? sm.wtot[lane] : 0;
+    if (active) {
+      sm.scoff[jl] = off;
+      sm.scnt[jl] = cnt;
+    }
+    int total;
+    const int pre = warp_excl(cnt, &total);
+    sm.spre[warp][lane] = pre;
+    if (active) sm.sceo[jl] = pre;  // chunk-local edge offset of the column
+    __syncwarp();
+    // flattened gather: every sampled row of the chunk is requested at once
+    // with cp.async straight into shared memory (no register cap on the
+    // number of random HBM sectors in flight)
+    for (int f = lane; f < total; f += 32) {
+      const int c = chunk_col(sm.spre[warp], f);
+      const int s = f - sm.spre[warp][c];
+      const int jc = ch * 32 + c;
+      const int qq = jc * ks + s;
+      const int32_t* src = P.core.indices + sm.scoff[jc] + sm.spos[qq];
+      const unsigned dst = (unsigned)__cvta_generic_to_shared(&sm.su[qq]);
+      asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
+                   "l"(src), "l"(pf)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    __syncwarp();
+    // first occurrence: first[u] = min over the slots holding row u.  A
+    // fire-and-forget red.min (no return, no probing); inside a warp only the
+    // lowest lane (= smallest slot) of each row issues it (hub rows recur).
+    for (int f = lane; f - lane < total; f += 32) {
+      const bool ok = f < total;
+      uint32_t u = 0xFFFFFFFFu, pslot = 0;
+      if (ok) {
+        const int c = chunk_col(sm.spre[warp], f);
+        const int s = f - sm.spre[warp][c];
+        const int jc = ch * 32 + c;
+        pslot = (uint32_t)(p_base + (int64_t)jc * k + s);
+        u = sm.su[jc * ks + s];
+      }
+      const uint32_t peers = __match_any_sync(0xffffffffu, u);
+      if (ok && (__ffs(peers) - 1) == lane)
+        asm volatile("red.global.min.u32 [%0], %1;" ::"l"(S.first + u), "r"(pslot) : "memory");
+    }
+    if (lane == 0) sm.wtot[warp] = total;
+  }
+  if (warp >= nchunks && lane == 0) sm.wtot[warp] = 0;  // nchunks <= NS_WARPS
+  __syncthreads();
+  if (warp == 0) {  // chunk edge totals -> tile-local column offsets
+    const int v = lane < NS_WARPS ? sm.wtot[lane] : 0;
+    int tot;
+    const int ex = warp_excl(v, &tot);
+    if (lane < NS_WARPS) sm.wtot[lane] = ex;
+    if (lane == 0) sm.x[2] = tot;  // tile edges
+  }
+  __syncthreads();
+  for (int jl = threadIdx.x; jl < ncols; jl += blockDim.x) sm.sceo[jl] += sm.wtot[jl >> 5];
+  const int maxt = P.max_tiles_all;
+  unsigned long long* sel = S.sel + (int64_t)l * maxt;
+  unsigned long long* lbs = S.lbs + (int64_t)l * maxt;
+  unsigned long long* lba = S.lba + (int64_t)l * maxt;
+  unsigned long long* lbp = S.lbp + (int64_t)l * maxt;
+  long long* rx = S.rx + (int64_t)l * maxt;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    st_rel_u64(&sel[t], btag);
+    if (trc) trc[2] = gtimer();
+  }
+  // ---- 2. wait for the inserts of every earlier tile ----
+  if (threadIdx.x == 0) {  // newest first: when t-1 is done, older ones usually are
+    for (int t0 = t - 1; t0 >= 0; --t0) {
+      Backoff bo;
+      while (ld_acq_u64(&sel[t0]) != btag) bo.wait();
+    }
+  }
+  __syncthreads();
+  if (trc && threadIdx.x == 0) trc[3] = gtimer();
+  // ---- 3. first-occurrence bitmap of this tile's slots (word-major) ----
+  const int wpw = (nwords + NS_WARPS - 1) / NS_WARPS;
+  const int wa = warp * wpw, wz = min(nwords, wa + wpw);
+  int wrun = 0;
+  for (int w0 = wa; w0 < wz; w0 += NW_ILP) {
+    uint32_t uu[NW_ILP], qq[NW_ILP];
+    bool vv[NW_ILP];
+    unsigned long long ee[NW_ILP];
+#pragma unroll
+    for (int i = 0; i < NW_ILP; ++i) {
+      const int r = (w0 + i) * 32 + lane;  // tile-local slot rank
+      vv[i] = false;
+      qq[i] = 0u;
+      if (w0 + i < wz && r < nslots) {
+        const int jl = r / k, s = r - jl * k;
+        vv[i] = s < sm.scnt[jl];
+        qq[i] = (uint32_t)(jl * ks + s);
+      }
+      uu[i] = vv[i] ? sm.su[qq[i]] : 0u;
+    }
+#pragma unroll
+    for (int i = 0; i < NW_ILP; ++i) ee[i] = vv[i] ? (unsigned long long)ldh(S.first + uu[i], pl) : 0ull;
+#pragma unroll
+    for (int i = 0; i < NW_ILP; ++i) {
+      const int wl = w0 + i;
+      const int64_t p = p_base + (int64_t)wl * 32 + lane;
+      bool first = false;
+      if (vv[i]) {
+        const uint32_t p0 = (uint32_t)ee[i];
+        if (p0 > (uint32_t)p) atomicOr(P.core.err, ERR_INTERNAL);
+        sm.sp0[qq[i]] = p0;
+        first = p0 == (uint32_t)p;
+      }
+      const uint32_t word = __ballot_sync(0xffffffffu, first);
+      if (wl < wz) {
+        if (lane == 0) {
+          sm.sbits[wl] = word;
+          sm.swpre[wl] = __popc(word);
+          sth(S.bits + (p_base >> 5) + wl, word, pl);
+        }
+        wrun += __popc(word);
+      }
+    }
+  }
+  if (lane == 0) sm.wtot[warp] = wrun;
+  __syncthreads();
+  if (warp == 0) {
+    const int v = lane < NS_WARPS ? sm.wtot[lane] : 0;
+    int tot;
+    const int ex = warp_excl(v, &tot);
+    if (lane < NS_WARPS) sm.wtot[lane] = ex;
+    if (lane == 0) sm.x[3] = tot;  // tile rows (first occurrences)
+  }
+  __syncthreads();
+  {  // per-word tile-local prefix (shared + global for later tiles)
+    int run = sm.wtot[warp];
+    for (int i0 = wa; i0 < wz; i0 += 32) {
+      const int i = i0 + lane;
+      const int c = i < wz ? sm.swpre[i] : 0;
       int tot;
-      const int ex = warp_excl(v, &tot);
-      if (lane < NS_WARPS) sm.wtot[lane] = ex;
-      if (lane == 0) sm.x[3] = tot;  // tile rows
-    }
-    __syncthreads();
-    {  // per-word tile-local prefix
-      int run = sm.wtot[warp];
-      for (int i0 = 0; i0 < wpw; i0 += 32) {
-        const int i = i0 + lane;
-        const int c = i < wpw ? sm.wcnt[warp * wpw + i] : 0;
-        int tot;
-        const int ex = warp_excl(c, &tot);
-        if (i < wpw && w0 + i < wend) S.wpre[w0 + i] = run + ex;
-        run += tot;
+      const int ex = warp_excl(c, &tot);
+      if (i < wz) {
+        sm.swpre[i] = run + ex;
+        sth(S.wpre + (p_base >> 5) + i, run + ex, pl);
       }
+      run += tot;
     }
-    // ---- 4. decoupled look-back over the hop's tiles ----
-    if (threadIdx.x == 0) {
-      const int64_t te = sm.x[2], tr = sm.x[3];
+  }
+  // ---- 4. decoupled look-back over the hop's tiles ----
+  if (threadIdx.x == 0) {
+    if (trc) trc[4] = gtimer();
+    const int64_t te = sm.x[2], tr = sm.x[3];
+    __threadfence();
+    int64_t xe = 0, xr = 0;
+    if (t > 0) {
+      lba[t] = lb_pack(te, tr);
       __threadfence();
-      int64_t xe = 0, xr = 0;
-      if (t > 0) {
-        lba[t] = lb_pack(te, tr);
-        __threadfence();
-        st_rel_u64(&lbs[t], lb_status_word(btag, LB_A));
-        for (int t0 = t - 1; t0 >= 0;) {
-          const unsigned long long w = ld_acq_u64(&lbs[t0]);
-          if (w == lb_status_word(btag, LB_P)) {
-            const unsigned long long v = __ldcg(&lbp[t0]);
-            xe += lb_e(v);
-            xr += lb_r(v);
-            break;
-          }
-          if (w == lb_status_word(btag, LB_A)) {
-            const unsigned long long v = __ldcg(&lba[t0]);
-            xe += lb_e(v);
-            xr += lb_r(v);
-            --t0;
-            continue;
-          }
-          __nanosleep(32);
+      st_rel_u64(&lbs[t], lb_status_word(btag, LB_A));
+      Backoff bo;
+      for (int t0 = t - 1; t0 >= 0;) {
+        const unsigned long long w = ld_acq_u64(&lbs[t0]);
+        if (w == lb_status_word(btag, LB_P)) {
+          const unsigned long long v = __ldcg(&lbp[t0]);
+          xe += lb_e(v);
+          xr += lb_r(v);
+          break;
         }
+        if (w == lb_status_word(btag, LB_A)) {
+          const unsigned long long v = __ldcg(&lba[t0]);
+          xe += lb_e(v);
+          xr += lb_r(v);
+          --t0;
+          continue;
+        }
+        bo.wait();
       }
-      rx[t] = xr;
-      lbp[t] = lb_pack(xe + te, xr + tr);
-      __threadfence();
-      st_rel_u64(&lbs[t], lb_status_word(btag, LB_P));
-      sm.x[0] = xe;
-      sm.x[1] = xr;
     }
-    __syncthreads();
-    // ---- 5. relabel + compaction ----
+    rx[t] = xr;
+    lbp[t] = lb_pack(xe + te, xr + tr);
+    __threadfence();
+    st_rel_u64(&lbs[t], lb_status_word(btag, LB_P));
+    sm.x[0] = xe;
+    sm.x[1] = xr;
+    if (trc) trc[5] = gtimer();
+  }
+  __syncthreads();
+  // ---- 5. relabel + compaction (word-major over the tile's slots) ----
+  {
     const int64_t xe = sm.x[0], xr = sm.x[1];
     const int64_t colbase = l == 0 ? bstart : bstart * P.K[l - 1];
     const int64_t rbase = bstart * P.K[l];
@@ -324,145 +488,186 @@ __device__ void ns_tile(const NSParams& P, NSSmem& sm, int64_t b, int l, int t) 
     int32_t* row_local = P.row_local[l] + rbase;
     int64_t* eid_out = P.eid[l] + rbase;
     float* val_out = P.val[l] ? P.val[l] + rbase : nullptr;
-    const int tile_slots = NS_COLS * k;
-    if (jb < tend) {
-      WarpChunk& C = sm.wc[warp];
-      const int64_t j = jb + lane;
-      const bool act = j < tend;
-      const int cnt = act ? __ldcg(S.stg.ccnt + j) : 0;
-      const int eo = act ? __ldcg(S.ceoff + j) : 0;
-      const int64_t off = act ? __ldcg(S.stg.coff + j) : 0;
-      int total;
-      const int cpre = warp_excl(cnt, &total);
-      C.pre[lane] = cpre;
-      C.coff[lane] = off;
-      C.cnt_all[lane] = eo;
-      if (act) {
-        P.indptr_out[l][ibase + j] = xe + eo;
-        if (l == 0) P.col0[bstart + j] = __ldcg(P.seeds + bstart + j);
+    const int tile_slots = TC * k;
+    for (int jl = threadIdx.x; jl < ncols; jl += blockDim.x) {
+      sth(P.indptr_out[l] + ibase + c0 + jl, (int64_t)(xe + sm.sceo[jl]), pf);
+      if (l == 0) sth(P.col0 + bstart + c0 + jl, __ldcg(P.seeds + bstart + c0 + jl), pf);
+    }
+    for (int r = threadIdx.x; r < nslots; r += blockDim.x) {
+      const int jl = r / k, s = r - jl * k;
+      if (s >= sm.scnt[jl]) continue;
+      const int q = jl * ks + s;
+      const int64_t p = p_base + r;
+      const uint32_t p0 = sm.sp0[q];
+      const int64_t e = xe + sm.sceo[jl] + s;
+      const int64_t eid = sm.scoff[jl] + sm.spos[q];
+      int64_t lid;
+      if ((int64_t)p0 >= p_base) {
+        const int wl = (int)((p0 - p_base) >> 5);
+        lid = xr + sm.swpre[wl] + __popc(sm.sbits[wl] & ((1u << (p0 & 31)) - 1u));
+      } else {  // first occurrence in an earlier tile: wait for its prefix
+        const int t0 = (int)(p0 / (uint32_t)tile_slots);
+        Backoff bo;
+        while (ld_acq_u64(&lbs[t0]) != lb_status_word(btag, LB_P)) bo.wait();
+        const int64_t wd = p0 >> 5;
+        lid = __ldcg(rx + t0) + ldh(S.wpre + wd, pl) +
+              __popc(ldh(S.bits + wd, pl) & ((1u << (p0 & 31)) - 1u));
       }
-      __syncwarp();
-      for (int f0 = 0; f0 < total; f0 += 32 * NW_ILP) {
-        int64_t p[NW_ILP], ee[NW_ILP], hh[NW_ILP];
-        uint32_t uu[NW_ILP], ps[NW_ILP];
-        int cc[NW_ILP];
-        bool ok[NW_ILP];
-#pragma unroll
-        for (int i = 0; i < NW_ILP; ++i) {
-          const int f = f0 + i * 32 + lane;
-          ok[i] = f < total;
-          cc[i] = 0;
-          p[i] = ee[i] = 0;
-          uu[i] = ps[i] = 0;
-          if (ok[i]) {
-            const int c = chunk_col(C.pre, f);
-            const int s = f - C.pre[c];
-            p[i] = (jb + c) * k + s;
-            ee[i] = xe + C.cnt_all[c] + s;
-            uu[i] = (uint32_t)__ldcg(S.stg.u + p[i]);
-            ps[i] = __ldcg(S.stg.pos + p[i]);
-            cc[i] = c;
-          }
-        }
-#pragma unroll
-        for (int i = 0; i < NW_ILP; ++i) {
-          hh[i] = -1;
-          if (ok[i]) {
-            eid_out[ee[i]] = C.coff[cc[i]] + ps[i];
-            if (val_out) val_out[ee[i]] = __ldcg(S.stg.val + p[i]);
-            hh[i] = ct_find(S.stg.tab, log_cap, uu[i]);
-          }
-        }
-#pragma unroll
-        for (int i = 0; i < NW_ILP; ++i) {
-          if (ok[i]) {
-            const uint32_t p0 = hh[i] >= 0 ? tab_val(__ldcg(S.stg.tab + hh[i])) : 0u;
-            const int t0 = (int)(p0 / (uint32_t)tile_slots);
-            long long base;
-            if (t0 == t) {
-              base = xr;
-            } else {  // the first slot is in an earlier tile: wait for its prefix
-              while (ld_acq_u64(&lbs[t0]) != lb_status_word(btag, LB_P)) __nanosleep(32);
-              base = __ldcg(rx + t0);
-            }
-            const int64_t wd = p0 >> 5;
-            const uint32_t bw = __ldcg(S.bits + wd);
-            const int64_t lid = base + __ldcg(S.wpre + wd) + __popc(bw & ((1u << (p0 & 31)) - 1u));
-            row_local[ee[i]] = (int32_t)lid;
-            if (p0 == (uint32_t)p[i]) row_map[lid] = (int32_t)uu[i];
-          }
-        }
+      sth(row_local + e, (int32_t)lid, pf);
+      sth(eid_out + e, eid, pf);
+      if (val_out) {
+        const float w = P.core.weights ? __ldg(P.core.weights + eid) : 1.0f;
+        sth(val_out + e, w / sm.scsum[jl], pf);
       }
-      __syncwarp();
+      if ((int64_t)p0 == p) sth(row_map + lid, (int32_t)sm.su[q], pf);
     }
   }
   // ---- 6. completion of the hop ----
   __syncthreads();
+  if (trc && threadIdx.x == 0) trc[6] = gtimer();
   if (threadIdx.x == 0) {
     __threadfence();
     const unsigned int d = atomicAdd(&B.cnt[l], 1u) + 1u;
-    sm.flag = (d == (unsigned int)P.maxtiles[l]);
+    sm.flag = (d == (unsigned int)ntiles);
     if (sm.flag) {
       __threadfence();
-      int64_t E = 0, R = 0;
-      if (ntiles > 0) {
-        const int64_t i = (int64_t)l * P.max_tiles_all + ntiles - 1;
-        while (ld_acq_u64(&S.lbs[i]) != lb_status_word(btag, LB_P)) __nanosleep(32);
-        const unsigned long long v = __ldcg(&S.lbp[i]);
-        E = lb_e(v);
-        R = lb_r(v);
-      }
-      sm.x[2] = E;
-      sm.x[3] = R;
+      const int64_t i = (int64_t)l * P.max_tiles_all + ntiles - 1;
+      Backoff bo;
+      while (ld_acq_u64(&S.lbs[i]) != lb_status_word(btag, LB_P)) bo.wait();
+      const unsigned long long v = __ldcg(&S.lbp[i]);
+      sm.x[2] = lb_e(v);
+      sm.x[3] = lb_r(v);
     }
   }
   __syncthreads();
-  if (sm.flag) {
-    // clear this hop's part of the table for the next user of the slot
-    const int64_t cap = 1ll << log_cap;
-    for (int64_t i = threadIdx.x; i < cap; i += blockDim.x) S.stg.tab[i] = ~0ull;
-    __syncthreads();
+  if (sm.flag) ns_hop_done(P, sm, b, l, T, sm.x[2], sm.x[3]);
+}
+
+// Appends hop job (b, l) with nt tiles (thread 0).
+__device__ void ns_append(const NSParams& P, int64_t b, int l, int nt) {
+  const unsigned long long old = atomicAdd(P.ticket + 1, (1ull << 40) | (unsigned long long)nt);
+  const int64_t j = (int64_t)(old >> 40);
+  NSJob& J = P.jobs[j];
+  J.start = (long long)(old & ((1ull << 40) - 1));
+  J.b = (int)b;
+  J.l = l;
+  J.nt = nt;
+  __threadfence();
+  st_rel_u32(&J.ready, 1u);
+}
+
+// Makes hop l of batch b (T columns) runnable, finishing empty hops on the spot.
+__device__ void ns_start_hop(const NSParams& P, NSSmem& sm, int64_t b, int l, int64_t T);
+
+// Hop l of batch b is complete (CTA-wide): write the block's meta, scrub the
+// scratch (clear the table, discard dead staging lines from L2 without
+// write-back) and release the next hop or the next batch of the window slot.
+__device__ void ns_hop_done(const NSParams& P, NSSmem& sm, int64_t b, int l, int64_t T,
+                            int64_t E, int64_t R) {
+  const NSSlot S = ns_slot(P, b);
+  const int k = P.k[l];
+  const uint64_t pl = pol_last();
+  // reset first[u] of exactly the rows this hop touched (its row_map), so the
+  // array is all ~0 for the next hop / the next batch of this window slot
+  if (R > 0) {
+    const int32_t* rows = P.row_map[l] + b * P.batch_size * P.K[l];
+    for (int64_t i = threadIdx.x; i < R; i += blockDim.x)
+      sth(S.first + __ldcg(rows + i), 0xFFFFFFFFu, pl);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const int64_t bstart = b * P.batch_size;
+    const int64_t colbase = l == 0 ? bstart : bstart * P.K[l - 1];
+    const int64_t rbase = bstart * P.K[l];
+    const int64_t ibase = colbase + b;
+    P.indptr_out[l][ibase + T] = E;
+    long long* m = (long long*)(P.meta + (b * P.L + l) * 8);
+    m[0] = T; m[1] = R; m[2] = E; m[3] = colbase; m[4] = rbase; m[5] = ibase; m[6] = rbase;
+    m[7] = 0;
+    __threadfence();
+  }
+  if (l + 1 < P.L) {
+    ns_start_hop(P, sm, b, l + 1, R);
+  } else {
     if (threadIdx.x == 0) {
-      const int64_t E = sm.x[2], R = sm.x[3];
-      const int64_t colbase = l == 0 ? bstart : bstart * P.K[l - 1];
-      const int64_t rbase = bstart * P.K[l];
-      const int64_t ibase = colbase + b;
-      P.indptr_out[l][ibase + T] = E;
-      long long* m = (long long*)(P.meta + (b * P.L + l) * 8);
-      m[0] = T; m[1] = R; m[2] = E; m[3] = colbase; m[4] = rbase; m[5] = ibase; m[6] = rbase;
-      m[7] = 0;
-      __threadfence();
-      if (l + 1 < P.L) {
-        B.T[l + 1] = R;
-        __threadfence();
-        st_rel_u32(&B.ready[l + 1], 1u);
-      } else {
-        st_rel_u32(&B.done, 1u);
-      }
+      st_rel_u32(&P.bs[b].done, 1u);
+      atomicAdd((unsigned int*)(P.ticket + 2), 1u);
     }
+    const int64_t nb = b + P.win;  // the window slot is free: admit the next batch
+    if (nb < P.num_batches)
+      ns_start_hop(P, sm, nb, 0, min(P.batch_size, P.num_seeds - nb * P.batch_size));
+  }
+}
+
+__device__ void ns_start_hop(const NSParams& P, NSSmem& sm, int64_t b, int l, int64_t T) {
+  const int nt = (int)((T + ns_tile_cols(P.k[l]) - 1) / ns_tile_cols(P.k[l]));
+  if (threadIdx.x == 0) {
+    P.bs[b].T[l] = T;
+    __threadfence();
+    if (nt > 0) ns_append(P, b, l, nt);
+  }
+  __syncthreads();
+  if (nt == 0) {  // empty frontier: the hop (and every later one) is empty
+    if (threadIdx.x == 0) {
+      const int64_t bstart = b * P.batch_size;
+      const int64_t colbase = l == 0 ? bstart : bstart * P.K[l - 1];
+      const int64_t ibase = colbase + b;
+      P.indptr_out[l][ibase] = 0;
+    }
+    ns_hop_done(P, sm, b, l, 0, 0, 0);
+  }
+}
+
+__global__ void stream_admit_kernel(NSParams P) {
+  // admit the first window of batches (hop 0 of batch b has min(bs, rest) columns)
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  const int64_t n = min((int64_t)P.win, P.num_batches);
+  for (int64_t b = 0; b < n; ++b) {
+    const int64_t T = min(P.batch_size, P.num_seeds - b * P.batch_size);
+    P.bs[b].T[0] = T;
+    ns_append(P, b, 0, (int)((T + ns_tile_cols(P.k[0]) - 1) / ns_tile_cols(P.k[0])));
   }
 }
 
 __global__ void __launch_bounds__(NS_THREADS, 2) nodewise_stream_kernel(NSParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   NSSmem& sm = *reinterpret_cast<NSSmem*>(smem_raw);
-  const unsigned long long total = (unsigned long long)P.nsteps * P.tps;
+  int64_t hint = 0;  // job index cursor (this CTA's tickets only increase)
   while (true) {
-    if (threadIdx.x == 0) sm.job[0] = (long long)atomicAdd(P.ticket, 1ull);
+    if (threadIdx.x == 0) {
+      const unsigned long long t = atomicAdd(P.ticket, 1ull);
+      long long kind = 0;  // 0 exit, 1 work
+      Backoff bo;
+      while (true) {
+        const unsigned long long tail = ld_acq_u64(P.ticket + 1);
+        if (t < (tail & ((1ull << 40) - 1))) {
+          kind = 1;
+          break;
+        }
+        if ((int64_t)ld_acq_u32((const unsigned int*)(P.ticket + 2)) >= P.num_batches) break;
+        bo.wait();
+      }
+      if (kind) {
+        while (true) {
+          NSJob& J = P.jobs[hint];
+          Backoff bj;
+          while (ld_acq_u32(&J.ready) == 0u) bj.wait();
+          if ((long long)t < J.start + J.nt) break;
+          ++hint;
+        }
+        const NSJob& J = P.jobs[hint];
+        sm.job[1] = J.b;
+        sm.job[2] = J.l;
+        sm.job[3] = (long long)t - J.start;
+      }
+      sm.job[0] = kind;
+      sm.job[0] |= (long long)t << 1;
+    }
     __syncthreads();
-    const unsigned long long tk = (unsigned long long)sm.job[0];
+    const long long w0 = sm.job[0], b = sm.job[1], l = sm.job[2], t = sm.job[3];
     __syncthreads();
-    if (tk >= total) break;
-    const int64_t step = (int64_t)(tk / P.tps);
-    const int r = (int)(tk % P.tps);
-    int l = 0;
-    while (l + 1 < P.L && r >= P.tile_off[l + 1]) ++l;  // tile_off is increasing in l's order
-    // hops are laid out deepest first: map the range index back to the hop
-    const int hop = P.L - 1 - l;
-    const int t = r - P.tile_off[l];
-    const int64_t b = step - (int64_t)hop * NS_LAG;
-    if (b < 0 || b >= P.num_batches) continue;
-    ns_tile(P, sm, b, hop, t);
+    if ((w0 & 1) == 0) break;
+    ns_tile(P, sm, b, (int)l, (int)t, (unsigned long long)(w0 >> 1));
   }
 }
 
@@ -496,24 +701,23 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
     P.k[l] = fanouts[l];
     const int64_t cols = batch_size * prod;  // bound on the hop's frontier
     col_cap = std::max(col_cap, cols);
-    P.maxtiles[l] = (int)((cols + NS_COLS - 1) / NS_COLS);
+    const int ks = fanouts[l] | 1;  // = ns_tile_cols() on the device
+    const int tcols = std::min(NS_COLS, std::max(1, NS_SLOTS / (ks * 32)) * 32);
+    P.maxtiles[l] = (int)((cols + tcols - 1) / tcols);
     max_t = std::max(max_t, P.maxtiles[l]);
     prod *= fanouts[l];
     P.K[l] = prod;
     slot_cap = std::max(slot_cap, cols * fanouts[l]);
   }
-  // deepest hop first inside a step
-  int off = 0;
-  for (int i = 0; i < L; ++i) {
-    const int hop = L - 1 - i;
-    P.tile_off[i] = off;
-    off += P.maxtiles[hop];
-  }
-  P.tps = off;
   P.max_tiles_all = max_t;
-  P.win = (L - 1) * NS_LAG + NS_LAG + 2;
+  {
+    const char* w = getenv("GS_WINDOW");
+    P.win = w ? std::max(1, atoi(w)) : 32;  // mini-batches in flight
+  }
   const int64_t nbatch = P.num_batches;
-  P.nsteps = nbatch + (int64_t)(L - 1) * NS_LAG;
+  int64_t tiles_bound = 0;
+  for (int l = 0; l < L; ++l) tiles_bound += P.maxtiles[l];
+  tiles_bound *= std::max<int64_t>(nbatch, 1);
   col_cap += NS_COLS;
   slot_cap += (int64_t)NS_COLS * MAX_FANOUT;
   blk->kind = gs_blocks::NODEWISE;
@@ -533,7 +737,8 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
          need(blk->b_rowl[l], rows * 4) && need(blk->b_eid[l], rows * 8);
     if (bias == GS_W_PASS_COLNORM) ok = ok && need(blk->b_val[l], rows * 4);
   }
-  const int64_t sched_bytes = nbatch * (int64_t)sizeof(NSBatch) + 256;
+  const int64_t jobs_off = align256(nbatch * (int64_t)sizeof(NSBatch) + 64);
+  const int64_t sched_bytes = jobs_off + (nbatch * L + 16) * (int64_t)sizeof(NSJob);
   ok = ok && need(blk->b_meta, nbatch * L * 8 * 8) && need(blk->b_err, 16) &&
        need(blk->b_ctr, 8 * (MAX_LAYERS + 2)) && need(blk->b_sched, sched_bytes);
   if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (blocks buffers)");
@@ -558,7 +763,8 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
   P.o_sel = o; o = align256(o + (int64_t)L * max_t * 8);
   P.o_agg = o; o = align256(o + (int64_t)3 * L * max_t * 8);
   P.o_rx = o; o = align256(o + (int64_t)L * max_t * 8);
-  P.o_tab = o; o = align256(o + (int64_t(8) << log_tab));
+  P.o_tab = o; o = align256(o + 256);  // (hash table unused: direct first[] array)
+  P.o_first = o; o = align256(o + g->num_nodes * 4);
   P.ws_stride = o;
   P.log_tab_cap = log_tab;
   const size_t ws_bytes = (size_t)P.ws_stride * P.win;
@@ -574,6 +780,7 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
   P.launch = (++blk->launch_id) & 0x3FFFFFFFu;
   P.bs = (NSBatch*)blk->b_sched.ptr;
   P.ticket = (unsigned long long*)((char*)blk->b_sched.ptr + nbatch * sizeof(NSBatch));
+  P.jobs = (NSJob*)((char*)blk->b_sched.ptr + jobs_off);
 
   P.col0 = (int32_t*)blk->b_col[0].ptr;
   for (int l = 0; l < L; ++l) {
@@ -613,8 +820,28 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     grid = std::max(1, per_sm) * sms;  // every CTA co-resident: waits only point backwards
   }
+  const char* trace_path = getenv("GS_TRACE");
+  unsigned long long* dtrace = nullptr;
+  const size_t ntk = (size_t)tiles_bound + 1024;
+  if (trace_path) {
+    GS_CUDA_TRY(cudaMalloc(&dtrace, ntk * 96));
+    GS_CUDA_TRY(cudaMemsetAsync(dtrace, 0, ntk * 96, stream));
+    P.trace = dtrace;
+    P.trace2 = dtrace + ntk * 8;
+  }
+  stream_admit_kernel<<<1, 32, 0, stream>>>(P);
   nodewise_stream_kernel<<<grid, NS_THREADS, sizeof(NSSmem), stream>>>(P);
   GS_CUDA_TRY(cudaGetLastError());
+  if (trace_path) {  // tracing aid: per-tile timestamps to a binary file
+    std::vector<unsigned long long> h(ntk * 12);
+    GS_CUDA_TRY(cudaStreamSynchronize(stream));
+    GS_CUDA_TRY(cudaMemcpy(h.data(), dtrace, ntk * 96, cudaMemcpyDeviceToHost));
+    cudaFree(dtrace);
+    if (FILE* f = fopen(trace_path, "wb")) {
+      fwrite(h.data(), 8, h.size(), f);
+      fclose(f);
+    }
+  }
   return GS_OK;
 }
 
