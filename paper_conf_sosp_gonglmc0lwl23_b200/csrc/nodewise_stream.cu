@@ -373,47 +373,46 @@ __device__ void ns_tile(const NSParams& P, NSSmem& sm, int64_t b, int l, int t, 
   __syncthreads();
   if (trc && threadIdx.x == 0) trc[3] = gtimer();
   // ---- 3. first-occurrence bitmap of this tile's slots (word-major) ----
+  // every first[u] lookup of the warp's words is issued at once (<= 12 per lane)
+  constexpr int NS_WPW = NS_SLOTS / 32 / NS_WARPS;  // words per warp, upper bound
   const int wpw = (nwords + NS_WARPS - 1) / NS_WARPS;
   const int wa = warp * wpw, wz = min(nwords, wa + wpw);
-  int wrun = 0;
-  for (int w0 = wa; w0 < wz; w0 += NW_ILP) {
-    uint32_t uu[NW_ILP], qq[NW_ILP];
-    bool vv[NW_ILP];
-    unsigned long long ee[NW_ILP];
+  uint32_t p0r[NS_WPW];
+  bool vr[NS_WPW];
 #pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) {
-      const int r = (w0 + i) * 32 + lane;  // tile-local slot rank
-      vv[i] = false;
-      qq[i] = 0u;
-      if (w0 + i < wz && r < nslots) {
-        const int jl = r / k, s = r - jl * k;
-        vv[i] = s < sm.scnt[jl];
-        qq[i] = (uint32_t)(jl * ks + s);
+  for (int i = 0; i < NS_WPW; ++i) {
+    const int r = (wa + i) * 32 + lane;
+    vr[i] = false;
+    p0r[i] = 0u;
+    if (wa + i < wz && r < nslots) {
+      const int jl = r / k, s = r - jl * k;
+      if (s < sm.scnt[jl]) {
+        vr[i] = true;
+        p0r[i] = ldh(S.first + sm.su[jl * ks + s], pl);
       }
-      uu[i] = vv[i] ? sm.su[qq[i]] : 0u;
     }
+  }
+  int wrun = 0;
 #pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) ee[i] = vv[i] ? (unsigned long long)ldh(S.first + uu[i], pl) : 0ull;
-#pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) {
-      const int wl = w0 + i;
-      const int64_t p = p_base + (int64_t)wl * 32 + lane;
-      bool first = false;
-      if (vv[i]) {
-        const uint32_t p0 = (uint32_t)ee[i];
-        if (p0 > (uint32_t)p) atomicOr(P.core.err, ERR_INTERNAL);
-        sm.sp0[qq[i]] = p0;
-        first = p0 == (uint32_t)p;
+  for (int i = 0; i < NS_WPW; ++i) {
+    const int wl = wa + i;
+    const int r = wl * 32 + lane;
+    const int64_t p = p_base + r;
+    bool first = false;
+    if (vr[i]) {
+      const int jl = r / k, s = r - jl * k;
+      sm.sp0[jl * ks + s] = p0r[i];
+      if (p0r[i] > (uint32_t)p) atomicOr(P.core.err, ERR_INTERNAL);
+      first = p0r[i] == (uint32_t)p;
+    }
+    const uint32_t word = __ballot_sync(0xffffffffu, first);
+    if (wl < wz) {
+      if (lane == 0) {
+        sm.sbits[wl] = word;
+        sm.swpre[wl] = __popc(word);
+        sth(S.bits + (p_base >> 5) + wl, word, pl);
       }
-      const uint32_t word = __ballot_sync(0xffffffffu, first);
-      if (wl < wz) {
-        if (lane == 0) {
-          sm.sbits[wl] = word;
-          sm.swpre[wl] = __popc(word);
-          sth(S.bits + (p_base >> 5) + wl, word, pl);
-        }
-        wrun += __popc(word);
-      }
+      wrun += __popc(word);
     }
   }
   if (lane == 0) sm.wtot[warp] = wrun;
