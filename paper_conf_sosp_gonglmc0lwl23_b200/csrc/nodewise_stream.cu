@@ -711,7 +711,7 @@ gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t n
   P.max_tiles_all = max_t;
   {
     const char* w = getenv("GS_WINDOW");
-    P.win = w ? std::max(1, atoi(w)) : 32;  // mini-batches in flight
+    P.win = w ? std::max(1, atoi(w)) : 48;  // mini-batches in flight
   }
   const int64_t nbatch = P.num_batches;
   int64_t tiles_bound = 0;
