@@ -7,7 +7,8 @@ neighbour sampling, batch 1024, one full epoch of seeds (196,615 = the
 ogbn-products train-split size, 193 mini-batches) on an Ogbn-Products-shaped
 R-MAT graph (2,449,029 nodes, 61,859,140 undirected edges -> 123,718,280 CSC
 entries).  One step = one epoch (every batch, every hop: Extract, Select,
-Finalize) = one launch of the cluster kernel.
+Finalize) = one launch of the node-wise stream kernel.  Other configs of
+BASELINE.json are selectable with --workload (parity cases / extra lines).
 
 Contract: python bench.py --gpus N --steps K --warmup W [--impl reference]
 Multi-GPU (torchrun): one process per GPU; rank 0 generates the graph and
@@ -18,7 +19,6 @@ from __future__ import annotations
 
 import argparse
 import json
-import math
 import os
 import statistics
 import sys
@@ -28,17 +28,21 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-import numpy as np  # noqa: E402
+import numpy as np  # noqa: E402,F401
 import torch  # noqa: E402
 
 METRIC = "sampled edges/s & epoch sampling time at 1/2/4/8 B200; % HBM roofline"
 UNIT = "sampled edges/s"
+# Random 32-byte-sector read ceiling of this B200's HBM, measured with
+# tools/microbench2.cu (profiles/r01_microbench.txt): ~55 G sectors/s.
+RANDOM_SECTOR_GBS = 1750.0
 
 WORKLOADS = {
     "graphsage_pd": dict(kind="nodewise", graph="PD", fanouts=[25, 10], batch=1024,
                          seeds=196_615, replace=False, bias=0,
                          desc="GraphSAGE [25,10] uniform, batch 1024, full epoch (196,615 seeds, "
-                              "193 batches), Ogbn-Products-shaped R-MAT graph"),
+                              "193 batches), Ogbn-Products-shaped R-MAT graph (2,449,029 nodes, "
+                              "61,859,140 undirected edges)"),
     "graphsage_tiny": dict(kind="nodewise", graph="tiny", fanouts=[5, 5], batch=512, seeds=512,
                            replace=False, bias=0,
                            desc="GraphSAGE [5,5] uniform, 512 seeds, 10k-node/100k-edge R-MAT"),
@@ -46,6 +50,9 @@ WORKLOADS = {
                     replace=True, bias=0, desc="KGCN [8,8] with replacement, PD-shaped"),
     "pass_pd": dict(kind="nodewise", graph="PDw", fanouts=[10, 10], batch=1024, seeds=196_615,
                     replace=False, bias=2, desc="PASS-style A3 [10,10], PD-shaped weighted"),
+    "ares_pp": dict(kind="nodewise", graph="PP", fanouts=[15, 10, 5], batch=1024,
+                    seeds=1_207_179, replace=False, bias=1,
+                    desc="GraphSAGE [15,10,5] weighted A-Res, Papers100M-shaped"),
     "shadow_pd": dict(kind="shadow", graph="PD", fanouts=[10, 5], batch=1024, seeds=196_615,
                       bias=0, desc="ShaDow [10,5] uniform + induce, PD-shaped"),
     "ladies_lj": dict(kind="layerwise", graph="LJ", n_per_layer=[512, 512, 512], batch=512,
@@ -74,9 +81,9 @@ def measured_peak_hbm():
 class ClockSampler:
     """Samples SM clocks and throttle reasons through NVML during the timed region."""
 
-    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
-               0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
-               0x80: "hw_power_brake_slowdown", 0x100: "display_clocks_setting"}
+    REASONS = {0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown"}
 
     def __init__(self, device_index):
         self.samples, self.reasons = [], set()
@@ -98,7 +105,7 @@ class ClockSampler:
                 self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
                 r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
                 for bit, name in self.REASONS.items():
-                    if r & bit and name != "gpu_idle":
+                    if r & bit:
                         self.reasons.add(name)
             except Exception:
                 pass
@@ -143,47 +150,6 @@ def make_graph_dist(name, world, rank, device):
     return g
 
 
-def nodewise_model_bytes(blocks, indptr, fanouts, L):
-    """Algorithmic bytes of one node-wise step (SURVEY.md 8(d) byte model):
-    per column 4 (frontier id) + 32*(1 + [v % 4 == 3]) (int64 indptr pair sector(s))
-    + 32 * |distinct 32-byte sectors of the sampled positions| + 8 (block indptr);
-    per sampled edge 4 (row_local) + 8 (eid); per new row 4 (row_map)."""
-    meta = blocks.device_meta()            # [B, L, 8]
-    total = 0
-    edges = 0
-    import ctypes
-    from paper_conf_sosp_gonglmc0lwl23_b200 import gs
-    for l in range(L):
-        lb = gs._lib  # noqa
-        m = meta[:, l, :]
-        n_cols, n_rows, n_edges = m[:, 0], m[:, 1], m[:, 2]
-        col_off, ind_off, e_off = m[:, 3], m[:, 5], m[:, 6]
-        view = _layer_arrays(blocks, l)
-        # per-edge column ids: from each batch's block indptr
-        ecount = int(n_edges.sum())
-        edges += ecount
-        colv_all, sec_all = [], []
-        for b in range(m.shape[0]):
-            T = int(n_cols[b])
-            if T == 0:
-                continue
-            ip = view["indptr"][int(ind_off[b]): int(ind_off[b]) + T + 1]
-            E = int(n_edges[b])
-            eids = view["eid"][int(e_off[b]): int(e_off[b]) + E]
-            cols = view["col_map"][int(col_off[b]): int(col_off[b]) + T].to(torch.int64)
-            cnt = ip[1:] - ip[:-1]
-            cid = torch.repeat_interleave(torch.arange(T, device=ip.device), cnt)
-            key = cid * (1 << 40) + (eids >> 3)
-            sec_all.append(torch.unique(key).numel())
-            colv_all.append(cols)
-        cols = torch.cat(colv_all) if colv_all else torch.empty(0, dtype=torch.int64)
-        ncols = cols.numel()
-        straddle = int(((cols & 3) == 3).sum()) if ncols else 0
-        total += ncols * (4 + 8) + 32 * (ncols + straddle) + 32 * sum(sec_all)
-        total += ecount * 12 + int(n_rows.sum()) * 4
-    return total, edges
-
-
 def _layer_arrays(blocks, l):
     import ctypes
     from paper_conf_sosp_gonglmc0lwl23_b200 import gs
@@ -199,45 +165,112 @@ def _layer_arrays(blocks, l):
     gs._lib.gs_blocks_layer.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.POINTER(LB)]
     gs._check(gs._lib.gs_blocks_layer(blocks._h, l, ctypes.byref(lb)))
     t = gs._dev_tensor
-    return {"col_map": t(lb.col_map, lb.col_capacity, torch.int32, blocks),
-            "row_map": t(lb.row_map, lb.row_capacity, torch.int32, blocks),
-            "indptr": t(lb.indptr, lb.indptr_capacity, torch.int64, blocks),
-            "row_local": t(lb.row_local, lb.edge_capacity, torch.int32, blocks),
-            "eid": t(lb.eid, lb.edge_capacity, torch.int64, blocks)}
+    d = {"col_map": t(lb.col_map, lb.col_capacity, torch.int32, blocks),
+         "row_map": t(lb.row_map, lb.row_capacity, torch.int32, blocks),
+         "indptr": t(lb.indptr, lb.indptr_capacity, torch.int64, blocks),
+         "row_local": t(lb.row_local, lb.edge_capacity, torch.int32, blocks),
+         "eid": t(lb.eid, lb.edge_capacity, torch.int64, blocks)}
+    if lb.val:
+        d["val"] = t(lb.val, lb.edge_capacity, torch.float32, blocks)
+    return d
 
 
-def ncu_traffic(workload):
-    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full capture."""
-    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    try:
-        with open(path) as f:
-            d = json.load(f)
-        return d.get(workload)
-    except Exception:
-        return None
+def _secs(off, d):
+    """32-byte int32 sectors spanned by [off, off + d) (0 when d == 0)."""
+    return torch.where(d > 0, ((off + d - 1) >> 3) - (off >> 3) + 1, torch.zeros_like(d))
+
+
+def _blocks_byte_model(blocks, g, kind, weighted, L):
+    """Algorithmic bytes of one step (SURVEY.md 8(d) byte model).
+    node-wise, per column: 4 (frontier id) + 32*(1 + [v%4==3]) (int64 indptr pair)
+      + 32 * distinct sectors of the sampled positions (the column when d <= k)
+      + 8 (block indptr); per edge 12 (row_local + eid); per row 4 (row_map).
+    shadow: per U node the whole column streamed once (4 + 32(1+straddle) +
+      32 secs(off, d)) + 12 per induced edge + 4 per node.
+    layer-wise: every frontier column streamed twice (indices, + weights for
+      LADIES) + 32(1+straddle) + 4; per block edge 16; per row 8."""
+    indptr = g["indptr"]
+    meta = blocks.device_meta()
+    total, edges = 0, 0
+    for l in range(L):
+        view = _layer_arrays(blocks, l)
+        m = meta[:, l, :].cpu()
+        cols_all, e_all = [], []
+        for b in range(m.shape[0]):
+            T, R, E = int(m[b, 0]), int(m[b, 1]), int(m[b, 2])
+            if T == 0:
+                continue
+            co, io, eo = int(m[b, 3]), int(m[b, 5]), int(m[b, 6])
+            cols_all.append(view["col_map"][co:co + T].to(torch.int64))
+            ip = view["indptr"][io:io + T + 1]
+            e_all.append((view["eid"][eo:eo + E], ip[1:] - ip[:-1]))
+            total += E * (12 if kind != "layerwise" else 16) + R * (4 if kind != "layerwise" else 8)
+            edges += E
+        if not cols_all:
+            continue
+        cols = torch.cat(cols_all)
+        off = indptr[cols]
+        d = indptr[cols + 1] - off
+        straddle = int(((cols & 3) == 3).sum())
+        ncols = cols.numel()
+        if kind == "nodewise":
+            sec = 0
+            for eids, cnt in e_all:
+                cid = torch.repeat_interleave(torch.arange(cnt.numel(), device=cnt.device), cnt)
+                sec += torch.unique(cid * (1 << 40) + (eids >> 3)).numel()
+            total += ncols * 12 + 32 * (ncols + straddle) + 32 * sec
+        elif kind == "shadow":
+            total += ncols * 4 + 32 * (ncols + straddle) + 32 * int(_secs(off, d).sum())
+        else:
+            s = int(_secs(off, d).sum())
+            total += 2 * (ncols * 4 + 32 * (ncols + straddle) + 32 * s * (2 if weighted else 1))
+    return total, edges
 
 
 # ---------------------------------------------------------------------------
-# CPU baseline / reference arm: the oracle as it stands
+# Oracle (CPU baseline / reference arm): the oracle as it stands
 # ---------------------------------------------------------------------------
-def oracle_nodewise_rate(g, seeds, wl, budget_s=15.0):
+def oracle_rate(g, inputs, wl, budget_s=15.0):
     import oracle
     O = oracle.Graph(g["indptr"].cpu().numpy(), g["indices"].cpu().numpy(),
                      None if g["weights"] is None else g["weights"].cpu().numpy())
     cores = len(os.sched_getaffinity(0))
-    s = seeds.cpu().numpy()
+    s = inputs.cpu().numpy()
+    kind = wl["kind"]
+    if kind == "walk":
+        n1 = min(len(s), 4096)
+        t0 = time.perf_counter()
+        oracle.random_walk(O, s[:n1], wl["length"], p=wl["p"], q=wl["q"], num_threads=1)
+        t1 = (time.perf_counter() - t0) / n1
+        n = int(max(1024, min(len(s), budget_s * cores / max(t1, 1e-9))))
+        t0 = time.perf_counter()
+        tr = oracle.random_walk(O, s[:n], wl["length"], p=wl["p"], q=wl["q"], num_threads=cores)
+        dt = time.perf_counter() - t0
+        edges = int((tr[:, 1:] >= 0).sum())
+        return {"value": edges / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+                "sample": f"first {n} of {len(s)} walkers ({edges} transitions, {dt:.2f} s on "
+                          f"{cores} threads)"}, edges, dt
     bs = wl["batch"]
     nb_total = (len(s) + bs - 1) // bs
-    # calibrate on one batch, one thread
+
+    def run(nbat, threads):
+        if kind == "nodewise":
+            return oracle.sample_neighbors(O, s[:nbat * bs], wl["fanouts"], batch_size=bs,
+                                           replace=wl["replace"], bias_mode=wl["bias"], rng_key=1,
+                                           num_threads=threads)
+        if kind == "shadow":
+            return [[x] for x in oracle.shadow(O, s[:nbat * bs], wl["fanouts"], batch_size=bs,
+                                               bias_mode=wl["bias"], rng_key=1,
+                                               num_threads=threads)]
+        return oracle.sample_layerwise(O, s[:nbat * bs], wl["n_per_layer"], batch_size=bs,
+                                       prob_mode=wl["mode"], rng_key=1, num_threads=threads)
+
     t0 = time.perf_counter()
-    r = oracle.sample_neighbors(O, s[:bs], wl["fanouts"], batch_size=bs, replace=wl["replace"],
-                                bias_mode=wl["bias"], rng_key=1, num_threads=1)
+    run(1, 1)
     t1 = time.perf_counter() - t0
     nb = int(max(1, min(nb_total, budget_s * cores / max(t1, 1e-4))))
     t0 = time.perf_counter()
-    r = oracle.sample_neighbors(O, s[:nb * bs], wl["fanouts"], batch_size=bs,
-                                replace=wl["replace"], bias_mode=wl["bias"], rng_key=1,
-                                num_threads=cores)
+    r = run(nb, cores)
     dt = time.perf_counter() - t0
     edges = sum(len(blk["eid"]) for layers in r for blk in layers)
     return {"value": edges / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
@@ -245,27 +278,37 @@ def oracle_nodewise_rate(g, seeds, wl, budget_s=15.0):
                       f"{dt:.2f} s wall on {cores} threads)"}, edges, dt
 
 
+def workload_inputs(wl, g, device):
+    import synth
+    if wl["kind"] == "walk":
+        return torch.arange(g["indptr"].numel() - 1, dtype=torch.int32, device=device)
+    return synth.make_seeds(wl["graph"], wl["seeds"], device=device)
+
+
 def run_reference(args, wl):
     world, rank, _ = dist_env()
     if rank != 0:
         return
     import synth
-    g = synth.make_graph(wl["graph"], device="cuda" if torch.cuda.is_available() else "cpu")
-    seeds = synth.make_seeds(wl["graph"], wl["seeds"])
-    rates, total_edges, total_t = [], 0, 0.0
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    g = synth.make_graph(wl["graph"], device=dev)
+    inputs = workload_inputs(wl, g, dev)
+    total_edges, total_t, cb = 0, 0.0, None
     for i in range(args.warmup + args.steps):
-        cb, e, dt = oracle_nodewise_rate(g, seeds, wl, budget_s=3.0)
+        cb, e, dt = oracle_rate(g, inputs, wl, budget_s=3.0)
         if i >= args.warmup:
-            rates.append(cb["value"])
             total_edges += e
             total_t += dt
     value = total_edges / total_t
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1000 * total_t / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-            "impl": "reference",
-            "config": {"workload": wl["desc"], "oracle": "oracle/gso.cpp (CPU, OpenMP over batches)"},
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic (deterministic R-MAT, DESIGN.md input recipe)", "impl": "reference",
+            "config": {"workload": wl["desc"],
+                       "reference": "CPU oracle oracle/gso.cpp as it stands (no reference "
+                                    "implementation exists; DESIGN.md section 10)",
+                       "step": "a bounded sample of the workload (see cpu_baseline.sample)"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cb["cores"], "kind": "oracle",
                              "sample": cb["sample"]},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
@@ -276,33 +319,80 @@ def run_reference(args, wl):
 # ---------------------------------------------------------------------------
 # GPU arm
 # ---------------------------------------------------------------------------
-def run_nodewise(args, wl, world, rank, device):
-    import synth
+def run_gpu(args, wl, world, rank, device):
     from paper_conf_sosp_gonglmc0lwl23_b200 import dist as gdist
     from paper_conf_sosp_gonglmc0lwl23_b200 import gs
     import torch.distributed as dist
     gs.use_torch_allocator()
+    kind = wl["kind"]
     t0 = time.time()
     g = make_graph_dist(wl["graph"], world, rank, device)
     gen_s = time.time() - t0
     G = gs.Graph(g["indptr"], g["indices"], g["weights"])
-    seeds = synth.make_seeds(wl["graph"], wl["seeds"], device=device)
-    bs = wl["batch"]
-    nb = (seeds.numel() + bs - 1) // bs
-    fan = wl["fanouts"]
+    inputs = workload_inputs(wl, g, device)
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=device)  # > 126 MB L2
     out = gs.Blocks()
     base_key = 0x5EED
+    if kind == "walk":
+        nunits = inputs.numel()
+        wbase = rank * nunits
+        traces = torch.empty((nunits, wl["length"] + 1), dtype=torch.int32, device=device)
+        L = 1
+    else:
+        bs = wl["batch"]
+        nunits = (inputs.numel() + bs - 1) // bs
+        wbase = gdist.weak_batch_base(rank, nunits)
+        L = 1 if kind == "shadow" else len(wl.get("fanouts") or wl.get("n_per_layer"))
 
-    def step(i, blocks):
-        return gs.sample_neighbors(G, seeds, fan, batch_size=bs, batch_index_base=gdist.weak_batch_base(rank, nb),
-                                   replace=wl["replace"], bias_mode=wl["bias"],
-                                   rng_key=base_key + 7919 * i, stream=stream, out=blocks)
+    def step(i, x=None):
+        x = inputs if x is None else x
+        key = base_key + 7919 * i
+        if kind == "nodewise":
+            gs.sample_neighbors(G, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
+                                replace=wl["replace"], bias_mode=wl["bias"], rng_key=key,
+                                stream=stream, out=out)
+        elif kind == "shadow":
+            gs.sample_shadow(G, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
+                             bias_mode=wl["bias"], rng_key=key, stream=stream, out=out,
+                             retry=False)
+        elif kind == "layerwise":
+            gs.sample_layerwise(G, x, wl["n_per_layer"], batch_size=bs, batch_index_base=wbase,
+                                prob_mode=wl["mode"], rng_key=key, stream=stream, out=out,
+                                retry=False)
+        else:
+            gs.random_walk(G, x, wl["length"], p=wl["p"], q=wl["q"], walker_index_base=wbase,
+                           rng_key=key, stream=stream, out=traces)
 
+    def grow_until_fits():
+        # layer-wise / ShaDow outputs are sized on the device: grow before timing
+        for _ in range(4):
+            step(0)
+            try:
+                out.sync()
+                return
+            except gs.GSError as e:
+                if e.status != 7:
+                    raise
+
+    def account():
+        if kind == "walk":
+            nxt = traces[:, 1:]
+            moved = nxt >= 0
+            edges = int(moved.sum())
+            prev = traces[:, :-1].to(torch.int64)
+            straddle = int((((prev & 3) == 3) & moved).sum())
+            return edges * (32 + 32 + 4) + 32 * straddle, edges
+        out.sync()
+        return _blocks_byte_model(out, g, kind, g["weights"] is not None and wl.get("mode") == 0,
+                                  L)
+
+    if kind in ("shadow", "layerwise"):
+        grow_until_fits()
     for i in range(args.warmup):
-        step(i, out)
-    out.sync()
+        step(i)
+    if kind != "walk":
+        out.sync()
     torch.cuda.synchronize()
     times, edges, model_bytes = [], 0, 0
     if world > 1:
@@ -313,41 +403,43 @@ def run_nodewise(args, wl, world, rank, device):
             flush.zero_()
             ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             ev0.record(stream)
-            step(args.warmup + i, out)
+            step(args.warmup + i)
             ev1.record(stream)
             ev1.synchronize()
             times.append(ev0.elapsed_time(ev1))
-            out.sync()
-            mb, e = nodewise_model_bytes(out, g["indptr"], fan, len(fan))
+            mb, e = account()
             model_bytes += mb
             edges += e
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     t_total_ms = sum(times)
-    # e2e: the same step through the C ABI with HOST buffers (pinned), copies inside
-    host_seeds = seeds.cpu().pin_memory()
-    lay = [_layer_arrays(out, l) for l in range(len(fan))]
-    host_out = [{k: torch.empty_like(v, device="cpu").pin_memory() for k, v in la.items()
-                 if k in ("row_map", "indptr", "row_local", "eid")} for la in lay]
-    meta_h = torch.empty_like(out.device_meta(), device="cpu").pin_memory()
-    dev_seeds = torch.empty_like(seeds)
-    h2d = host_seeds.numel() * 4
-    d2h = meta_h.numel() * 8 + sum(t.numel() * t.element_size() for ho in host_out for t in ho.values())
+
+    # e2e: the same step through the C ABI with HOST buffers (pinned host
+    # inputs copied in, every output copied back, both inside the timed region)
+    host_in = inputs.cpu().pin_memory()
+    dev_in = torch.empty_like(inputs)
+    if kind == "walk":
+        outs = [traces]
+    else:
+        outs = []
+        for l in range(L):
+            la = _layer_arrays(out, l)
+            outs += [la[k2] for k2 in ("row_map", "indptr", "row_local", "eid") if k2 in la]
+        outs.append(out.device_meta())
+    host_out = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in outs]
+    h2d = host_in.numel() * host_in.element_size()
+    d2h = sum(t.numel() * t.element_size() for t in host_out)
     e2e_times = []
     for i in range(max(2, min(args.steps, 5))):
         flush.zero_()
         torch.cuda.synchronize()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
-        dev_seeds.copy_(host_seeds, non_blocking=True)
-        gs.sample_neighbors(G, dev_seeds, fan, batch_size=bs, batch_index_base=gdist.weak_batch_base(rank, nb),
-                            replace=wl["replace"], bias_mode=wl["bias"], rng_key=base_key + i,
-                            stream=stream, out=out)
-        meta_h.copy_(out.device_meta(), non_blocking=True)
-        for la, ho in zip(lay, host_out):
-            for k, t in ho.items():
-                t.copy_(la[k], non_blocking=True)
+        dev_in.copy_(host_in, non_blocking=True)
+        step(args.warmup + i, dev_in)
+        for src, dst in zip(outs, host_out):
+            dst.copy_(src, non_blocking=True)
         ev1.record(stream)
         ev1.synchronize()
         e2e_times.append(ev0.elapsed_time(ev1))
@@ -358,21 +450,31 @@ def run_nodewise(args, wl, world, rank, device):
         c = torch.tensor([edges, model_bytes], dtype=torch.float64, device=device)
         dist.all_reduce(c, op=dist.ReduceOp.SUM)
         t_total_ms, e2e_ms = float(t[0]), float(t[1])
-        edges_all, bytes_all = float(c[0]), float(c[1])
+        edges_all = float(c[0])
     else:
-        edges_all, bytes_all = float(edges), float(model_bytes)
-    ms_per_step = t_total_ms / args.steps
-    value = edges_all / (t_total_ms / 1000.0)
+        edges_all = float(edges)
     peak, peak_src = measured_peak_hbm()
-    bytes_per_launch = model_bytes / args.steps           # this rank, one launch = one epoch
+    bytes_per_launch = model_bytes / args.steps  # this rank, one launch = one step
     achieved = bytes_per_launch / (statistics.mean(times) / 1000.0) / 1e9
-    res = {"value": value, "ms_per_step": ms_per_step, "edges_per_step": edges_all / args.steps,
-           "e2e_value": edges_all / args.steps * world / (e2e_ms / 1000.0) if False else
-           (edges / args.steps) * world / (e2e_ms / 1000.0),
-           "h2d": h2d, "d2h": d2h, "achieved": achieved, "peak": peak, "peak_src": peak_src,
-           "bytes_per_launch": bytes_per_launch, "clocks": clk.summary(), "gen_s": gen_s,
-           "num_batches": nb, "times": times, "graph": g, "seeds": seeds}
-    return res
+    return {"value": edges_all / (t_total_ms / 1000.0), "ms_per_step": t_total_ms / args.steps,
+            "edges_per_step": edges_all / args.steps,
+            "e2e_value": (edges / args.steps) * world / (e2e_ms / 1000.0), "h2d": h2d, "d2h": d2h,
+            "achieved": achieved, "peak": peak, "peak_src": peak_src,
+            "bytes_per_launch": bytes_per_launch, "clocks": clk.summary(), "gen_s": gen_s,
+            "units": nunits, "graph": g, "inputs": inputs}
+
+
+KERNEL_OF = {"nodewise": "gsb::nodewise_stream_kernel", "shadow": "gsb::nodewise_kernel",
+             "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
+
+
+def ncu_traffic(workload):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            return json.load(f).get(workload)
+    except Exception:
+        return None
 
 
 def main():
@@ -387,10 +489,6 @@ def main():
     wl = WORKLOADS[args.workload]
     world, rank, local = dist_env()
     if args.impl == "reference":
-        if world > 1:
-            import torch.distributed as dist
-            if rank != 0:
-                return
         run_reference(args, wl)
         return
     assert torch.cuda.is_available(), "bench.py needs a CUDA device"
@@ -401,37 +499,39 @@ def main():
         dist.init_process_group("nccl", device_id=device)
     import __graft_entry__
     __graft_entry__.build()
-    if wl["kind"] != "nodewise":
-        raise SystemExit(f"workload kind {wl['kind']} not wired into bench.py yet")
-    r = run_nodewise(args, wl, world, rank, device)
+    r = run_gpu(args, wl, world, rank, device)
     if rank == 0:
         cpu = None
         if not args.no_cpu_baseline and world == 1:
-            cpu, _, _ = oracle_nodewise_rate(r["graph"], r["seeds"], wl)
-        traffic = ncu_traffic(args.workload)
+            cpu, _, _ = oracle_rate(r["graph"], r["inputs"], wl)
+        kind = wl["kind"]
         line = {
             "metric": METRIC, "value": r["value"], "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": r["ms_per_step"],
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
             "data": "synthetic (deterministic R-MAT, DESIGN.md input recipe)",
             "config": {"workload": wl["desc"], "graph": wl["graph"],
-                       "fanouts": wl.get("fanouts"), "batch_size": wl["batch"],
-                       "num_batches_per_rank": r["num_batches"],
+                       "units_per_rank": r["units"],
                        "sampled_edges_per_step": r["edges_per_step"],
                        "epoch_ms": r["ms_per_step"],
-                       "l2": "flushed between timed steps (256 MiB write), graph 0.5 GB > L2",
-                       "parallelism": f"dp{world} (epoch per rank, graph replicated)",
+                       "l2": "flushed between timed steps (256 MiB write)",
+                       "parallelism": f"dp{world} (one epoch per rank, graph replicated)",
                        "graph_gen_s": round(r["gen_s"], 2)},
             "roofline": {"bound": "hbm", "achieved": r["achieved"], "peak": r["peak"],
                          "unit": "GB/s", "frac": r["achieved"] / r["peak"],
-                         "traffic": traffic, "peak_source": r["peak_src"],
-                         "kernel": "gsb::nodewise_kernel<8> (1 launch = 1 epoch)",
-                         "algorithmic_bytes_per_launch": r["bytes_per_launch"]},
+                         "traffic": ncu_traffic(args.workload), "peak_source": r["peak_src"],
+                         "kernel": KERNEL_OF[kind] + " (1 launch = 1 step)",
+                         "algorithmic_bytes_per_launch": r["bytes_per_launch"],
+                         "random_sector_ceiling_gbs": RANDOM_SECTOR_GBS,
+                         "frac_of_random_sector_ceiling": r["achieved"] / RANDOM_SECTOR_GBS},
             "e2e": {"value": r["e2e_value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d"],
                     "d2h_bytes_per_step": r["d2h"]},
-            "gpu_launches": args.steps,
+            "gpu_launches": args.steps * (2 if kind == "nodewise" else 1),
             "clocks": r["clocks"],
         }
+        if kind == "nodewise":
+            line["config"]["fanouts"] = wl["fanouts"]
+            line["config"]["batch_size"] = wl["batch"]
         if cpu is not None:
             line["cpu_baseline"] = cpu
         print(json.dumps(line), flush=True)

@@ -81,8 +81,10 @@ CONFIGS = {
 }
 
 
-def _rmat_pairs(spec: GraphSpec, n_gen: int, salt: int, device, chunk: int = 1 << 26):
-    """n_gen R-MAT (src, dst) pairs with ids < N (rejected ones dropped)."""
+def _rmat_pairs(spec: GraphSpec, n_gen: int, salt: int, device, chunk: int = 1 << 26,
+                first: int = 0):
+    """R-MAT (src, dst) pairs number first .. first + n_gen - 1 with ids < N
+    (rejected ones dropped)."""
     N = spec.num_nodes
     scale = max(1, math.ceil(math.log2(N)))
     a, b, c, _ = RMAT
@@ -90,8 +92,8 @@ def _rmat_pairs(spec: GraphSpec, n_gen: int, salt: int, device, chunk: int = 1 <
     tb = int((a + b) * 2 ** 32)
     tc = int((a + b + c) * 2 ** 32)
     srcs, dsts = [], []
-    for start in range(0, n_gen, chunk):
-        e = torch.arange(start, min(n_gen, start + chunk), device=device, dtype=torch.int64)
+    for start in range(first, first + n_gen, chunk):
+        e = torch.arange(start, min(first + n_gen, start + chunk), device=device, dtype=torch.int64)
         src = torch.zeros_like(e)
         dst = torch.zeros_like(e)
         base = e * 64
@@ -117,31 +119,82 @@ def _permutation(stream: int, n: int, device) -> torch.Tensor:
     return new_id
 
 
+_CHUNK = 1 << 29  # elements per torch sort/unique call (CUB handles < 2^31)
+
+
+def _range_parts(x: torch.Tensor, parts: int, salt: int) -> list:
+    """Value boundaries splitting x into ~equal ranges (quantiles of a keyed sample)."""
+    if parts <= 1:
+        return []
+    n = x.numel()
+    idx = hash64(salt, torch.arange(min(n, 1 << 22), device=x.device)) % n
+    sample = torch.sort(x[idx]).values
+    q = torch.linspace(0, sample.numel() - 1, parts + 1, device=x.device)[1:-1].long()
+    return torch.unique(sample[q]).tolist()
+
+
+def _sorted_unique(x: torch.Tensor, unique: bool, salt: int) -> torch.Tensor:
+    """torch.unique / torch.sort for tensors of any length (range-partitioned)."""
+    if x.numel() <= _CHUNK:
+        return torch.unique(x) if unique else torch.sort(x).values
+    bounds = _range_parts(x, (x.numel() + _CHUNK - 1) // _CHUNK * 2, salt)
+    out, lo = [], None
+    for hi in bounds + [None]:
+        m = torch.ones_like(x, dtype=torch.bool)
+        if lo is not None:
+            m &= x > lo
+        if hi is not None:
+            m &= x <= hi
+        part = x[m]
+        del m
+        out.append(torch.unique(part) if unique else torch.sort(part).values)
+        del part
+        lo = hi
+    return torch.cat(out)
+
+
+def _trim(key: torch.Tensor, target: int, salt: int) -> torch.Tensor:
+    """Keeps exactly `target` keys: those with the smallest keyed 32-bit hash
+    (ties by key), chosen with a 16-bit histogram; order of `key` preserved."""
+    h = hash_u32(salt, key)
+    hist = torch.bincount(_srl(h, 16), minlength=1 << 16).cumsum(0)
+    cut = int(torch.searchsorted(hist, torch.tensor(target, device=key.device)))
+    below = int(hist[cut - 1]) if cut > 0 else 0
+    keep = _srl(h, 16) < cut
+    border = torch.nonzero(_srl(h, 16) == cut).flatten()
+    order = torch.argsort(h[border] * (1 << 31) + (border % (1 << 31)))
+    keep[border[order[:target - below]]] = True
+    return key[keep]
+
+
 def _unique_keys(spec: GraphSpec, device) -> torch.Tensor:
-    """Exactly spec.num_edges unique edge keys (undirected: lo*N+hi; directed: dst*N+src)."""
+    """Exactly spec.num_edges unique edge keys, sorted (undirected: lo*N+hi;
+    directed: dst*N+src)."""
     N = spec.num_nodes
     target = spec.num_edges
     perm = _permutation(spec.seed * 7 + 1, N, device)
     factor = 1.25
     for attempt in range(8):
         n_gen = int(target * factor) + 1024
-        src, dst = _rmat_pairs(spec, n_gen, attempt, device)
-        src = perm[src]
-        dst = perm[dst]
-        keep = src != dst
-        src, dst = src[keep], dst[keep]
-        if spec.undirected:
-            key = torch.minimum(src, dst) * N + torch.maximum(src, dst)
-        else:
-            key = dst * N + src
-        del src, dst, keep
-        key = torch.unique(key)
+        chunks = []
+        for start in range(0, n_gen, 1 << 28):
+            src, dst = _rmat_pairs(spec, min(n_gen, start + (1 << 28)) - start, attempt, device,
+                                   first=start)
+            src = perm[src]
+            dst = perm[dst]
+            keep = src != dst
+            src, dst = src[keep], dst[keep]
+            if spec.undirected:
+                chunks.append(torch.minimum(src, dst) * N + torch.maximum(src, dst))
+            else:
+                chunks.append(dst * N + src)
+            del src, dst, keep
+        key = torch.cat(chunks)
+        del chunks
+        key = _sorted_unique(key, True, spec.seed * 7 + 11)
         if key.numel() >= target:
             if key.numel() > target:
-                h = hash64(spec.seed * 7 + 3, key)
-                idx = torch.argsort(h)[:target]
-                key = torch.sort(key[idx]).values
-                del h, idx
+                key = _trim(key, target, spec.seed * 7 + 3)
             return key
         factor *= 1.25 * target / max(1, key.numel())
     raise RuntimeError(f"R-MAT generator could not reach {target} unique edges")
@@ -160,21 +213,28 @@ def make_graph(spec: GraphSpec | str, device="cpu"):
         # column v, row u: both directions of every pair
         ckey = torch.cat([hi * N + lo, lo * N + hi])
         del lo, hi
-        ckey = torch.sort(ckey).values
+        ckey = _sorted_unique(ckey, False, spec.seed * 7 + 13)
     else:
         ckey = key
-    col = torch.div(ckey, N, rounding_mode="floor")
-    indices = (ckey - col * N).to(torch.int32)
+    nnz = ckey.numel()
+    indices = torch.empty(nnz, dtype=torch.int32, device=device)
+    counts = torch.zeros(N, dtype=torch.int64, device=device)
+    for a in range(0, nnz, _CHUNK):
+        c = ckey[a:a + _CHUNK]
+        col = torch.div(c, N, rounding_mode="floor")
+        indices[a:a + _CHUNK] = (c - col * N).to(torch.int32)
+        counts += torch.bincount(col, minlength=N)
+        del c, col
     del ckey
-    counts = torch.bincount(col, minlength=N)
-    del col
     indptr = torch.zeros(N + 1, dtype=torch.int64, device=device)
     indptr[1:] = torch.cumsum(counts, 0)
     weights = None
-    nnz = indices.numel()
     if spec.weights == "uniform":
-        r = hash_u32(spec.seed * 7 + 5, torch.arange(nnz, device=device, dtype=torch.int64))
-        weights = ((_srl(r, 8) + 1).to(torch.float64) * 2.0 ** -24).to(torch.float32)
+        weights = torch.empty(nnz, dtype=torch.float32, device=device)
+        for a in range(0, nnz, _CHUNK):
+            r = hash_u32(spec.seed * 7 + 5,
+                         torch.arange(a, min(nnz, a + _CHUNK), device=device, dtype=torch.int64))
+            weights[a:a + _CHUNK] = ((_srl(r, 8) + 1).to(torch.float64) * 2.0 ** -24).to(torch.float32)
     elif spec.weights == "gcn":
         din = counts.to(torch.float64).clamp_min(1.0)
         dout = torch.bincount(indices.to(torch.int64), minlength=N).to(torch.float64).clamp_min(1.0)
