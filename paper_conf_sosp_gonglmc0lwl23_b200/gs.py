@@ -210,9 +210,12 @@ class Graph:
         return self._h
 
     def __del__(self):
-        if getattr(self, "_h", None) and _alive():
-            _pending.append(("g", self._h))
-            self._h = None
+        try:
+            if getattr(self, "_h", None) and _alive():
+                _pending.append(("g", self._h))
+                self._h = None
+        except TypeError:  # interpreter shutdown: module globals already cleared
+            pass
 
 
 class Blocks:
@@ -269,9 +272,12 @@ class Blocks:
         return out
 
     def __del__(self):
-        if getattr(self, "_h", None) and self._h.value and _alive():
-            _pending.append(("b", self._h))
-            self._h = None
+        try:
+            if getattr(self, "_h", None) and self._h.value and _alive():
+                _pending.append(("b", self._h))
+                self._h = None
+        except TypeError:  # interpreter shutdown: module globals already cleared
+            pass
 
 
 def _host_i32(xs):
