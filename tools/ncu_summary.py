@@ -70,7 +70,7 @@ def main():
             def gb(key):
                 i = hdr.index(key)
                 v = float(r[i])
-                return v * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0}.get(units[i], 1.0)
+                return v * {"Tbyte": 1e12, "Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0}.get(units[i], 1.0)
             traffic = gb("dram__bytes_read.sum") + gb("dram__bytes_write.sum")
             lines.append(f"DRAM bytes (read + write) per launch: {traffic:.4g}")
             lines.append("")
