@@ -86,23 +86,17 @@ struct Graph {
   float w(int64_t e) const { return weights ? weights[e] : 1.0f; }
 };
 
-// Finalize (R3): row_map = unique rows in first-occurrence order
-// while scanning the block's edges in CSC order; row_local = index in row_map.
-void finalize_first_occurrence(const std::vector<int32_t>& edge_u, Block& blk) {
-  std::unordered_map<int32_t, int32_t> local;
+// Finalize (R3): row_map = A.row() = the unique rows of the
+// block in ascending node-id order (the row set of a sparse matrix);
+// row_local[e] = index of the edge's row in row_map.
+void finalize_rows_ascending(const std::vector<int32_t>& edge_u, Block& blk) {
+  blk.row_map = edge_u;
+  std::sort(blk.row_map.begin(), blk.row_map.end());
+  blk.row_map.erase(std::unique(blk.row_map.begin(), blk.row_map.end()), blk.row_map.end());
   blk.row_local.resize(edge_u.size());
-  for (size_t e = 0; e < edge_u.size(); ++e) {
-    int32_t u = edge_u[e];
-    auto it = local.find(u);
-    if (it == local.end()) {
-      int32_t id = (int32_t)blk.row_map.size();
-      local.emplace(u, id);
-      blk.row_map.push_back(u);
-      blk.row_local[e] = id;
-    } else {
-      blk.row_local[e] = it->second;
-    }
-  }
+  for (size_t e = 0; e < edge_u.size(); ++e)
+    blk.row_local[e] = (int32_t)(std::lower_bound(blk.row_map.begin(), blk.row_map.end(),
+                                                  edge_u[e]) - blk.row_map.begin());
 }
 
 // ---------------------------------------------------------------------------
@@ -191,7 +185,7 @@ Block nodewise_layer(const Graph& g, const std::vector<int32_t>& frontier, int k
     }
     blk.indptr.push_back((int64_t)edge_u.size());
   }
-  finalize_first_occurrence(edge_u, blk);
+  finalize_rows_ascending(edge_u, blk);
   return blk;
 }
 
@@ -398,7 +392,7 @@ int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int6
     int64_t lo = b * batch_size, hi = std::min(num_seeds, lo + batch_size);
     std::vector<int32_t> frontier(seeds + lo, seeds + hi);
     uint32_t gb = (uint32_t)(batch_index_base + b);
-    // U = first-occurrence unique of (F0, row_map_0, row_map_1, ...)  (R12)
+    // U = unique of (F0, row_map_0, row_map_1, ...) in ascending order (R12)
     std::vector<int32_t> all(frontier);
     for (int l = 0; l < num_layers; ++l) {
       Block blk = nodewise_layer(gg, frontier, fanouts[l], l, gb, 0, bias_mode, rng_key);
@@ -406,12 +400,11 @@ int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int6
       all.insert(all.end(), blk.row_map.begin(), blk.row_map.end());
     }
     Block ind;
+    std::sort(all.begin(), all.end());
+    all.erase(std::unique(all.begin(), all.end()), all.end());
+    ind.row_map = all;
     std::unordered_map<int32_t, int32_t> local;
-    for (int32_t u : all)
-      if (!local.count(u)) {
-        local[u] = (int32_t)ind.row_map.size();
-        ind.row_map.push_back(u);
-      }
+    for (size_t i = 0; i < all.size(); ++i) local[all[i]] = (int32_t)i;
     ind.col_map = ind.row_map;
     ind.indptr.push_back(0);
     // Induce: every edge u->v of A with u, v in U, CSC order.

@@ -2,7 +2,8 @@
 weighted A-Res, PASS-style A3 probabilities, and the Finalize relabel.
 
 Pins: structural invariants (every sampled edge exists, count = min(k, d), no
-duplicates without replacement, first-occurrence relabel), exact sampling laws
+duplicates without replacement, row() = the block's unique rows ascending and
+row_local their ranks, R3), exact sampling laws
 by enumeration + chi-square (p > 0.001), and the paper's Fig. 1(b) narration
 (two frontiers that both sample f give 3 layer-2 nodes).
 """
@@ -37,11 +38,8 @@ def check_block_invariants(og, blk, k=None, replace=False, exact_count=True):
     # row_map: no duplicates; row_map[row_local[e]] is the edge's source node
     assert len(set(blk["row_map"].tolist())) == len(blk["row_map"])
     assert np.all(blk["row_map"][blk["row_local"]] == ix[blk["eid"]])
-    # first-occurrence order: row i first appears before row i+1
-    first = {}
-    for e, r in enumerate(blk["row_local"]):
-        first.setdefault(int(r), e)
-    assert [first[i] for i in range(len(blk["row_map"]))] == sorted(first.values())
+    # R3: row_map is exactly the set of the block's rows, ascending
+    assert blk["row_map"].tolist() == sorted(set(ix[blk["eid"]].tolist()))
     for j in range(n_cols):
         v = blk["col_map"][j]
         lo, hi = blk["indptr"][j], blk["indptr"][j + 1]
@@ -193,8 +191,8 @@ def test_fig1b_two_frontiers_share_f(oracle_lib):
         if F in rows_b and F in rows_e:
             found += 1
             assert len(blk["row_map"]) == 3
-            # first-occurrence order: b's picks, then e's new pick
-            assert blk["row_map"].tolist() == sorted(rows_b) + sorted(rows_e - {F})
+            # R3: the union of both picks, ascending
+            assert blk["row_map"].tolist() == sorted(rows_b | rows_e)
         else:
             assert len(blk["row_map"]) == 4
     assert found > 0

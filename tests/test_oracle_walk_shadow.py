@@ -117,10 +117,9 @@ def test_shadow_brute_force(oracle_lib, tiny, bias_mode):
                                      rng_key=8)
     ip, ix = tiny.indptr, tiny.indices
     for b, blk in enumerate(ind):
-        U = []
-        for x in np.concatenate([seeds[b * 100:(b + 1) * 100]] + [L["row_map"] for L in nw[b]]):
-            if x not in U:
-                U.append(int(x))
+        # R12: U = unique of the seeds and every hop's rows, ascending
+        U = sorted(set(np.concatenate([seeds[b * 100:(b + 1) * 100]] +
+                                      [L["row_map"] for L in nw[b]]).tolist()))
         assert blk["row_map"].tolist() == U and blk["col_map"].tolist() == U
         Uset = set(U)
         want = sorted(e for v in U for e in range(ip[v], ip[v + 1]) if ix[e] in Uset)
