@@ -6,6 +6,7 @@
 #include <stdint.h>
 #include <stdio.h>
 #include <string.h>
+#include <stdlib.h>
 
 #include <algorithm>
 #include <new>
@@ -84,14 +85,10 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
                        int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                        int replace, int bias, uint64_t key, bool shadow, cudaStream_t stream,
                        gs_blocks* blk);
-gs_status run_nodewise_pq(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
-                          int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
-                          int replace, int bias, uint64_t key, cudaStream_t stream,
-                          gs_blocks* blk);
-gs_status run_nodewise_stream(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
-                              int64_t batch_size, int64_t batch_base, const int32_t* fanouts,
-                              int L, int replace, int bias, uint64_t key, cudaStream_t stream,
-                              gs_blocks* blk);
+gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                            int replace, int bias, uint64_t key, cudaStream_t stream,
+                            gs_blocks* blk);
 gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
@@ -309,8 +306,8 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
   }
   cudaStream_t stream = (cudaStream_t)stream_;
   if ((st = prepare_blocks(out, stream))) return st;
-  return run_nodewise_stream(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
-                             num_layers, replace, bias_mode, rng_key, stream, *out);
+  return run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
+                           num_layers, replace, bias_mode, rng_key, stream, *out);
 }
 
 gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
