@@ -464,7 +464,7 @@ def run_gpu(args, wl, world, rank, device):
             "units": nunits, "graph": g, "inputs": inputs}
 
 
-KERNEL_OF = {"nodewise": "gsb::nodewise_wave_kernel", "shadow": "gsb::nodewise_kernel",
+KERNEL_OF = {"nodewise": "gsb::nodewise_wave_kernel", "shadow": "gsb::shadow_induce_kernel",
              "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
 
 
@@ -526,7 +526,7 @@ def main():
                          "frac_of_random_sector_ceiling": r["achieved"] / RANDOM_SECTOR_GBS},
             "e2e": {"value": r["e2e_value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d"],
                     "d2h_bytes_per_step": r["d2h"]},
-            "gpu_launches": args.steps,
+            "gpu_launches": args.steps * (2 if kind == "shadow" else 1),
             "clocks": r["clocks"],
         }
         if kind == "nodewise":

@@ -1,6 +1,6 @@
 // capi.cu -- the C ABI of libgsb200 (include/gs.h): argument validation, error
 // reporting, the allocator hook, graph ingest (a0) and result objects.  Every
-// sampling step runs in the kernels of nodewise.cu / layerwise.cu / walk.cu.
+// sampling step runs in the kernels of nodewise_wave.cu / shadow.cu / layerwise.cu / walk.cu.
 #include <cuda_runtime.h>
 #include <stdarg.h>
 #include <stdint.h>
@@ -81,10 +81,9 @@ void DevBuf::reset(const Allocator& al, cudaStream_t s) {
   bytes = 0;
 }
 
-gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
-                       int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
-                       int replace, int bias, uint64_t key, bool shadow, cudaStream_t stream,
-                       gs_blocks* blk);
+gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                     int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                     int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk);
 gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                             int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                             int replace, int bias, uint64_t key, cudaStream_t stream,
@@ -328,8 +327,8 @@ gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_
   }
   cudaStream_t stream = (cudaStream_t)stream_;
   if ((st = prepare_blocks(out, stream))) return st;
-  return run_nodewise(g, seeds, num_seeds, batch_size, batch_index_base, fanouts, num_layers, 0,
-                      bias_mode, rng_key, true, stream, *out);
+  return run_shadow(g, seeds, num_seeds, batch_size, batch_index_base, fanouts, num_layers,
+                    bias_mode, rng_key, stream, *out);
 }
 
 gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
@@ -447,6 +446,7 @@ gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out) 
 
 void gs_blocks_destroy(gs_blocks* b) {
   if (!b) return;
+  if (b->aux) gs_blocks_destroy(b->aux);
   cudaStream_t s = b->stream;
   for (int l = 0; l < MAX_LAYERS; ++l) {
     b->b_col[l].reset(b->al, s);

@@ -83,4 +83,5 @@ struct gs_blocks {
   int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;
+  gs_blocks* aux = nullptr;    // ShaDow: the internal node-wise result
 };

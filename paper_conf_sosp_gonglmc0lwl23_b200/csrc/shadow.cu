@@ -1,0 +1,382 @@
+// shadow.cu -- ShaDow (R12): node-wise sampling of every hop
+// (nodewise_wave.cu), then per mini-batch the subgraph of A induced on
+// U = unique(seeds, rows of every hop), ascending (R3/R12).
+//
+// Induce is one persistent kernel of thread-block CLUSTERS, one cluster per
+// mini-batch at a time.  U's membership bitmap (N bits) is split across the
+// cluster's shared memories (DSMEM): CTA r holds bits [r*bpc, (r+1)*bpc) plus
+// a popcount prefix per 256 bits, so the membership test of every streamed
+// edge -- the hot loop, Sum of in-degrees over U per batch -- and the rank of a
+// kept row are shared-memory reads (local or a peer's), never L2/HBM probes.
+// Per batch: mark U -> scan (U ascending) -> count kept edges per column ->
+// scan (CSC indptr, bump-allocated edge range) -> write kept edges in CSC order.
+#include <algorithm>
+#include <new>
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "gs_internal.h"
+
+namespace cg = cooperative_groups;
+
+namespace gsb {
+
+gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                            int replace, int bias, uint64_t key, cudaStream_t stream,
+                            gs_blocks* blk);
+
+constexpr int SH_THREADS = 512;
+constexpr int SH_WARPS = SH_THREADS / 32;
+constexpr int SH_MAX_CS = 8;                      // portable cluster size
+constexpr int SH_ILP = 8;                         // column positions per lane in flight
+constexpr int64_t SH_SMEM_CAP = 200 * 1024;      // dynamic shared memory per CTA (bitmap + prefix)
+
+struct SHParams {
+  const int64_t* indptr;
+  const int32_t* indices;
+  int64_t N;
+  const int32_t* seeds;
+  int64_t num_seeds, batch_size, num_batches;
+  int L;
+  const int32_t* rows[MAX_LAYERS];  // node-wise row_map of every hop
+  int64_t K[MAX_LAYERS];
+  const int64_t* nmeta;             // node-wise meta [b][L][8]
+  int64_t stride;                   // U capacity per batch
+  int32_t* U;                       // [b * stride] U ascending (col_map == row_map)
+  int64_t* indptr_out;              // [b * stride + b] CSC over U
+  int32_t* row_local;
+  int64_t* eid;
+  int64_t edge_cap;
+  unsigned long long* edge_ctr;     // bump allocator of the edge range (total = need)
+  int32_t* ucnt;                    // [b * stride] kept edges per column, then its prefix
+  int64_t* meta;
+  int* err;
+  unsigned int* claim;
+  int64_t bpc;                      // bitmap bits per CTA (multiple of 256)
+};
+
+struct SHShared {                   // static part; the bitmap + prefix are dynamic
+  long long b;
+  long long total, base[SH_MAX_CS];
+  long long etotal, ebase, eoff, E, nU;
+  long long scr64[40];
+  int scr32[40];
+};
+
+__device__ __forceinline__ bool sh_member(const cg::cluster_group& cl, uint32_t* bm, int64_t bpc,
+                                          uint32_t u) {
+  const unsigned owner = (unsigned)(u / (uint64_t)bpc);
+  const uint32_t x = u - owner * (uint32_t)bpc;
+  const uint32_t* w = cl.map_shared_rank(bm, owner);
+  return (w[x >> 5] >> (x & 31)) & 1u;
+}
+
+__device__ __forceinline__ long long sh_rank(const cg::cluster_group& cl, uint32_t* bm, int32_t* gp,
+                                             const SHShared& ss, int64_t bpc, uint32_t u) {
+  const unsigned owner = (unsigned)(u / (uint64_t)bpc);
+  const uint32_t x = u - owner * (uint32_t)bpc;
+  const uint32_t* w = cl.map_shared_rank(bm, owner);
+  const int32_t* p = cl.map_shared_rank(gp, owner);
+  const uint32_t wi = x >> 5, g0 = (x >> 8) << 3;
+  long long r = ss.base[owner] + p[x >> 8];
+  for (uint32_t i = g0; i < wi; ++i) r += __popc(w[i]);
+  return r + __popc(w[wi] & ((1u << (x & 31)) - 1u));
+}
+
+__global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ SHShared ss;
+  cg::cluster_group cl = cg::this_cluster();
+  const unsigned rank = cl.block_rank(), CS = cl.num_blocks();
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t bpc = P.bpc;
+  const int nwords = (int)(bpc >> 5), ngroups = (int)(bpc >> 8);
+  uint32_t* bm = (uint32_t*)smem_raw;
+  int32_t* gp = (int32_t*)(smem_raw + (size_t)nwords * 4);
+  const uint64_t pf = pol_first();
+  while (true) {
+    if (rank == 0 && tid == 0) ss.b = (long long)atomicAdd(P.claim, 1u);
+    cl.sync();
+    const long long b = *cl.map_shared_rank(&ss.b, 0);
+    cl.sync();  // no CTA may exit (or re-claim) while a peer still reads its shared memory
+    if (b >= P.num_batches) break;
+    // ---- mark U ----
+    for (int i = tid; i < nwords; i += SH_THREADS) bm[i] = 0u;
+    cl.sync();
+    const int64_t bstart = b * P.batch_size;
+    const long long T0 = min(P.batch_size, P.num_seeds - bstart);
+    long long nitems = T0;
+    long long cnt_l[MAX_LAYERS];
+    for (int l = 0; l < P.L; ++l) {
+      cnt_l[l] = __ldcg(P.nmeta + (b * P.L + l) * 8 + 1);
+      nitems += cnt_l[l];
+    }
+    for (long long i = (long long)rank * SH_THREADS + tid; i < nitems; i += (long long)CS * SH_THREADS) {
+      long long x = i;
+      int32_t u;
+      if (x < T0) {
+        u = __ldg(P.seeds + bstart + x);
+      } else {
+        x -= T0;
+        int l = 0;
+        while (x >= cnt_l[l]) x -= cnt_l[l++];
+        u = __ldcg(P.rows[l] + bstart * P.K[l] + x);
+      }
+      if (u < 0 || (int64_t)u >= P.N) {
+        atomicOr(P.err, ERR_SEED_RANGE);
+        continue;
+      }
+      const unsigned owner = (unsigned)((uint32_t)u / (uint64_t)bpc);
+      const uint32_t xb = (uint32_t)u - owner * (uint32_t)bpc;
+      atomicOr(cl.map_shared_rank(bm, owner) + (xb >> 5), 1u << (xb & 31));
+    }
+    cl.sync();
+    // ---- local prefix per 256 bits, U ascending ----
+    long long run = 0;
+    for (int g0 = 0; g0 < ngroups; g0 += SH_THREADS) {
+      const int g = g0 + tid;
+      int c = 0;
+      if (g < ngroups)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) c += __popc(bm[g * 8 + i]);
+      int tot;
+      const int ex = block_exclusive_scan<int>(c, ss.scr32, &tot);
+      if (g < ngroups) gp[g] = (int32_t)(run + ex);
+      run += tot;
+    }
+    if (tid == 0) ss.total = run;
+    cl.sync();
+    if (tid < (int)CS) ss.base[tid] = 0;
+    if (tid == 0) {
+      long long acc = 0;
+      for (unsigned r = 0; r < CS; ++r) {
+        ss.base[r] = acc;
+        acc += *cl.map_shared_rank(&ss.total, r);
+      }
+      ss.nU = acc;
+    }
+    __syncthreads();
+    const long long nU = ss.nU;
+    int32_t* U = P.U + b * P.stride;
+    for (int g = tid; g < ngroups; g += SH_THREADS) {
+      long long r = ss.base[rank] + gp[g];
+      for (int i = 0; i < 8; ++i) {
+        uint32_t m = bm[g * 8 + i];
+        while (m) {
+          const int bit = __ffs(m) - 1;
+          m &= m - 1u;
+          U[r++] = (int32_t)((int64_t)rank * bpc + (int64_t)(g * 8 + i) * 32 + bit);
+        }
+      }
+    }
+    __threadfence();
+    cl.sync();
+    // ---- count kept edges per column (this CTA's share of U) ----
+    const long long c_lo = nU * rank / CS, c_hi = nU * (rank + 1) / CS;
+    int32_t* ucnt = P.ucnt + b * P.stride;
+    for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
+      const int32_t v = __ldcg(U + c);
+      const int64_t o = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - o;
+      int cnt = 0;
+      for (int64_t i0 = 0; i0 < d; i0 += 32 * SH_ILP) {  // SH_ILP loads, then tests, in flight
+        uint32_t u[SH_ILP];
+#pragma unroll
+        for (int q = 0; q < SH_ILP; ++q) {
+          const int64_t i = i0 + q * 32 + lane;
+          u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
+        }
+#pragma unroll
+        for (int q = 0; q < SH_ILP; ++q)
+          cnt += __popc(__ballot_sync(0xffffffffu, u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc, u[q])));
+      }
+      if (lane == 0) ucnt[c] = cnt;
+    }
+    __threadfence();
+    cl.sync();
+    // ---- scan: CSC indptr over U, the batch's edge range ----
+    long long erun = 0;
+    for (long long c0 = c_lo; c0 < c_hi; c0 += SH_THREADS) {
+      const long long c = c0 + tid;
+      const int x = c < c_hi ? __ldcg(ucnt + c) : 0;
+      int tot;
+      const int ex = block_exclusive_scan<int>(x, ss.scr32, &tot);
+      if (c < c_hi) ucnt[c] = (int32_t)(erun + ex);  // CTA-local exclusive prefix
+      erun += tot;
+    }
+    if (tid == 0) ss.etotal = erun;
+    cl.sync();
+    if (tid == 0) {
+      long long acc = 0, mine = 0;
+      for (unsigned r = 0; r < CS; ++r) {
+        if (r == rank) mine = acc;
+        acc += *cl.map_shared_rank(&ss.etotal, r);
+      }
+      ss.ebase = mine;
+      ss.E = acc;
+      if (rank == 0) ss.eoff = (long long)atomicAdd(P.edge_ctr, (unsigned long long)acc);
+    }
+    cl.sync();
+    const long long E = ss.E, ebase = ss.ebase;
+    const long long eoff = *cl.map_shared_rank(&ss.eoff, 0);
+    const bool fits = eoff + E <= P.edge_cap;
+    int64_t* ip = P.indptr_out + b * P.stride + b;
+    for (long long c = c_lo + tid; c < c_hi; c += SH_THREADS) ip[c] = ebase + __ldcg(ucnt + c);
+    if (rank == 0 && tid == 0) {
+      ip[nU] = E;
+      long long* m = (long long*)(P.meta + b * 8);
+      m[0] = nU; m[1] = nU; m[2] = E; m[3] = b * P.stride; m[4] = b * P.stride;
+      m[5] = b * P.stride + b; m[6] = fits ? eoff : 0; m[7] = 0;
+      if (!fits) atomicOr(P.err, ERR_CAPACITY);
+    }
+    // ---- write kept edges in CSC order ----
+    if (fits) {
+      for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
+        const int32_t v = __ldcg(U + c);
+        const int64_t o = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - o;
+        long long pos = eoff + ebase + __ldcg(ucnt + c);
+        for (int64_t i0 = 0; i0 < d; i0 += 32 * SH_ILP) {
+          uint32_t u[SH_ILP];
+          bool m[SH_ILP];
+#pragma unroll
+          for (int q = 0; q < SH_ILP; ++q) {
+            const int64_t i = i0 + q * 32 + lane;
+            u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
+          }
+#pragma unroll
+          for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc, u[q]);
+#pragma unroll
+          for (int q = 0; q < SH_ILP; ++q) {
+            const uint32_t bal = __ballot_sync(0xffffffffu, m[q]);
+            if (m[q]) {
+              const long long e = pos + __popc(bal & ((1u << lane) - 1u));
+              sth(P.row_local + e, (int32_t)sh_rank(cl, bm, gp, ss, bpc, u[q]), pf);
+              sth(P.eid + e, (int64_t)(o + i0 + q * 32 + lane), pf);
+            }
+            pos += __popc(bal);
+          }
+        }
+      }
+    }
+    cl.sync();  // the bitmap is reused by the next batch
+  }
+}
+
+gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                     int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                     int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  // cluster size: the N-bit bitmap (+ 1/64 prefix) split over at most 8 CTAs
+  const int64_t N = g->num_nodes;
+  int CS = 1;
+  int64_t bpc = 0;
+  for (; CS <= SH_MAX_CS; CS *= 2) {
+    bpc = ((N + CS - 1) / CS + 255) / 256 * 256;
+    if (bpc / 8 + bpc / 64 <= SH_SMEM_CAP) break;
+  }
+  if (CS > SH_MAX_CS)
+    return fail(GS_ERR_NOT_SUPPORTED, "ShaDow: N = %lld exceeds the shared-memory bitmap envelope (%lld nodes)",
+                (long long)N, (long long)(SH_MAX_CS * (SH_SMEM_CAP * 64 / 9)));
+  // 1. node-wise sampling of every hop (internal result object)
+  if (!blk->aux) {
+    blk->aux = new (std::nothrow) gs_blocks();
+    if (!blk->aux) return fail(GS_ERR_OUT_OF_MEMORY, "host allocation failed");
+    blk->aux->al = blk->al;
+  }
+  blk->aux->stream = stream;
+  gs_status st = run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias,
+                                   key, stream, blk->aux);
+  if (st) return st;
+  const gs_blocks* nw = blk->aux;
+  // 2. induce
+  const Allocator& al = blk->al;
+  const int64_t nbatch = (num_seeds + batch_size - 1) / batch_size;
+  int64_t sumK = 0, prod = 1;
+  for (int l = 0; l < L; ++l) {
+    prod *= fanouts[l];
+    sumK += prod;
+  }
+  const int64_t stride = batch_size * (1 + sumK);
+  const int64_t nodes = nbatch * stride;
+  blk->kind = gs_blocks::SHADOW;
+  blk->num_batches = nbatch;
+  blk->num_layers = 1;
+  blk->stream = stream;
+  blk->synced = false;
+  auto need = [&](DevBuf& b, int64_t bytes) -> bool {
+    return b.ensure(al, (size_t)std::max<int64_t>(bytes, 256), stream);
+  };
+  int64_t edges = std::max<int64_t>(std::max<int64_t>(int64_t(1) << 20, blk->sh_edge_hint), nodes * 4);
+  bool ok = need(blk->b_col[1], nodes * 4) && need(blk->b_indptr[0], (nodes + nbatch) * 8) &&
+            need(blk->b_rowl[0], edges * 4) && need(blk->b_eid[0], edges * 8) &&
+            need(blk->b_row[0], nodes * 4) && need(blk->b_meta, std::max<int64_t>(nbatch, 1) * 64) &&
+            need(blk->b_err, 16) && need(blk->b_ctr, 8 * (MAX_LAYERS + 2));
+  if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (ShaDow buffers)");
+  edges = (int64_t)std::min(blk->b_rowl[0].bytes / 4, blk->b_eid[0].bytes / 8);
+  gs_layer_buffers& lb = blk->layers[0];
+  lb = gs_layer_buffers{};
+  lb.col_map = lb.row_map = (int32_t*)blk->b_col[1].ptr;
+  lb.col_capacity = lb.row_capacity = nodes;
+  lb.indptr = (int64_t*)blk->b_indptr[0].ptr;
+  lb.indptr_capacity = nodes + nbatch;
+  lb.row_local = (int32_t*)blk->b_rowl[0].ptr;
+  lb.eid = (int64_t*)blk->b_eid[0].ptr;
+  lb.edge_capacity = edges;
+
+  SHParams P = {};
+  P.indptr = g->indptr;
+  P.indices = g->indices;
+  P.N = N;
+  P.seeds = seeds;
+  P.num_seeds = num_seeds;
+  P.batch_size = batch_size;
+  P.num_batches = nbatch;
+  P.L = L;
+  for (int l = 0; l < L; ++l) {
+    P.rows[l] = nw->layers[l].row_map;
+    P.K[l] = l == 0 ? fanouts[0] : P.K[l - 1] * fanouts[l];
+  }
+  P.nmeta = (const int64_t*)nw->b_meta.ptr;
+  P.stride = stride;
+  P.U = lb.row_map;
+  P.indptr_out = lb.indptr;
+  P.row_local = lb.row_local;
+  P.eid = lb.eid;
+  P.edge_cap = edges;
+  P.edge_ctr = (unsigned long long*)blk->b_ctr.ptr;
+  P.ucnt = (int32_t*)blk->b_row[0].ptr;
+  P.meta = (int64_t*)blk->b_meta.ptr;
+  P.err = (int*)blk->b_err.ptr;
+  P.claim = (unsigned int*)((char*)blk->b_ctr.ptr + 8 * (MAX_LAYERS + 1));
+  P.bpc = bpc;
+  GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
+  GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
+  if (nbatch == 0) return GS_OK;
+  // the node-wise kernel's error word (out-of-range seeds) is folded in
+  GS_CUDA_TRY(cudaMemcpyAsync(blk->b_err.ptr, nw->b_err.ptr, 4, cudaMemcpyDeviceToDevice, stream));
+
+  const size_t smem = (size_t)(bpc / 8 + bpc / 64);
+  GS_CUDA_TRY(cudaFuncSetAttribute(shadow_induce_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)smem));
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)CS;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.blockDim = dim3(SH_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cfg.gridDim = dim3((unsigned)CS);
+  int nclusters = 0;
+  GS_CUDA_TRY(cudaOccupancyMaxActiveClusters(&nclusters, (void*)shadow_induce_kernel, &cfg));
+  nclusters = (int)std::max<int64_t>(1, std::min<int64_t>(nclusters, nbatch));
+  cfg.gridDim = dim3((unsigned)(nclusters * CS));
+  GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, shadow_induce_kernel, P));
+  return GS_OK;
+}
+
+}  // namespace gsb
