@@ -126,6 +126,23 @@ __global__ void validate_csc_kernel(const int64_t* __restrict__ indptr,
   }
 }
 
+// a0 pre-processing of weighted graphs: colsum[v] = fp32(sum_fp64 of
+// the column's weights) -- the PASS A3 denominator (R11) and the scale of the
+// A-Res candidate threshold (nodewise_wave.cu).
+__global__ void colsum_kernel(const int64_t* __restrict__ indptr, const float* __restrict__ w,
+                              int64_t N, float* __restrict__ colsum) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = warp; v < N; v += nwarps) {
+    const int64_t a = indptr[v], b = indptr[v + 1];
+    double sum = 0.0;
+    for (int64_t i = a + lane; i < b; i += 32) sum += (double)w[i];
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+    if (lane == 0) colsum[v] = (float)sum;
+  }
+}
+
 static int num_sms() {
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -230,6 +247,14 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
   if (vflags & 2) return cleanup(fail(GS_ERR_INVALID_GRAPH, "gs_graph_create: an index is outside [0, num_nodes)"));
   g->sorted = (vflags & 4) ? 0 : 1;
   g->max_in_degree = (int64_t)mdeg;
+  if (g->weights) {
+    if (!g->b_colsum.ensure(g->al, std::max<int64_t>(num_nodes, 1) * 4, stream))
+      return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_create: device allocation failed"));
+    g->colsum = (float*)g->b_colsum.ptr;
+    colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, num_nodes, g->colsum);
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cleanup(cuda_fail(e, "colsum_kernel launch"));
+  }
   cudaMemsetAsync(g->d_err, 0, 64, stream);
   *out = g;
   return GS_OK;
@@ -254,6 +279,7 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_indptr.reset(g->al, s);
   g->b_indices.reset(g->al, s);
   g->b_weights.reset(g->al, s);
+  g->b_colsum.reset(g->al, s);
   g->b_err.reset(g->al, s);
   delete g;
 }

@@ -53,11 +53,12 @@ struct gs_graph {
   int64_t* indptr = nullptr;
   int32_t* indices = nullptr;
   float* weights = nullptr;
+  float* colsum = nullptr;   // weighted graphs: fp32(sum_fp64 w) per column (a0 pre-processing)
   bool owns = false;
   int sorted = 0;
   int64_t max_in_degree = 0;
   gsb::Allocator al;
-  gsb::DevBuf b_indptr, b_indices, b_weights, b_err;
+  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_err;
   int* d_err = nullptr;  // walk error word
 };
 

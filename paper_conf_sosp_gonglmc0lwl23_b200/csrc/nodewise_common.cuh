@@ -1,8 +1,6 @@
 // nodewise_common.cuh -- device building blocks of the node-wise select
-// (Extract + Select fused): per-warp chunks of 32 frontier columns,
-// Floyd / replacement / A-Res positions in shared memory, flattened gather of
-// the sampled rows with NW_ILP loads in flight per lane, staging and the
-// ordered-hash first-occurrence insert.
+// (Extract + Select fused): per-warp chunks of 32 frontier columns and
+// the weighted without-replacement select (A-Res, R6) by candidate filtering.
 #pragma once
 #include <cuda_runtime.h>
 #include <math.h>
@@ -13,45 +11,28 @@
 
 namespace gsb {
 
-constexpr int NW_ILP = 4;  // independent slots per lane in flight
-
 // Read-only graph + sampling parameters shared by the node-wise kernels.
 struct NWCore {
   const int64_t* indptr;
   const int32_t* indices;
   const float* weights;
+  const float* colsum;  // weighted graphs: fp32(sum_fp64 w) per column (a0)
   int64_t N;
   int* err;
   int replace, bias;
   uint64_t key;
 };
 
-// Per-batch-hop staging written by the select step.
-struct NWStage {
-  int32_t* u;      // [slot] sampled row
-  uint32_t* pos;   // [slot] position inside the column
-  float* val;      // [slot] PASS prob (or NULL)
-  int64_t* coff;   // [col] indptr[v]
-  int32_t* ccnt;   // [col] sampled edges of the column
-  unsigned long long* tab;
-};
-
 // Shared memory of one warp's chunk of 32 columns.
 struct WarpChunk {
   uint32_t list[MAX_FANOUT][32];  // positions, [rank][column lane]
-  int64_t coff[32];
+  int64_t coff[32];               // indptr[v]
+  int64_t dcol[32];               // in-degree (0 for an invalid column)
+  int32_t vcol[32];               // frontier node
   int32_t pre[32];                // exclusive prefix of the chunk's counts
   float csum[32];                 // PASS column sums
   int32_t cnt_all[32];            // count; bit 30: positions are 0..cnt-1
 };
-
-__device__ __forceinline__ int pow2ceil_int(int k) { return k <= 1 ? 1 : 1 << (32 - __clz(k - 1)); }
-
-__device__ __forceinline__ int log2_pow2ceil64(int64_t x) {
-  int l = 0;
-  while ((1ll << l) < x) ++l;
-  return l;
-}
 
 __device__ __forceinline__ uint32_t sel_word(const U4& r, int i) {
   return i == 0 ? r.x : (i == 1 ? r.y : (i == 2 ? r.z : r.w));
@@ -81,279 +62,116 @@ __device__ __forceinline__ int chunk_col(const int32_t* pre, int f) {
   return lo;
 }
 
-// A-Res top-k for the chunk's columns (R6): groups of G = pow2ceil(k) lanes
-// stream a column's weights, keep the k smallest (key, position), and write
-// the selected positions (ascending) into list[.][c] and the count into
-// cnt_all[c]; csum[c] = fp32(sum_fp64 w over the whole column) (PASS A3).
-template <typename Out>
-__device__ inline void ares_chunk_t(const NWCore& P, Out out, int l, uint32_t gb, int k,
-                                    int32_t my_v, bool my_valid, int64_t my_off, int64_t my_d) {
-  const int G = pow2ceil_int(k);
-  const int lane = threadIdx.x & 31;
-  const int s = lane & (G - 1), gbase = lane & ~(G - 1);
-  const int gpw = 32 / G;
-  const uint32_t FULL = 0xffffffffu;
-  const uint32_t gbits = (G == 32) ? FULL : (((1u << G) - 1u) << gbase);
-  for (int cb = 0; cb < 32; cb += gpw) {
-    const int c = cb + lane / G;
-    const int32_t v = __shfl_sync(FULL, my_v, c);
-    const bool valid = __shfl_sync(FULL, my_valid ? 1 : 0, c) != 0;
-    const int64_t off = __shfl_sync(FULL, my_off, c);
-    const int64_t dsh = __shfl_sync(FULL, my_d, c);
-    const int64_t d = valid ? dsh : 0;
-    double bk = INFINITY, mk = INFINITY, csum = 0.0;
-    int64_t bp = INT64_MAX, mp = INT64_MAX;
-    int ml = 0;
-    int rounds = valid ? (int)((d + G - 1) / G) : 0;
-    rounds = (int)__reduce_max_sync(FULL, (unsigned)rounds);
-    for (int rd = 0; rd < rounds; ++rd) {
-      const int64_t i = (int64_t)rd * G + s;
-      const bool in = valid && i < d;
-      const float w = in ? (P.weights ? __ldg(P.weights + off + i) : 1.0f) : 0.0f;
-      csum += in ? (double)w : 0.0;
-      const bool elig = in && w > 0.0f;
-      double kk = INFINITY;
-      if (elig) {
-        const U4 r = philox((uint32_t)v, (uint32_t)(i >> 2), ctr2(l, TAG_ARES_NODE), gb, P.key);
-        kk = ares_key(sel_word(r, (int)(i & 3)), (double)w);
-      }
-      uint32_t cand = __ballot_sync(FULL, elig && key_less(kk, i, mk, mp)) & gbits;
-      while (__any_sync(FULL, cand != 0u)) {
-        const int cl = cand ? (__ffs(cand) - 1) : 0;
-        const double ck = __shfl_sync(FULL, kk, cl);
-        const int64_t cp = __shfl_sync(FULL, i, cl);
-        const bool ins = cand != 0u && key_less(ck, cp, mk, mp);
-        if (ins && s == ml) {
-          bk = ck;
-          bp = cp;
-        }
-        if (cand) cand &= cand - 1u;
-        // new group maximum over the k held entries: (key, pos, lane) lexicographic
-        double tk = (s < k) ? bk : -INFINITY;
-        int64_t tp = (s < k) ? bp : -1;
-        int tl = s;
-        for (int o = G >> 1; o > 0; o >>= 1) {
-          const double ok = __shfl_xor_sync(FULL, tk, o);
-          const int64_t op = __shfl_xor_sync(FULL, tp, o);
-          const int ol = __shfl_xor_sync(FULL, tl, o);
-          if (key_less(tk, tp, ok, op) || (tk == ok && tp == op && ol > tl)) {
-            tk = ok;
-            tp = op;
-            tl = ol;
-          }
-        }
-        if (ins) {
-          mk = tk;
-          mp = tp;
-          ml = tl;
-        }
-      }
-    }
-    const bool sel = s < k && bp != INT64_MAX;
-    const uint32_t selb = __ballot_sync(FULL, sel) & gbits;
-    int rnk = 0;
-    for (int i = 0; i < G; ++i) {
-      const int64_t pi = __shfl_sync(FULL, bp, gbase + i);
-      rnk += (((selb >> (gbase + i)) & 1u) && pi < bp) ? 1 : 0;
-    }
-    for (int o = G >> 1; o > 0; o >>= 1) csum += __shfl_xor_sync(FULL, csum, o);
-    if (sel) out.pos(c, rnk, (uint32_t)bp);
-    if (s == 0) out.col(c, __popc(selb), (float)csum);
+// ---------------------------------------------------------------------------
+// A-Res by candidate filtering (R6).  The k smallest exact keys
+// key_i = -ln((r_i + 0.5) 2^-32) / w_i (fp64, as the oracle) are found among
+// the candidates {i : E_lb(r_i) <= tau w_i (1 + 1%)}, a superset of
+// {i : key_i < tau}; whenever at least k exact keys fall below tau those
+// candidates hold the answer.  tau = 2k / W (W = column weight sum) expects
+// ~2k candidates, so only a handful of exact fp64 logarithms are taken per
+// column: the stream costs one Philox per 4 edges, one weight load and one
+// fp32 log per edge.  A tau that yields too few (or too many) is widened (or
+// narrowed) and the column re-streamed -- rare.
+// ---------------------------------------------------------------------------
+// Lower bound of E = -ln((r + 0.5) 2^-32) in fp32.
+__device__ __forceinline__ float ares_e_lb(uint32_t r) {
+  if (r >= 0x80000000u) {  // u >= 1/2: E = -ln(1 - x) >= x + x^2/2
+    const float x = __fmul_rn(__uint2float_rn(0xFFFFFFFFu - r) + 0.5f, 2.3283064365386963e-10f);
+    return __fmaf_rn(0.5f * x, x, x);
   }
-  __syncwarp();
+  const float u = __fmul_rn(__uint2float_rn(r) + 0.5f, 2.3283064365386963e-10f);
+  return -__logf(u) * 0.999f;
 }
 
-struct ChunkOut {
-  WarpChunk* C;
-  __device__ void pos(int c, int r, uint32_t v) const { C->list[r][c] = v; }
-  __device__ void col(int c, int cnt, float cs) const {
-    C->cnt_all[c] = cnt;
-    C->csum[c] = cs;
-  }
+struct AresState {   // per filtering group (warp or CTA), in shared memory
+  int m;             // candidates appended (may exceed the capacity)
+  int elig;          // eligible (w > 0) edges seen
 };
-__device__ inline void ares_chunk(const NWCore& P, WarpChunk& C, int l, uint32_t gb, int k,
-                                  int32_t my_v, bool my_valid, int64_t my_off, int64_t my_d) {
-  ares_chunk_t(P, ChunkOut{&C}, l, gb, k, my_v, my_valid, my_off, my_d);
+
+// Filter pass over column [off, off + d) by a group of NT threads (gtid in
+// [0, NT)); candidate positions are appended to pos[0 .. cap).  tau < 0 means
+// "every eligible edge".  The caller synchronises the group before and after.
+template <int NT>
+__device__ __forceinline__ void ares_filter(const NWCore& P, int32_t v, int64_t off, int64_t d, int l,
+                                            uint32_t gb, float tau, int gtid, uint32_t* pos, int cap,
+                                            AresState* st) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t pf = pol_first();
+  int elig = 0;
+  for (int64_t base = 0; base < d; base += 4 * NT) {
+    const int64_t i0 = base + 4 * (int64_t)gtid;
+    float w[4] = {0.f, 0.f, 0.f, 0.f};
+    uint32_t r[4] = {0u, 0u, 0u, 0u};
+    if (i0 < d) {
+      const U4 R = philox((uint32_t)v, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.key);
+      r[0] = R.x; r[1] = R.y; r[2] = R.z; r[3] = R.w;
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        w[q] = i0 + q < d ? (P.weights ? ldg_h(P.weights + off + i0 + q, pf) : 1.0f) : 0.0f;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const bool e = w[q] > 0.0f;
+      elig += e ? 1 : 0;
+      const bool cand = e && (tau < 0.0f || ares_e_lb(r[q]) <= __fmul_rn(__fmul_rn(tau, w[q]), 1.01f));
+      const uint32_t bal = __ballot_sync(0xffffffffu, cand);
+      if (bal) {
+        int slot0 = 0;
+        if (lane == 0) slot0 = atomicAdd(&st->m, __popc(bal));
+        slot0 = __shfl_sync(0xffffffffu, slot0, 0);
+        const int slot = slot0 + __popc(bal & ((1u << lane) - 1u));
+        if (cand && slot < cap) pos[slot] = (uint32_t)(i0 + q);
+      }
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) elig += __shfl_xor_sync(0xffffffffu, elig, o);
+  if (lane == 0 && elig) atomicAdd(&st->elig, elig);
 }
 
-// Select for one warp chunk of up to 32 columns [jb, min(jb + 32, jend)) of
-// frontier F (batch-local column j -> padded slots j*k .. j*k+k-1), stage the
-// sampled edges and insert every (u, slot) into the ordered hash (first
-// occurrence = minimum slot; kFixed: fixed-position CAS table, safe for
-// lookups concurrent with later inserts).  Returns the chunk's edge count (warp-uniform);
-// C.pre / C.cnt_all describe the chunk afterwards.
-template <bool kFixed = false>
-__device__ inline int select_chunk(const NWCore& P, const NWStage& W, WarpChunk& C, int l, int k,
-                                   int log_cap, uint32_t tag, const int32_t* F, int64_t jb,
-                                   int64_t jend, uint32_t gb, unsigned long long* dbg = nullptr) {
+// Exact step (one warp): fp64 keys of the candidates, then either the k
+// smallest (ascending positions into out[.][c], returns the count) or a
+// verdict: -1 widen tau, -2 narrow tau, -3 collect every eligible edge.
+__device__ __forceinline__ int ares_exact(const NWCore& P, int32_t v, int64_t off, int l, uint32_t gb,
+                                          int k, float tau, const uint32_t* pos, double* key, int* rk, int cap,
+                                          const AresState& st, uint32_t (*out)[32], int c) {
   const int lane = threadIdx.x & 31;
-  const uint64_t pf = pol_first(), pl = pol_last();
-  const int64_t j = jb + lane;
-  const bool active = j < jend;
-  const int32_t v = active ? (kFixed ? ldh(F + j, pl) : __ldcg(F + j)) : -1;
-  const bool valid = active && v >= 0 && (int64_t)v < P.N;
-  if (active && !valid) atomicOr(P.err, ERR_SEED_RANGE);
-  int64_t off = 0, d = 0;
-  if (valid) {
-    off = __ldg(P.indptr + v);
-    d = __ldg(P.indptr + v + 1) - off;
+  const int m = min(st.m, cap);
+  if (st.elig <= k) {  // at most k eligible: all of them (R6)
+    if (tau >= 0.0f) return -3;
+  } else if (st.m > cap) {
+    return -2;
   }
-  int cnt = 0;
-  bool all = false;
-  const bool weighted = !P.replace && P.bias != GS_W_UNIFORM;
-  if (dbg && lane == 0) {
-    unsigned long long tt;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
-    dbg[0] = tt + (unsigned long long)(d & 0);
+  int below = 0;
+  for (int j = lane; j < m; j += 32) {
+    const uint32_t p = pos[j];
+    const U4 R = philox((uint32_t)v, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.key);
+    const float w = P.weights ? __ldg(P.weights + off + p) : 1.0f;
+    const double kk = ares_key(sel_word(R, (int)(p & 3)), (double)w);
+    key[j] = kk;
+    below += (tau < 0.0f || kk < (double)tau) ? 1 : 0;
   }
-  if (weighted) {
-    ares_chunk(P, C, l, gb, k, v, valid, off, d);
-    cnt = C.cnt_all[lane];
-  } else if (P.replace) {
-    // KGCN (R10): k i.i.d. uniform positions in slot order.
-    cnt = d > 0 ? k : 0;
-    for (int s = 0; s < cnt; ++s) {
-      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.key);
-      C.list[s][lane] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
-    }
-  } else if (d <= k) {
-    // GraphSAGE, d <= k: every neighbour, no randomness (R5)
-    cnt = (int)d;
-    all = true;
-  } else {
-    // GraphSAGE (R5): Floyd's algorithm; the list is kept sorted (m exceeds
-    // every element chosen so far, so it is appended).
-    cnt = k;
-    int n = 0;
-    for (int s = 0; s < k; ++s) {
-      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.key);
-      const uint32_t m = (uint32_t)(d - k + s);
-      const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
-      int lo = 0, hi = n;
-      while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (C.list[mid][lane] < t) lo = mid + 1;
-        else hi = mid;
-      }
-      if (lo < n && C.list[lo][lane] == t) {
-        C.list[n][lane] = m;
-      } else {
-        for (int q = n; q > lo; --q) C.list[q][lane] = C.list[q - 1][lane];
-        C.list[lo][lane] = t;
-      }
-      ++n;
-    }
-  }
-  int total;
-  const int pre = warp_excl(cnt, &total);
-  if (dbg && lane == 0) {
-    unsigned long long tt;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
-    dbg[1] = tt;
-  }
-  C.coff[lane] = off;
-  C.pre[lane] = pre;
-  if (!weighted) C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
-  if (active) {
-    if (kFixed) {
-      sth(W.coff + j, off, pl);
-      sth(W.ccnt + j, cnt, pl);
-    } else {
-      W.coff[j] = off;
-      W.ccnt[j] = cnt;
-    }
+  for (int o = 16; o > 0; o >>= 1) below += __shfl_xor_sync(0xffffffffu, below, o);
+  __syncwarp();
+  const int want = min(k, st.elig);
+  if (below < want) return -1;
+  // rank by (key, position); the selected ones are then ordered by position
+  for (int j = lane; j < m; j += 32) {
+    const double kj = key[j];
+    const uint32_t pj = pos[j];
+    int r = 0;
+    for (int i = 0; i < m; ++i) r += key_less(key[i], pos[i], kj, pj) ? 1 : 0;
+    rk[j] = r;
   }
   __syncwarp();
-  // Flattened gather + stage + insert: flat slot f of the chunk -> column c, rank s.
-  const uint32_t mask = (1u << log_cap) - 1u;
-  for (int f0 = 0; f0 < total; f0 += 32 * NW_ILP) {
-    int32_t u[NW_ILP];
-    int64_t p[NW_ILP];
-    uint32_t ps[NW_ILP];
-    int cc[NW_ILP];
-    bool ok[NW_ILP];
-#pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) {
-      const int f = f0 + i * 32 + lane;
-      ok[i] = f < total;
-      cc[i] = 0;
-      p[i] = 0;
-      ps[i] = 0;
-      u[i] = 0;
-      if (ok[i]) {
-        const int c = chunk_col(C.pre, f);
-        const int s = f - C.pre[c];
-        ps[i] = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)s : C.list[s][c];
-        p[i] = (jb + c) * k + s;
-        u[i] = kFixed ? ldg_h(P.indices + C.coff[c] + ps[i], pf)
-                      : __ldg(P.indices + C.coff[c] + ps[i]);
-        cc[i] = c;
-      }
-    }
-    unsigned long long old[NW_ILP], carry[NW_ILP];
-    uint32_t h[NW_ILP];
-#pragma unroll
-    for (int i = 0; i < NW_ILP; ++i) {
-      h[i] = 0;
-      carry[i] = 0;
-      if (ok[i]) {
-        if (kFixed) {
-          sth(W.u + p[i], u[i], pl);
-          sth(W.pos + p[i], ps[i], pl);
-        } else {
-          W.u[p[i]] = u[i];
-          W.pos[p[i]] = ps[i];
-        }
-        if (W.val) {
-          const float w = P.weights ? __ldg(P.weights + C.coff[cc[i]] + ps[i]) : 1.0f;
-          W.val[p[i]] = w / C.csum[cc[i]];
-        }
-        h[i] = tab_hash((uint32_t)u[i], log_cap);
-        carry[i] = kFixed ? ct_entry((uint32_t)u[i], (uint32_t)p[i])
-                          : tab_entry(tag, (uint32_t)u[i], (uint32_t)p[i]);
-      }
-    }
-    if (kFixed) {
-      // Hot rows (hubs) recur in many columns: a CAS per occurrence would
-      // serialise on one L2 address.  Only the first occurrence inside the
-      // warp (lowest lane = smallest slot) proceeds, and it first reads the
-      // home slot: a row already holding a smaller slot needs no atomic.
-      bool go[NW_ILP];
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i) {
-        const uint32_t peers = __match_any_sync(0xffffffffu, ok[i] ? (uint32_t)u[i] : 0xFFFFFFFFu);
-        go[i] = ok[i] && (__ffs(peers) - 1) == lane;
-        old[i] = go[i] ? ldh(&W.tab[h[i]], pl) : 0ull;
-      }
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i) {
-        if (!go[i]) continue;
-        if (old[i] != CT_EMPTY && (old[i] >> TAB_VAL_BITS) == (carry[i] >> TAB_VAL_BITS) &&
-            old[i] <= carry[i]) {
-          go[i] = false;  // present with an earlier slot
-          continue;
-        }
-        old[i] = atom_cas_h(&W.tab[h[i]], CT_EMPTY, carry[i], pl);
-      }
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i)
-        if (go[i]) ct_finish(W.tab, mask, h[i], carry[i], old[i], pl);
-    } else {
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i)
-        if (ok[i]) old[i] = atomicMin(&W.tab[h[i]], carry[i]);
-#pragma unroll
-      for (int i = 0; i < NW_ILP; ++i)
-        if (ok[i]) otab_finish(W.tab, mask, tag, h[i], carry[i], old[i]);
-    }
+  for (int j = lane; j < m; j += 32) {
+    if (rk[j] >= want) continue;
+    const uint32_t pj = pos[j];
+    int o = 0;
+    for (int i = 0; i < m; ++i) o += (rk[i] < want && pos[i] < pj) ? 1 : 0;
+    out[o][c] = pj;
   }
   __syncwarp();
-  if (dbg && lane == 0) {
-    unsigned long long tt;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tt));
-    dbg[2] = tt;
-  }
-  return total;
+  return want;
 }
 
 }  // namespace gsb

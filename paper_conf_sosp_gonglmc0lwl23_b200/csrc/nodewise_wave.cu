@@ -116,24 +116,56 @@ __device__ __forceinline__ unsigned long long gtimer_ns() {
 }
 
 struct NVSeg {
-  long long b, T;
-  int j, l, g, st;
-  long long task0;          // exclusive prefix of tasks over the step's segments
+  long long b;
+  int T;                    // frontier columns (< 2^25)
+  int task0;                // exclusive prefix of tasks over the step's segments
+  int g;
+  short j;
+  unsigned char l, st;
 };
 
+struct NVTileC {            // stage C's per-tile arrays
+  int32_t sceo[NV_TC];
+  int32_t scnt[NV_TC];
+  int64_t scoff[NV_TC];
+};
+
+// Kept small: two CTAs per SM plus as much L1 as possible (the carveout is
+// the smallest that fits both CTAs' shared memory).
 struct NVSmem {
-  WarpChunk wc[NV_WARPS];
+  union {
+    WarpChunk wc[NV_WARPS];  // stage A
+    NVTileC tc;              // stage C (tasks never overlap inside a CTA)
+  };
   NVSeg seg[NV_MAXSEG];
   long long ntasks;
   int nseg;
   long long work;
-  int32_t sceo[NV_TC];
-  int32_t scnt[NV_TC];
-  int64_t scoff[NV_TC];
   int wtot[NV_WARPS];
   int flag;
   long long scr64[40];
   int scr32[40];
+};
+
+constexpr int NV_WCAP = 128;      // A-Res candidates per warp
+constexpr int NV_CCAP = 512;      // A-Res candidates per CTA (heavy columns)
+constexpr int64_t NV_DHEAVY = 2048;  // columns above this are filtered by the whole CTA
+
+struct NVWarpA {
+  uint32_t pos[NV_WCAP];
+  double key[NV_WCAP];
+  int rk[NV_WCAP];
+  AresState st;
+};
+
+struct NVWeighted {  // weighted mode only: placed after NVSmem in dynamic shared memory
+  NVWarpA a[NV_WARPS];
+  uint32_t hpos[NV_CCAP];
+  double hkey[NV_CCAP];
+  int hrk[NV_CCAP];
+  AresState hst;
+  int hres, nheavy;
+  int heavy[NV_TC];
 };
 
 __device__ __forceinline__ int nv_find_seg(const NVSmem& sm, long long x) {
@@ -182,7 +214,7 @@ __device__ void nv_segments(const NVParams& P, NVSmem& sm, int s) {
   const int live = (b >= 0) ? 1 : 0;
   int nlive;
   const int pos = block_exclusive_scan<int>(live, sm.scr32, &nlive);
-  if (live) sm.seg[pos] = NVSeg{b, T, j, l, g, st, x};
+  if (live) sm.seg[pos] = NVSeg{b, (int)T, (int)x, g, (short)j, (unsigned char)l, (unsigned char)st};
   if (tid == 0) sm.nseg = nlive;
   __syncthreads();
 }
@@ -190,7 +222,251 @@ __device__ void nv_segments(const NVParams& P, NVSmem& sm, int s) {
 // ---------------------------------------------------------------------------
 // Stage A: select + gather + bitmap insert for one chunk of 32 columns.
 // ---------------------------------------------------------------------------
-__device__ int nv_chunk(const NVParams& P, WarpChunk& C, const NVSeg& sg, long long jb) {
+// Per lane: the chunk's column jb + lane (v, indptr[v], in-degree) into C.
+__device__ __forceinline__ void nv_cols(const NVParams& P, WarpChunk& C, const NVSeg& sg, long long jb,
+                                        int32_t& v_out, int64_t& d_out) {
+  const int lane = threadIdx.x & 31;
+  const int32_t* F = nv_frontier(P, sg.b, sg.l);
+  const long long jcol = jb + lane;
+  const bool active = jcol < sg.T;
+  const int32_t v = active ? __ldcg(F + jcol) : -1;
+  const bool valid = active && v >= 0 && (int64_t)v < P.core.N;
+  if (active && !valid) atomicOr(P.core.err, ERR_SEED_RANGE);
+  int64_t off = 0, d = 0;
+  if (valid) {
+    off = __ldg(P.core.indptr + v);
+    d = __ldg(P.core.indptr + v + 1) - off;
+  }
+  C.vcol[lane] = v;
+  C.coff[lane] = off;
+  C.dcol[lane] = d;
+  C.csum[lane] = 1.0f;
+  v_out = v;
+  d_out = d;
+}
+
+// Uniform select (GraphSAGE Floyd, R5; KGCN replacement, R10), lane per column.
+// (v, d in registers: the Floyd loop stores into C.list, which would force
+// reloads of anything read back from the same shared-memory struct)
+__device__ void nv_select_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg, const int32_t v,
+                                  const int64_t d) {
+  const int lane = threadIdx.x & 31;
+  const int l = sg.l, k = P.k[l];
+  const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
+  int cnt = 0;
+  bool all = false;
+  if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
+    cnt = d > 0 ? k : 0;
+    for (int s = 0; s < cnt; ++s) {
+      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
+      C.list[s][lane] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
+    }
+  } else if (d <= k) {  // GraphSAGE, d <= k: every neighbour (R5)
+    cnt = (int)d;
+    all = true;
+  } else {  // GraphSAGE (R5): Floyd; the list stays sorted (m is always appended)
+    cnt = k;
+    int n = 0;
+    for (int s = 0; s < k; ++s) {
+      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.core.key);
+      const uint32_t m = (uint32_t)(d - k + s);
+      const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
+      int lo = 0, hi = n;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (C.list[mid][lane] < t) lo = mid + 1;
+        else hi = mid;
+      }
+      if (lo < n && C.list[lo][lane] == t) {
+        C.list[n][lane] = m;
+      } else {
+        for (int q = n; q > lo; --q) C.list[q][lane] = C.list[q - 1][lane];
+        C.list[lo][lane] = t;
+      }
+      ++n;
+    }
+  }
+  C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
+}
+
+// A-Res threshold search state: tau is widened / narrowed geometrically, or
+// bisected once both a too-small and a too-large value are known.
+struct TauSearch {
+  float tau, lo, hi;
+  __device__ bool next(int verdict, float tau0) {  // false: give up
+    if (verdict == -3) { tau = -1.0f; return true; }
+    if (verdict == -1) lo = tau;                     // too few below tau
+    else hi = tau < 0.0f ? tau0 * 4.0f : tau;        // too many candidates
+    if (lo > 0.0f && hi > 0.0f) {
+      if (hi <= lo * 1.0001f) return false;
+      tau = sqrtf(lo * hi);
+    } else {
+      tau = lo > 0.0f ? lo * 4.0f : hi * 0.25f;
+    }
+    return true;
+  }
+};
+
+__device__ __forceinline__ float nv_tau0(const NVParams& P, int k, int32_t v, int64_t d) {
+  const float W = P.core.weights ? __ldg(P.core.colsum + v) : (float)d;
+  return W > 0.0f ? 2.0f * (float)k / W : -1.0f;
+}
+
+// Weighted select (A-Res, R6), phase 1 (warp): columns with d <= k take every
+// eligible edge (lane per column); k < d <= NV_DHEAVY are filtered by the whole
+// warp one at a time; heavier columns are queued for the CTA (phase 2).
+__device__ void nv_select_weighted(const NVParams& P, NVSmem& sm, NVWeighted& W, WarpChunk& C,
+                                   const NVSeg& sg) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int l = sg.l, k = P.k[l];
+  const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
+  const int32_t v = C.vcol[lane];
+  const int64_t off = C.coff[lane], d = C.dcol[lane];
+  if (d > 0) C.csum[lane] = P.core.weights ? __ldg(P.core.colsum + v) : (float)d;  // PASS A3 denominator
+  int cnt = 0;
+  if (d <= k) {
+    for (int i = 0; i < (int)d; ++i) {
+      const float w = P.core.weights ? __ldg(P.core.weights + off + i) : 1.0f;
+      if (w > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
+    }
+  }
+  C.cnt_all[lane] = cnt;
+  if (d > NV_DHEAVY) W.heavy[atomicAdd(&W.nheavy, 1)] = (warp << 5) | lane;
+  NVWarpA& A = W.a[warp];
+  uint32_t med = __ballot_sync(0xffffffffu, d > k && d <= NV_DHEAVY);
+  while (med) {
+    const int c = __ffs(med) - 1;
+    med &= med - 1u;
+    const int32_t vc = C.vcol[c];
+    const int64_t oc = C.coff[c], dc = C.dcol[c];
+    const float tau0 = dc <= 64 ? -1.0f : nv_tau0(P, k, vc, dc);
+    TauSearch ts{tau0, 0.0f, 0.0f};
+    int r;
+    while (true) {
+      if (lane == 0) A.st = AresState{0, 0};
+      __syncwarp();
+      ares_filter<32>(P.core, vc, oc, dc, l, gb, ts.tau, lane, A.pos, NV_WCAP, &A.st);
+      __syncwarp();
+      r = ares_exact(P.core, vc, oc, l, gb, k, ts.tau, A.pos, A.key, A.rk, NV_WCAP, A.st, C.list, c);
+      if (r >= 0) break;
+      if (!ts.next(r, tau0 > 0.0f ? tau0 : 2.0f * k / (float)dc)) {
+        if (lane == 0) atomicOr(P.core.err, ERR_INTERNAL);
+        r = 0;
+        break;
+      }
+    }
+    if (lane == 0) C.cnt_all[c] = r;
+    __syncwarp();
+  }
+}
+
+// Weighted select, phase 2 (whole CTA): the queued heavy columns one by one.
+__device__ void nv_select_heavy(const NVParams& P, NVSmem& sm, NVWeighted& W, const NVSeg& sg) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int l = sg.l, k = P.k[l];
+  const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
+  const int nh = W.nheavy;
+  for (int h = 0; h < nh; ++h) {
+    const int e = W.heavy[h];
+    WarpChunk& C = sm.wc[e >> 5];
+    const int c = e & 31;
+    const int32_t v = C.vcol[c];
+    const int64_t off = C.coff[c], d = C.dcol[c];
+    const float tau0 = nv_tau0(P, k, v, d);
+    TauSearch ts{tau0, 0.0f, 0.0f};
+    while (true) {
+      if (threadIdx.x == 0) W.hst = AresState{0, 0};
+      __syncthreads();
+      ares_filter<NV_THREADS>(P.core, v, off, d, l, gb, ts.tau, threadIdx.x, W.hpos, NV_CCAP, &W.hst);
+      __syncthreads();
+      if (warp == 0) {
+        const int r = ares_exact(P.core, v, off, l, gb, k, ts.tau, W.hpos, W.hkey, W.hrk, NV_CCAP,
+                                 W.hst, C.list, c);
+        if (lane == 0) W.hres = r;
+      }
+      __syncthreads();
+      const int r = W.hres;
+      __syncthreads();
+      if (r >= 0) {
+        if (threadIdx.x == 0) C.cnt_all[c] = r;
+        break;
+      }
+      if (!ts.next(r, tau0 > 0.0f ? tau0 : 2.0f * k / (float)d)) {
+        if (threadIdx.x == 0) {
+          atomicOr(P.core.err, ERR_INTERNAL);
+          C.cnt_all[c] = 0;
+        }
+        break;
+      }
+    }
+  }
+  __syncthreads();
+}
+
+// Stage A, per warp after the select: stage the positions, gather every
+// sampled row of the chunk at once and set the rows' bits.  Returns the
+// chunk's edge count.
+__device__ int nv_gather(const NVParams& P, WarpChunk& C, const NVSeg& sg, long long jb) {
+  const int lane = threadIdx.x & 31;
+  const int l = sg.l;
+  const int k = P.k[l];
+  const NVStage S = nv_stage(P, sg.j, l, sg.g);
+  const uint64_t pf = pol_first(), pl = pol_last();
+  const long long jcol = jb + lane;
+  const int cnt = C.cnt_all[lane] & ~(1 << 30);
+  int total;
+  const int pre = warp_excl(cnt, &total);
+  C.pre[lane] = pre;
+  if (jcol < sg.T) {
+    sth(S.coff + jcol, C.coff[lane], pl);
+    sth(S.cnt + jcol, cnt, pl);
+  }
+  __syncwarp();
+  // (a) every sampled row of the chunk is requested at once: cp.async of the
+  // gathered id straight into the position's own list cell (the position is
+  // read, and staged, before its cell is overwritten)
+  for (int f = lane; f < total; f += 32) {
+    const int c = chunk_col(C.pre, f);
+    const int q = f - C.pre[c];
+    const uint32_t ps = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)q : C.list[q][c];
+    const uint32_t p = (uint32_t)((jb + c) * k + q);
+    sth(S.pos + p, ps, pl);
+    if (S.val) {
+      const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
+      sth(S.val + p, w / C.csum[c], pl);
+    }
+    const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
+                 "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  __syncwarp();
+  // (b) stage the rows and set their bits in the segment's row bitmap
+  // (fire-and-forget red.or; a row's bit is set once per warp round)
+  for (int f0 = 0; f0 < total; f0 += 32) {
+    const int f = f0 + lane;
+    uint32_t u = 0xFFFFFFFFu;
+    if (f < total) {
+      const int c = chunk_col(C.pre, f);
+      const int q = f - C.pre[c];
+      u = C.list[q][c];
+      sth(S.u + (jb + c) * k + q, (int32_t)u, pl);
+    }
+    const uint32_t peers = __match_any_sync(0xffffffffu, u);
+    if (f < total && (__ffs(peers) - 1) == lane)
+      asm volatile("red.global.or.b32 [%0], %1;" ::"l"((uint32_t*)(S.bm + (u >> 5))),
+                   "r"(1u << (u & 31))
+                   : "memory");
+  }
+  __syncwarp();
+  return total;
+}
+
+// Stage A for the uniform modes: select + gather of one chunk in one pass
+// (column data stay in registers).
+__device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg, long long jb) {
   const int lane = threadIdx.x & 31;
   const int l = sg.l;
   const int k = P.k[l];
@@ -208,13 +484,10 @@ __device__ int nv_chunk(const NVParams& P, WarpChunk& C, const NVSeg& sg, long l
     off = __ldg(P.core.indptr + v);
     d = __ldg(P.core.indptr + v + 1) - off;
   }
-  const bool weighted = !P.core.replace && P.core.bias != GS_W_UNIFORM;
+  const bool weighted = false;
   int cnt = 0;
   bool all = false;
-  if (weighted) {
-    ares_chunk(P.core, C, l, gb, k, v, valid, off, d);
-    cnt = C.cnt_all[lane];
-  } else if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
+  if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
     cnt = d > 0 ? k : 0;
     for (int s = 0; s < cnt; ++s) {
       const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
@@ -298,10 +571,29 @@ __device__ int nv_chunk(const NVParams& P, WarpChunk& C, const NVSeg& sg, long l
 }
 
 // Stage A tile: 512 columns, one 32-column chunk per warp; the tile's edge count.
+template <bool WEIGHTED>
 __device__ void nv_stage_a(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long jb = (long long)t * NV_TC + warp * 32;
-  const int e = jb < sg.T ? nv_chunk(P, sm.wc[warp], sg, jb) : 0;
+  const bool has = jb < sg.T;
+  WarpChunk& C = sm.wc[warp];
+  int e = 0;
+  if (WEIGHTED) {
+    NVWeighted& W = *reinterpret_cast<NVWeighted*>(&sm + 1);
+    if (threadIdx.x == 0) W.nheavy = 0;
+    __syncthreads();
+    if (has) {
+      int32_t v;
+      int64_t d;
+      nv_cols(P, C, sg, jb, v, d);
+      nv_select_weighted(P, sm, W, C, sg);
+    }
+    __syncthreads();
+    nv_select_heavy(P, sm, W, sg);
+    if (has) e = nv_gather(P, C, sg, jb);
+  } else if (has) {
+    e = nv_chunk_uniform(P, C, sg, jb);
+  }
   if (lane == 0) sm.wtot[warp] = e;
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -399,9 +691,9 @@ __device__ void nv_stage_c(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
     int tot;
     const int ex = block_exclusive_scan<int>(c, sm.scr32, &tot);
     if (jl < ncols) {
-      sm.sceo[jl] = ex;
-      sm.scnt[jl] = c;
-      sm.scoff[jl] = __ldcg(S.coff + c0 + jl);
+      sm.tc.sceo[jl] = ex;
+      sm.tc.scnt[jl] = c;
+      sm.tc.scoff[jl] = __ldcg(S.coff + c0 + jl);
       sth(P.indptr_out[l] + ibase + c0 + jl, (int64_t)(xe + ex), pf);
       if (l == 0) sth(P.col0 + bstart + c0 + jl, __ldcg(P.seeds + bstart + c0 + jl), pf);
     }
@@ -421,7 +713,7 @@ __device__ void nv_stage_c(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
       vv[i] = false;
       if (r < nslots) {
         const int jl = r / k, q = r - jl * k;
-        vv[i] = q < sm.scnt[jl];
+        vv[i] = q < sm.tc.scnt[jl];
       }
       uu[i] = vv[i] ? (uint32_t)ldh(S.u + s0 + r, pl) : 0u;
       ps[i] = vv[i] ? ldh(S.pos + s0 + r, pl) : 0u;
@@ -438,12 +730,12 @@ __device__ void nv_stage_c(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
       if (!vv[i]) continue;
       const int r = r0 + i * NV_THREADS;
       const int jl = r / k, q = r - jl * k;
-      const long long e = xe + sm.sceo[jl] + q;
+      const long long e = xe + sm.tc.sceo[jl] + q;
       const long long lid = (long long)bx[i] + (long long)(wd[i] >> 32) +
                             __popc((uint32_t)wd[i] & ((1u << (uu[i] & 31)) - 1u));
       sth(row_local + e, (int32_t)lid, pf);
       sth(row_map + lid, (int32_t)uu[i], pf);  // every slot of the row writes the same id
-      sth(eid_out + e, (int64_t)(sm.scoff[jl] + ps[i]), pf);
+      sth(eid_out + e, (int64_t)(sm.tc.scoff[jl] + ps[i]), pf);
       if (val_out) sth(val_out + e, ldh(S.val + s0 + r, pl), pf);
     }
   }
@@ -461,6 +753,9 @@ __device__ void nv_stage_z(const NVParams& P, const NVSeg& sg, int t) {
     S.bm[__ldcg(rows + i) >> 5] = 0ull;
 }
 
+// WEIGHTED: A-Res / PASS select (its own instantiation: the uniform kernel
+// carries none of the weighted code, which would cost it registers / ILP).
+template <bool WEIGHTED>
 __global__ void __launch_bounds__(NV_THREADS, 2) nodewise_wave_kernel(NVParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   NVSmem& sm = *reinterpret_cast<NVSmem*>(smem_raw);
@@ -482,7 +777,7 @@ __global__ void __launch_bounds__(NV_THREADS, 2) nodewise_wave_kernel(NVParams P
       if (P.trace2 && threadIdx.x == 0) t_start = gtimer_ns();
       switch (sg.st) {
         case ST_B: nv_stage_b(P, sm, sg, t, &ctr[4 + si]); break;
-        case ST_A: nv_stage_a(P, sm, sg, t); break;
+        case ST_A: nv_stage_a<WEIGHTED>(P, sm, sg, t); break;
         case ST_C: nv_stage_c(P, sm, sg, t); break;
         default: nv_stage_z(P, sg, t); break;
       }
@@ -514,6 +809,7 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   P.core.indptr = g->indptr;
   P.core.indices = g->indices;
   P.core.weights = g->weights;
+  P.core.colsum = g->colsum;
   P.core.N = g->num_nodes;
   P.core.replace = replace;
   P.core.bias = bias;
@@ -631,17 +927,24 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_sched.ptr, 0, ctr_bytes, stream));
   if (nbatch == 0) return GS_OK;
 
-  static int grid = 0;
+  // dynamic shared memory: the A-Res candidate buffers only in weighted mode;
+  // cooperative grid = every CTA co-resident
+  const bool weighted = !replace && bias != GS_W_UNIFORM;
+  const size_t smem = sizeof(NVSmem) + (weighted ? sizeof(NVWeighted) : 0);
+  static int grid_for[2] = {0, 0};
+  int& grid = grid_for[weighted ? 1 : 0];
+  void* kfn = weighted ? (void*)nodewise_wave_kernel<true> : (void*)nodewise_wave_kernel<false>;
+  GS_CUDA_TRY(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)smem));
   if (grid == 0) {
-    GS_CUDA_TRY(cudaFuncSetAttribute(nodewise_wave_kernel,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)sizeof(NVSmem)));
     int per_sm = 0, dev = 0, sms = 148;
-    GS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, nodewise_wave_kernel,
-                                                              NV_THREADS, sizeof(NVSmem)));
+    GS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn,
+                                                              NV_THREADS, smem));
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     grid = std::max(1, per_sm) * sms;
+    if (getenv("GS_VERBOSE"))
+      fprintf(stderr, "nodewise_wave: smem %zu B, %d CTAs/SM, grid %d\n", smem, per_sm, grid);
   }
   const char* trace_path = getenv("GS_TRACE");
   const size_t tr2 = (size_t)P.S * 4096 * 24;
@@ -651,8 +954,8 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
     GS_CUDA_TRY(cudaMemsetAsync(P.trace2, 0, tr2, stream));
   }
   void* args[] = {&P};
-  GS_CUDA_TRY(cudaLaunchCooperativeKernel((void*)nodewise_wave_kernel, dim3(grid),
-                                          dim3(NV_THREADS), args, sizeof(NVSmem), stream));
+  GS_CUDA_TRY(cudaLaunchCooperativeKernel(kfn, dim3(grid),
+                                          dim3(NV_THREADS), args, smem, stream));
   if (trace_path) {  // tracing aid: per-super-step timestamps
     std::vector<unsigned long long> h((size_t)P.S * 4);
     GS_CUDA_TRY(cudaStreamSynchronize(stream));

@@ -91,6 +91,7 @@ def load_library(path: str = LIB_PATH):
     global _lib
     if _lib is not None:
         return _lib
+    path = os.environ.get("GS_LIB_PATH", path)  # A/B experiments against another build
     if not os.path.exists(path):
         raise ImportError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
     L = ctypes.CDLL(path)
