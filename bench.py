@@ -180,11 +180,12 @@ def _secs(off, d):
     return torch.where(d > 0, ((off + d - 1) >> 3) - (off >> 3) + 1, torch.zeros_like(d))
 
 
-def _blocks_byte_model(blocks, g, kind, weighted, L):
+def _blocks_byte_model(blocks, g, kind, weighted, L, weighted_select=False):
     """Algorithmic bytes of one step (SURVEY.md 8(d) byte model).
     node-wise, per column: 4 (frontier id) + 32*(1 + [v%4==3]) (int64 indptr pair)
       + 32 * distinct sectors of the sampled positions (the column when d <= k)
       + 8 (block indptr); per edge 12 (row_local + eid); per row 4 (row_map).
+    weighted node-wise (A-Res / PASS): + 32 * sectors of the column's weights.
     shadow: per U node the whole column streamed once (4 + 32(1+straddle) +
       32 secs(off, d)) + 12 per induced edge + 4 per node.
     layer-wise: every frontier column streamed twice (indices, + weights for
@@ -219,6 +220,8 @@ def _blocks_byte_model(blocks, g, kind, weighted, L):
                 cid = torch.repeat_interleave(torch.arange(cnt.numel(), device=cnt.device), cnt)
                 sec += torch.unique(cid * (1 << 40) + (eids >> 3)).numel()
             total += ncols * 12 + 32 * (ncols + straddle) + 32 * sec
+            if weighted_select:  # A-Res streams every weight of the column
+                total += 32 * int(_secs(off, d).sum())
         elif kind == "shadow":
             total += ncols * 4 + 32 * (ncols + straddle) + 32 * int(_secs(off, d).sum())
         else:
@@ -385,7 +388,7 @@ def run_gpu(args, wl, world, rank, device):
             return edges * (32 + 32 + 4) + 32 * straddle, edges
         out.sync()
         return _blocks_byte_model(out, g, kind, g["weights"] is not None and wl.get("mode") == 0,
-                                  L)
+                                  L, weighted_select=kind == "nodewise" and wl.get("bias", 0) != 0)
 
     if kind in ("shadow", "layerwise"):
         grow_until_fits()

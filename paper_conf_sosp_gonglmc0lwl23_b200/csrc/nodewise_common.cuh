@@ -73,14 +73,18 @@ __device__ __forceinline__ int chunk_col(const int32_t* pre, int f) {
 // fp32 log per edge.  A tau that yields too few (or too many) is widened (or
 // narrowed) and the column re-streamed -- rare.
 // ---------------------------------------------------------------------------
-// Lower bound of E = -ln((r + 0.5) 2^-32) in fp32.
-__device__ __forceinline__ float ares_e_lb(uint32_t r) {
-  if (r >= 0x80000000u) {  // u >= 1/2: E = -ln(1 - x) >= x + x^2/2
+// Candidate test E(r) <= t (conservatively: never rejects a true candidate)
+// for E(r) = -ln((r + 0.5) 2^-32).  For r >= 2^31, E = -ln(1 - x) >= x + x^2/2
+// with x = (2^32 - r - 0.5) 2^-32; for r < 2^31, E >= ln 2, so with
+// t < 0.69 (the usual case: tau w is small) no logarithm is taken at all.
+__device__ __forceinline__ bool ares_maybe_below(uint32_t r, float t) {
+  if (r >= 0x80000000u) {
     const float x = __fmul_rn(__uint2float_rn(0xFFFFFFFFu - r) + 0.5f, 2.3283064365386963e-10f);
-    return __fmaf_rn(0.5f * x, x, x);
+    return __fmaf_rn(0.5f * x, x, x) <= t;
   }
+  if (t < 0.69f) return false;
   const float u = __fmul_rn(__uint2float_rn(r) + 0.5f, 2.3283064365386963e-10f);
-  return -__logf(u) * 0.999f;
+  return -__logf(u) * 0.999f <= t;
 }
 
 struct AresState {   // per filtering group (warp or CTA), in shared memory
@@ -113,7 +117,7 @@ __device__ __forceinline__ void ares_filter(const NWCore& P, int32_t v, int64_t 
     for (int q = 0; q < 4; ++q) {
       const bool e = w[q] > 0.0f;
       elig += e ? 1 : 0;
-      const bool cand = e && (tau < 0.0f || ares_e_lb(r[q]) <= __fmul_rn(__fmul_rn(tau, w[q]), 1.01f));
+      const bool cand = e && (tau < 0.0f || ares_maybe_below(r[q], __fmul_rn(__fmul_rn(tau, w[q]), 1.01f)));
       const uint32_t bal = __ballot_sync(0xffffffffu, cand);
       if (bal) {
         int slot0 = 0;

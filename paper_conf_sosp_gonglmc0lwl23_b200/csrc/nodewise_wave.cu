@@ -147,8 +147,8 @@ struct NVSmem {
   int scr32[40];
 };
 
-constexpr int NV_WCAP = 128;      // A-Res candidates per warp
-constexpr int NV_CCAP = 512;      // A-Res candidates per CTA (heavy columns)
+constexpr int NV_WCAP = 64;       // A-Res candidates per warp (expected ~2k)
+constexpr int NV_CCAP = 256;      // A-Res candidates per CTA (heavy columns)
 constexpr int64_t NV_DHEAVY = 2048;  // columns above this are filtered by the whole CTA
 
 struct NVWarpA {
