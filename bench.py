@@ -368,15 +368,17 @@ def run_gpu(args, wl, world, rank, device):
                            rng_key=key, stream=stream, out=traces)
 
     def grow_until_fits():
-        # layer-wise / ShaDow outputs are sized on the device: grow before timing
-        for _ in range(4):
-            step(0)
-            try:
-                out.sync()
-                return
-            except gs.GSError as e:
-                if e.status != 7:
-                    raise
+        # layer-wise / ShaDow outputs are sized on the device: every rng key the
+        # run will use is tried (and the buffers grown) before anything is timed
+        for i in range(args.warmup + args.steps):
+            for _ in range(6):
+                step(i)
+                try:
+                    out.sync()
+                    break
+                except gs.GSError as e:
+                    if e.status != 7:
+                        raise
 
     def account():
         if kind == "walk":

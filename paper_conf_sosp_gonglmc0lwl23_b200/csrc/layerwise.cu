@@ -28,7 +28,7 @@
 
 namespace gsb {
 
-constexpr int LW_THREADS = 512;
+constexpr int LW_THREADS = 1024;  // one CTA per SM: 148 batches in flight keep their tables L2-resident
 constexpr int LW_MAX_K = 4096;
 constexpr int RADIX_BITS = 11;
 constexpr int RADIX_BINS = 1 << RADIX_BITS;
@@ -61,6 +61,8 @@ struct LWParams {
   int64_t o_tab, o_acc, o_b, o_cu, o_ckey, o_ch, o_ccnt, o_cc, o_ceoff;
   int64_t tab_cap;  // entries
   uint32_t* gen;
+  int maxT;         // largest frontier (batch_size, max K)
+  int64_t o_flat;   // per flat edge: table slot of its row (-1: column invalid)
 };
 
 struct LWs {
@@ -73,6 +75,7 @@ struct LWs {
   int32_t* ccnt;
   float* cc;
   int32_t* ceoff;
+  int32_t* flat;   // [flat edge] table slot of the edge's row
 };
 
 __device__ __forceinline__ int lw_log2ceil(int64_t x) {
@@ -85,7 +88,27 @@ __device__ __forceinline__ unsigned long long dbits(double d) {
   return (unsigned long long)__double_as_longlong(d);
 }
 
+// Flat edge e of the frontier's columns -> column (binary search of the
+// column starts in shared memory).
+__device__ __forceinline__ int lw_col(const int32_t* fstart, int T, int64_t e) {
+  int lo = 0, hi = T - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (fstart[mid] <= e) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+constexpr int LW_ILP = 4;  // flat edges per thread in flight
+
 __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
+  extern __shared__ __align__(16) unsigned char lw_dyn[];
+  // per frontier column (T <= P.maxT): flat start, indptr, kept count, sum of a
+  int32_t* s_fstart = (int32_t*)lw_dyn;
+  int64_t* s_off = (int64_t*)(lw_dyn + (((size_t)(P.maxT + 1) * 4 + 7) & ~(size_t)7));
+  int32_t* s_cnt = (int32_t*)(s_off + P.maxT);
+  double* s_cs = (double*)(s_cnt + P.maxT + (P.maxT & 1));
   __shared__ unsigned long long s_scan[33];
   __shared__ double s_dred[33];
   __shared__ int s_hist[RADIX_BINS];
@@ -104,6 +127,7 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
   W.ccnt = (int32_t*)(base + P.o_ccnt);
   W.cc = (float*)(base + P.o_cc);
   W.ceoff = (int32_t*)(base + P.o_ceoff);
+  W.flat = (int32_t*)(base + P.o_flat);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
   uint32_t gen = P.gen[blockIdx.x];
 
@@ -118,27 +142,45 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
       const int K = P.K[l];
       const int64_t rbase = b * (int64_t)K;
       const int64_t ibase = colbase + b;
-      // ---- size the table: sum of frontier degrees ----
-      double dsum_local = 0.0;
-      for (int64_t j = threadIdx.x; j < T; j += blockDim.x) {
-        const int32_t v = __ldcg(F + j);
-        if (v < 0 || (int64_t)v >= P.N) {
-          atomicOr(P.err, ERR_SEED_RANGE);
-          continue;
+      // ---- frontier: column starts in the flat edge order, table size ----
+      {
+        int64_t run = 0;
+        for (int64_t j0 = 0; j0 < T; j0 += blockDim.x) {
+          const int64_t j = j0 + threadIdx.x;
+          int64_t d = 0, off = 0;
+          if (j < T) {
+            const int32_t v = __ldcg(F + j);
+            if (v < 0 || (int64_t)v >= P.N) {
+              atomicOr(P.err, ERR_SEED_RANGE);
+            } else {
+              off = __ldg(P.indptr + v);
+              d = __ldg(P.indptr + v + 1) - off;
+            }
+          }
+          unsigned long long tot;
+          const unsigned long long ex = block_exclusive_scan((unsigned long long)d, s_scan, &tot);
+          if (j < T) {
+            s_fstart[j] = (int32_t)(run + (int64_t)ex);
+            s_off[j] = off;
+          }
+          run += (int64_t)tot;
         }
-        dsum_local += (double)(__ldg(P.indptr + v + 1) - __ldg(P.indptr + v));
+        if (threadIdx.x == 0) s_fstart[T] = (int32_t)run;
+        s_u64[1] = (unsigned long long)run;
       }
-      const double dsum = block_reduce_sum(dsum_local, s_dred);
-      const int log_cap = lw_log2ceil((int64_t)(dsum * 4.0 / 3.0) + 64);
+      __syncthreads();
+      const int64_t dsum = (int64_t)s_u64[1];
+      const int log_cap = lw_log2ceil((dsum * 4) / 3 + 64);
       const int64_t cap = 1ll << log_cap;
-      if (cap > P.tab_cap) {
+      if (cap > P.tab_cap || dsum > P.tab_cap) {
         // does not fit this CTA's workspace: report the size, emit an empty layer
         if (threadIdx.x == 0) {
           atomicOr(P.err, ERR_CAPACITY);
-          atomicMax(P.need_tab, (unsigned long long)cap);
+          atomicMax(P.need_tab, (unsigned long long)(cap > dsum ? cap : dsum));
         }
         T = 0;
       }
+      const int Ti = (int)T;
       if (gen == 255u) {
         for (int64_t i = threadIdx.x; i < P.tab_cap; i += blockDim.x) W.tab[i] = 0ull;
       }
@@ -147,67 +189,93 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
         for (int64_t i = threadIdx.x; i < cap && T > 0; i += blockDim.x) W.acc[i] = 0.0;
       __syncthreads();
 
-      // ---- L1: Extract + bias accumulation ----
-      for (int64_t j = warp; j < T; j += nwarps) {
-        const int32_t v = __ldcg(F + j);
-        if (v < 0 || (int64_t)v >= P.N) continue;
-        const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
-        for (int64_t i = lane; i < d; i += 32) {
-          const uint32_t u = (uint32_t)__ldg(P.indices + off + i);
-          bool ins;
-          const uint32_t h = tab_insert_once(W.tab, log_cap, gen, u, 0u, &ins);
-          if (P.mode == GS_PROB_LADIES) {
-            const float w = P.weights ? __ldg(P.weights + off + i) : 1.0f;
-            atomicAdd(W.acc + h, (double)__fmul_rn(w, w));
-          } else if (P.mode == GS_PROB_COUNT) {
-            atomicAdd(W.acc + h, 1.0);
+      // ---- L1: Extract + bias accumulation over the flat edges of A[:, F]
+      // (LW_ILP rows in flight per thread); a row's first insert appends it
+      // to the candidate list C ----
+      if (threadIdx.x == 0) s_misc[4] = 0;
+      __syncthreads();
+      const int64_t nflat = T > 0 ? dsum : 0;
+      for (int64_t e0 = (int64_t)threadIdx.x - lane; e0 < nflat; e0 += (int64_t)blockDim.x * LW_ILP) {
+        uint32_t u[LW_ILP];
+        float w[LW_ILP];
+        bool ok[LW_ILP];
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          const int64_t e = e0 + (int64_t)q * blockDim.x + lane;
+          ok[q] = e < nflat;
+          u[q] = 0;
+          w[q] = 1.0f;
+          if (ok[q]) {
+            const int c = lw_col(s_fstart, Ti, e);
+            const int64_t pos = s_off[c] + (e - s_fstart[c]);
+            u[q] = (uint32_t)__ldg(P.indices + pos);
+            if (P.mode == GS_PROB_LADIES && P.weights) w[q] = __ldg(P.weights + pos);
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          const int64_t e = e0 + (int64_t)q * blockDim.x + lane;
+          bool ins = false;
+          uint32_t h = 0;
+          if (ok[q]) {
+            h = tab_insert_once(W.tab, log_cap, gen, u[q], 0u, &ins);
+            W.flat[e] = (int32_t)h;
+            if (P.mode == GS_PROB_LADIES) atomicAdd(W.acc + h, (double)__fmul_rn(w[q], w[q]));
+            else if (P.mode == GS_PROB_COUNT) atomicAdd(W.acc + h, 1.0);
+          }
+          const uint32_t m = __ballot_sync(0xffffffffu, ins);
+          if (m) {
+            int slot0 = 0;
+            if (lane == 0) slot0 = atomicAdd(&s_misc[4], __popc(m));
+            slot0 = __shfl_sync(0xffffffffu, slot0, 0);
+            if (ins) {
+              const int slot = slot0 + __popc(m & ((1u << lane) - 1u));
+              W.cu[slot] = (int32_t)u[q];
+              W.ch[slot] = (int32_t)h;
+            }
           }
         }
       }
       __syncthreads();
+      const int64_t ncand = T > 0 ? s_misc[4] : 0;
 
-      // ---- L2: candidates, bias, B, A-Res keys ----
-      unsigned long long carry = 0;
+      // ---- L2: bias, B, A-Res keys of the candidates (b <= 0: ineligible,
+      // key +inf, never selected) ----
       double bsum_local = 0.0;
-      for (int64_t ht = 0; ht < cap && T > 0; ht += blockDim.x) {
-        const int64_t h = ht + threadIdx.x;
-        bool elig = false;
-        uint32_t u = 0;
-        float bias = 0.f;
-        if (h < cap) {
-          const unsigned long long e = __ldcg(W.tab + h);
-          if (tab_gen(e) == gen) {
-            u = tab_key(e);
-            if (P.mode == GS_PROB_DEGREE) bias = (float)(__ldg(P.indptr + u + 1) - __ldg(P.indptr + u));
-            else bias = (float)__ldcg(W.acc + h);
-            W.b[h] = bias;
-            bsum_local += (double)bias;
-            elig = bias > 0.0f;
-          }
-        }
-        unsigned long long tot;
-        const unsigned long long ex = block_exclusive_scan((unsigned long long)(elig ? 1 : 0), s_scan, &tot) + carry;
-        if (elig) {
+      int elig_local = 0;
+      for (int64_t i = threadIdx.x; i < ncand; i += blockDim.x) {
+        const uint32_t u = (uint32_t)__ldcg(W.cu + i);
+        const int32_t h = __ldcg(W.ch + i);
+        float bias;
+        if (P.mode == GS_PROB_DEGREE) bias = (float)(__ldg(P.indptr + u + 1) - __ldg(P.indptr + u));
+        else bias = (float)__ldcg(W.acc + h);
+        W.b[h] = bias;
+        bsum_local += (double)bias;
+        double kk = INFINITY;
+        if (bias > 0.0f) {
           const U4 r = philox(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.key);
-          W.cu[ex] = (int32_t)u;
-          W.ckey[ex] = ares_key(r.x, (double)bias);
-          W.ch[ex] = (int32_t)h;
+          kk = ares_key(r.x, (double)bias);
+          ++elig_local;
         }
-        carry += tot;
+        W.ckey[i] = kk;
       }
-      const int64_t nc = (int64_t)carry;
       const double Btot = block_reduce_sum(bsum_local, s_dred);
       const float B32 = (float)Btot;
+      const int64_t nelig = (int64_t)block_reduce_sum((double)elig_local, s_dred);
+      const int64_t nc = ncand;
       __syncthreads();
 
       // ---- L3: select the K smallest (key, u) ----
       if (threadIdx.x == 0) s_misc[0] = 0;
       __syncthreads();
       int nsel;
-      if (nc <= K) {
-        for (int64_t i = threadIdx.x; i < nc; i += blockDim.x)
-          s_sel[i] = ((unsigned long long)(uint32_t)__ldcg(W.cu + i) << 32) | (uint32_t)__ldcg(W.ch + i);
-        nsel = (int)nc;
+      if (nelig <= K) {  // every eligible candidate (R24)
+        for (int64_t i = threadIdx.x; i < nc; i += blockDim.x) {
+          if (!(__ldcg(W.ckey + i) < INFINITY)) continue;
+          const int slot = atomicAdd(&s_misc[0], 1);
+          s_sel[slot] = ((unsigned long long)(uint32_t)__ldcg(W.cu + i) << 32) | (uint32_t)__ldcg(W.ch + i);
+        }
+        nsel = (int)nelig;
       } else {
         unsigned long long prefix = 0, pmask = 0;
         int remaining = K;
@@ -316,80 +384,96 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
       }
       __syncthreads();
 
-      // ---- L5a: per column count and c_j = sum a over kept edges ----
-      for (int64_t j = warp; j < T; j += nwarps) {
-        const int32_t v = __ldcg(F + j);
-        int cnt = 0;
-        double cs = 0.0;
-        if (v >= 0 && (int64_t)v < P.N) {
-          const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
-          for (int64_t i = lane; i < d; i += 32) {
-            const uint32_t u = (uint32_t)__ldg(P.indices + off + i);
-            const int64_t h = tab_find(W.tab, log_cap, gen, u);
-            const uint32_t val = tab_val(__ldcg(W.tab + h));
-            if (val) {
-              const float w = P.weights ? __ldg(P.weights + off + i) : 1.0f;
-              const float a = __fdiv_rn(w, __ldcg(W.b + h));
-              ++cnt;
-              cs += (double)a;
-            }
+      // ---- L5a: per column kept count and c_j = sum_fp64 a over its kept
+      // edges (flat edges, slots staged by L1: no second hash probe) ----
+      for (int j = threadIdx.x; j < Ti; j += blockDim.x) {
+        s_cnt[j] = 0;
+        s_cs[j] = 0.0;
+      }
+      __syncthreads();
+      for (int64_t e0 = threadIdx.x; e0 < nflat; e0 += (int64_t)blockDim.x * LW_ILP) {
+        int32_t h[LW_ILP];
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          const int64_t e = e0 + (int64_t)q * blockDim.x;
+          h[q] = e < nflat ? __ldcg(W.flat + e) : -1;
+        }
+        uint32_t val[LW_ILP];
+        float pb[LW_ILP], w[LW_ILP];
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          val[q] = h[q] >= 0 ? tab_val(__ldcg(W.tab + h[q])) : 0u;
+          pb[q] = val[q] ? __ldcg(W.b + h[q]) : 1.0f;
+          w[q] = 1.0f;
+          const int64_t e = e0 + (int64_t)q * blockDim.x;
+          if (val[q] && P.weights) {
+            const int c = lw_col(s_fstart, Ti, e);
+            w[q] = __ldg(P.weights + s_off[c] + (e - s_fstart[c]));
           }
         }
-        cnt = __reduce_add_sync(0xffffffffu, (unsigned)cnt);
-        for (int o = 16; o > 0; o >>= 1) cs += __shfl_xor_sync(0xffffffffu, cs, o);
-        if (lane == 0) {
-          W.ccnt[j] = cnt;
-          W.cc[j] = (float)cs;
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          if (!val[q]) continue;
+          const int64_t e = e0 + (int64_t)q * blockDim.x;
+          const int c = lw_col(s_fstart, Ti, e);
+          atomicAdd(&s_cnt[c], 1);
+          atomicAdd(&s_cs[c], (double)__fdiv_rn(w[q], pb[q]));
         }
       }
       __syncthreads();
-      carry = 0;
-      for (int64_t jt = 0; jt < T; jt += blockDim.x) {
-        const int64_t j = jt + threadIdx.x;
-        const unsigned long long cv = j < T ? (unsigned long long)__ldcg(W.ccnt + j) : 0ull;
+      int64_t E = 0;
+      for (int j0 = 0; j0 < Ti; j0 += blockDim.x) {
+        const int j = j0 + threadIdx.x;
+        const unsigned long long cv = j < Ti ? (unsigned long long)s_cnt[j] : 0ull;
         unsigned long long tot;
-        const unsigned long long ex = block_exclusive_scan(cv, s_scan, &tot) + carry;
-        if (j < T) W.ceoff[j] = (int32_t)ex;
-        carry += tot;
+        const unsigned long long ex = block_exclusive_scan(cv, s_scan, &tot);
+        if (j < Ti) W.ceoff[j] = (int32_t)(E + (int64_t)ex);
+        E += (int64_t)tot;
       }
-      const int64_t E = (int64_t)carry;
       if (threadIdx.x == 0) s_u64[0] = atomicAdd(P.edge_ctr + l, (unsigned long long)E);
       __syncthreads();
       const int64_t ebase = (int64_t)s_u64[0];
       const bool fits = ebase + E <= P.edge_cap[l];
       if (!fits && threadIdx.x == 0) atomicOr(P.err, ERR_CAPACITY);
+      for (int64_t j = threadIdx.x; j < T; j += blockDim.x) {
+        P.indptr_out[l][ibase + j] = __ldcg(W.ceoff + j);
+        if (l == 0) P.col0[bstart + j] = __ldcg(F + j);
+      }
 
-      // ---- L5b: emit the block in CSC order ----
-      for (int64_t j = warp; j < T; j += nwarps) {
-        const int32_t v = __ldcg(F + j);
-        int64_t e = __ldcg(W.ceoff + j);
-        if (lane == 0) {
-          P.indptr_out[l][ibase + j] = e;
-          if (l == 0) P.col0[bstart + j] = v;
+      // ---- L5b: emit the block in CSC order: the flat order is column-major
+      // with ascending positions, so an exclusive scan of the keep flags over
+      // the flat edges is each kept edge's output index ----
+      int64_t krun = 0;
+      for (int64_t e0 = 0; e0 < nflat && fits; e0 += (int64_t)blockDim.x * LW_ILP) {
+        // thread t owns flat edges e0 + t*LW_ILP .. + LW_ILP-1 (contiguous)
+        const int64_t eb = e0 + (int64_t)threadIdx.x * LW_ILP;
+        int32_t h[LW_ILP];
+        uint32_t val[LW_ILP];
+        int kc = 0;
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) h[q] = eb + q < nflat ? __ldcg(W.flat + eb + q) : -1;
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          val[q] = h[q] >= 0 ? tab_val(__ldcg(W.tab + h[q])) : 0u;
+          kc += val[q] ? 1 : 0;
         }
-        if (!fits || v < 0 || (int64_t)v >= P.N) continue;
-        const float cj = __ldcg(W.cc + j);
-        const int64_t off = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - off;
-        for (int64_t i0 = 0; i0 < d; i0 += 32) {
-          const int64_t i = i0 + lane;
-          uint32_t val = 0;
-          int64_t h = 0;
-          if (i < d) {
-            const uint32_t u = (uint32_t)__ldg(P.indices + off + i);
-            h = tab_find(W.tab, log_cap, gen, u);
-            val = tab_val(__ldcg(W.tab + h));
-          }
-          const uint32_t m = __ballot_sync(0xffffffffu, val != 0u);
-          if (val) {
-            const int64_t o = ebase + e + __popc(m & ((1u << lane) - 1u));
-            const float w = P.weights ? __ldg(P.weights + off + i) : 1.0f;
-            const float a = __fdiv_rn(w, __ldcg(W.b + h));
-            P.row_local[l][o] = (int32_t)(val - 1u);
-            P.eid[l][o] = off + i;
-            P.val[l][o] = __fdiv_rn(a, cj);
-          }
-          e += __popc(m);
+        unsigned long long tot;
+        const unsigned long long ex = block_exclusive_scan((unsigned long long)kc, s_scan, &tot);
+        int64_t o = ebase + krun + (int64_t)ex;
+#pragma unroll
+        for (int q = 0; q < LW_ILP; ++q) {
+          if (!val[q]) continue;
+          const int64_t e = eb + q;
+          const int c = lw_col(s_fstart, Ti, e);
+          const int64_t pos = s_off[c] + (e - s_fstart[c]);
+          const float w = P.weights ? __ldg(P.weights + pos) : 1.0f;
+          const float a = __fdiv_rn(w, __ldcg(W.b + h[q]));
+          P.row_local[l][o] = (int32_t)(val[q] - 1u);
+          P.eid[l][o] = pos;
+          P.val[l][o] = __fdiv_rn(a, (float)s_cs[c]);
+          ++o;
         }
+        krun += (int64_t)tot;
       }
       if (threadIdx.x == 0) {
         P.indptr_out[l][ibase + T] = E;
@@ -463,8 +547,13 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  P.maxT = (int)std::max<int64_t>(batch_size, maxK);
+  const size_t dyn = (((size_t)(P.maxT + 1) * 4 + 7) & ~(size_t)7) + (size_t)P.maxT * 8 +
+                     (size_t)(P.maxT + (P.maxT & 1)) * 4 + (size_t)P.maxT * 8;
+  GS_CUDA_TRY(cudaFuncSetAttribute(layerwise_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)dyn));
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, layerwise_kernel, LW_THREADS, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, layerwise_kernel, LW_THREADS, dyn);
   per_sm = std::max(1, per_sm);
   const int nctas = (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, (int64_t)sms * per_sm));
   int64_t tab_cap = std::max<int64_t>(int64_t(1) << 15, blk->lw_tab_hint);
@@ -481,6 +570,7 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
   P.o_ccnt = o; o = align256(o + col_cap * 4);
   P.o_cc = o; o = align256(o + col_cap * 4);
   P.o_ceoff = o; o = align256(o + col_cap * 4);
+  P.o_flat = o; o = align256(o + tab_cap * 4);
   P.ws_stride = o;
   P.tab_cap = tab_cap;
   const size_t ws_bytes = (size_t)o * nctas;
@@ -525,7 +615,7 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
-  layerwise_kernel<<<nctas, LW_THREADS, 0, stream>>>(P);
+  layerwise_kernel<<<nctas, LW_THREADS, dyn, stream>>>(P);
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
