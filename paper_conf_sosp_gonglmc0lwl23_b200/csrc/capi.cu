@@ -280,6 +280,7 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_indices.reset(g->al, s);
   g->b_weights.reset(g->al, s);
   g->b_colsum.reset(g->al, s);
+  g->b_deg.reset(g->al, s);
   g->b_err.reset(g->al, s);
   delete g;
 }

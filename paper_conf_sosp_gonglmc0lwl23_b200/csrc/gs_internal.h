@@ -58,7 +58,8 @@ struct gs_graph {
   int sorted = 0;
   int64_t max_in_degree = 0;
   gsb::Allocator al;
-  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_err;
+  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_err, b_deg;
+  int32_t* deg = nullptr;    // FastGCN a0 pre-processing: in-degree per node (built on first use)
   int* d_err = nullptr;  // walk error word
 };
 
@@ -80,7 +81,7 @@ struct gs_blocks {
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch
   unsigned int launch_id = 0;  // per-call tag for device-side flags
-  int ws_kind_prev = 0;        // 1 node-wise (tables cleared to ~0), 2 layer-wise (cleared to 0)
+  int ws_kind_prev = 0;        // workspace layout tag of the previous launch (per kernel family)
   int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;

@@ -22,6 +22,8 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 #include "common.cuh"
 #include "gs_internal.h"
@@ -492,9 +494,48 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
 
 static int64_t align256(int64_t x) { return (x + 255) & ~int64_t(255); }
 
+gs_status run_layerwise_old(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
+                            int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
+size_t layerwise_bm_smem(int64_t N, int maxT, int* gw_log_out, int* ng_out, int64_t* n4_out);
+gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                           int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
+                           int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk,
+                           size_t smem, int gw_log, int ng, int64_t n4);
+
+// Chooses the kernel.  FastGCN (DEGREE): the bitmap kernel (layerwise_bm.cu)
+// when the candidate bitmaps of one CTA per SM fit (N/8 bytes each, <= 2 GB
+// in all) and its rank prefixes fit shared memory -- hub-biased frontiers give
+// ~280 k candidates per batch-layer (measured on LJ: 282 ms vs 514 ms).
+// LADIES / COUNT (~10 k candidates): the hash-table kernel below (31 ms vs
+// 69 ms: four dense bitmap scans per batch-layer cost more than the table).
+// GS_LW_PATH=old|bm forces one (experiments / tests).
 gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  {
+    int maxK = 1;
+    for (int l = 0; l < L; ++l) maxK = std::max(maxK, n_per_layer[l]);
+    const int maxT = (int)std::max<int64_t>(batch_size, maxK);
+    int gw_log = 0, ng = 0;
+    int64_t n4 = 0;
+    const size_t smem = layerwise_bm_smem(g->num_nodes, maxT, &gw_log, &ng, &n4);
+    const char* path = getenv("GS_LW_PATH");
+    bool bm = prob_mode == GS_PROB_DEGREE && smem > 0 && n4 * 16 * 148 <= (int64_t(2) << 30) &&
+              maxK <= 4096;
+    if (path && !strcmp(path, "old")) bm = false;
+    if (path && !strcmp(path, "bm") && smem > 0) bm = true;
+    if (bm)
+      return run_layerwise_bm(g, seeds, num_seeds, batch_size, batch_base, n_per_layer, L, prob_mode,
+                              key, stream, blk, smem, gw_log, ng, n4);
+  }
+  return run_layerwise_old(g, seeds, num_seeds, batch_size, batch_base, n_per_layer, L, prob_mode,
+                           key, stream, blk);
+}
+
+gs_status run_layerwise_old(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
+                            int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
   const Allocator& al = blk->al;
   LWParams P = {};
   P.indptr = g->indptr;

@@ -1,0 +1,727 @@
+// layerwise_bm.cu -- layer-wise ECSF sampling (FastGCN / LADIES / COUNT) with
+// the candidate set C of a batch-layer held as an N-bit row bitmap.
+//
+// collective_sample with the compute/finalize of Fig. 3(b)
+// (P:207-229), Table 2 and the FastGCN degree pre-processing
+// (P:300).  Same results as layerwise.cu (R7, R9, R24); what
+// differs is where the per-batch state lives.  layerwise.cu keys a hash table
+// by row and stages a table slot per streamed edge: for FastGCN's hub-biased
+// frontiers (~365 k edges, ~280 k candidates per batch-layer) that is ~11 MB
+// of random-access state per CTA, so 148 CTAs thrash L2 and every probe is a
+// 128-byte HBM line (profiles/r01_random_access_probe.md).  Here one persistent
+// 1024-thread CTA per SM owns one mini-batch at a time and keeps:
+//   * C as an N-bit bitmap in global memory (N/8 bytes per CTA: 0.6 MB for
+//     the LJ-shaped graph, L2-resident), set by fire-and-forget red.or;
+//   * a rank prefix per group of GW bitmap words in shared memory, so the rank
+//     of a candidate (its index in ascending-id order) is one smem load plus
+//     the popcounts of <= GW-1 words;
+//   * b(u) for LADIES / COUNT in a rank-indexed fp64 array (|C| entries);
+//   * the A-Res candidates, S and a hash of S in shared memory.
+// Per batch-layer:
+//   L1 Extract: stream A[:, F] (flat edges, ILP 4), set the rows' bits;
+//   L2 ranks: warp-contiguous scan of the bitmap -> group prefixes (+ FastGCN:
+//      b(u) = in-degree from the a0 degree array, B = sum b, eligible count);
+//   L3 (LADIES / COUNT) Compute: stream A[:, F] again, b(rank(u)) += w*w / 1
+//      (fp64 atomics, the edge-map + row reduce of Fig. 3(b) lines 2-3);
+//   L4 Select: every eligible candidate if <= K, else the K smallest A-Res
+//      keys E_u / b(u): a threshold tau = 2K/B keeps ~2K candidates (cheap
+//      float pre-test, exact fp64 key only for survivors) in shared memory,
+//      which are sorted by (key, u); S sorted by u; p(u) = b(u)/B;
+//   L5 Finalize: stream A[:, F], keep rows in S (smem hash), per column count
+//      and c_j = sum_fp64 a_e (a_e = w_e / p(u)), then emit the block in CSC
+//      order with val_e = a_e / c_j (flat keep-scan).
+// The bitmap and b(u) are cleared by the CTA after the select.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "gs_internal.h"
+#include "nodewise_common.cuh"
+
+namespace gsb {
+
+constexpr int LB_THREADS = 1024;
+constexpr int LB_WARPS = LB_THREADS / 32;
+constexpr int LB_CAP = 4096;        // A-Res candidate buffer (select), >= max K
+constexpr int LB_HS = 8192;         // hash of S (aliases the candidate buffer)
+constexpr int LB_ILP = 4;           // flat edges per thread in flight
+constexpr int LB_MAX_K = 4096;
+
+struct LBParams {
+  const int64_t* indptr;
+  const int32_t* indices;
+  const float* weights;
+  const int32_t* deg;               // a0: in-degree per node (FastGCN)
+  int64_t N;
+  const int32_t* seeds;
+  int64_t num_seeds, batch_size, num_batches, batch_base;
+  int L;
+  int K[MAX_LAYERS];
+  int mode;
+  uint64_t key;
+  int32_t* col0;
+  int32_t* row_map[MAX_LAYERS];
+  float* row_prob[MAX_LAYERS];
+  int64_t* indptr_out[MAX_LAYERS];
+  int32_t* row_local[MAX_LAYERS];
+  int64_t* eid[MAX_LAYERS];
+  float* val[MAX_LAYERS];
+  int64_t edge_cap[MAX_LAYERS];
+  unsigned long long* edge_ctr;     // [MAX_LAYERS] bump allocators of the edge ranges
+  unsigned long long* need_tab;     // largest |C| a batch-layer needed (LADIES / COUNT)
+  int64_t* meta;
+  int* err;
+  uint32_t* bm;                     // [CTA][n4 * 4] row bitmaps (zero between batch-layers)
+  int64_t n4;                       // uint4 per bitmap (a multiple of GW / 4)
+  double* acc;                      // [CTA][acc_cap] b(u) by rank (zero between uses)
+  int64_t acc_cap;
+  int gw_log;                       // log2 words per rank group (>= 2)
+  int ng;                           // rank groups per bitmap
+  int maxT;
+};
+
+struct LBShared {
+  unsigned long long scan[33];
+  double dred[33];
+  int misc[8];
+  unsigned long long u64[4];
+  int wtot[LB_WARPS];
+};
+
+__device__ __forceinline__ int lb_col(const int32_t* fstart, int T, int64_t e) {
+  int lo = 0, hi = T - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (fstart[mid] <= e) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int popc4(const uint4& x) {
+  return __popc(x.x) + __popc(x.y) + __popc(x.z) + __popc(x.w);
+}
+
+__device__ __forceinline__ uint32_t word4(const uint4& x, int j) {
+  return j == 0 ? x.x : (j == 1 ? x.y : (j == 2 ? x.z : x.w));
+}
+
+// Rank of row u in the batch-layer's candidate set (ascending ids).
+__device__ __forceinline__ int64_t lb_rank(const LBParams& P, const uint32_t* bm, const int32_t* s_gp,
+                                           uint32_t u) {
+  const int64_t wi = u >> 5;
+  const int64_t g = wi >> P.gw_log;
+  int64_t r = s_gp[g];
+  for (int64_t k = g << P.gw_log; k < wi; ++k) r += __popc(__ldcg(bm + k));
+  return r + __popc(__ldcg(bm + wi) & ((1u << (u & 31)) - 1u));
+}
+
+// Walks the set bits of the bitmap in warp-contiguous ranges of rank groups:
+// f(u, rank) for every candidate.  Ranks come from s_gp (built by lb_ranks).
+template <class Fn>
+__device__ __forceinline__ void lb_for_bits(const LBParams& P, const uint4* bm4, const int32_t* s_gp,
+                                            Fn f) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int gq = 1 << (P.gw_log - 2);            // uint4 per group
+  const int gpw = (P.ng + LB_WARPS - 1) / LB_WARPS;
+  const int64_t i_beg = (int64_t)min(warp * gpw, P.ng) * gq;
+  const int64_t i_end = (int64_t)min((warp + 1) * gpw, P.ng) * gq;
+  for (int64_t i0 = i_beg; i0 < i_end; i0 += 32) {
+    const int64_t i = i0 + lane;
+    const uint4 x = i < i_end ? __ldcg(bm4 + i) : make_uint4(0, 0, 0, 0);
+    const int pc = popc4(x);
+    const int inc = warp_inclusive_scan(pc);
+    const int first = lane - (lane & (gq - 1));  // first lane of this lane's group
+    const int ex_first = __shfl_sync(0xffffffffu, inc, first) - __shfl_sync(0xffffffffu, pc, first);
+    if (pc == 0) continue;
+    int64_t r = (int64_t)s_gp[i >> (P.gw_log - 2)] + (inc - pc - ex_first);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      uint32_t w = word4(x, j);
+      while (w) {
+        const int bpos = __ffs(w) - 1;
+        w &= w - 1u;
+        f((uint32_t)((i * 4 + j) * 32 + bpos), r);
+        ++r;
+      }
+    }
+  }
+}
+
+// s_gp[g] = number of candidates before rank group g; returns |C|.  FastGCN:
+// also b(u) = deg(u) summed (B, fp64) and the eligible count.
+__device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, int32_t* s_gp,
+                            bool degree, double* B_out, int64_t* nelig_out) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int gq = 1 << (P.gw_log - 2);
+  const int gpw = (P.ng + LB_WARPS - 1) / LB_WARPS;
+  const int g_beg = min(warp * gpw, P.ng), g_end = min((warp + 1) * gpw, P.ng);
+  const int64_t i_beg = (int64_t)g_beg * gq, i_end = (int64_t)g_end * gq;
+  int run = 0;
+  double bsum = 0.0;
+  int elig = 0;
+  for (int64_t i0 = i_beg; i0 < i_end; i0 += 32) {
+    const int64_t i = i0 + lane;
+    const uint4 x = i < i_end ? __ldcg(bm4 + i) : make_uint4(0, 0, 0, 0);
+    const int pc = popc4(x);
+    const int inc = warp_inclusive_scan(pc);
+    if (i < i_end && (lane & (gq - 1)) == 0) s_gp[i >> (P.gw_log - 2)] = run + inc - pc;
+    run += __shfl_sync(0xffffffffu, inc, 31);
+    if (degree && pc) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        uint32_t w = word4(x, j);
+        while (w) {
+          const int bpos = __ffs(w) - 1;
+          w &= w - 1u;
+          const int32_t dg = __ldg(P.deg + (i * 4 + j) * 32 + bpos);
+          bsum += (double)(float)dg;
+          elig += dg > 0 ? 1 : 0;
+        }
+      }
+    }
+  }
+  if (lane == 0) sh.wtot[warp] = run;
+  __syncthreads();
+  if (warp == 0) {
+    const int v = sh.wtot[lane];
+    const int inc = warp_inclusive_scan(v);
+    sh.wtot[lane] = inc - v;
+    if (lane == 31) sh.misc[5] = inc;
+  }
+  __syncthreads();
+  const int off = sh.wtot[warp];
+  for (int g = g_beg + lane; g < g_end; g += 32) s_gp[g] += off;
+  if (warp == 0 && lane == 0) s_gp[P.ng] = sh.misc[5];
+  const int64_t total = sh.misc[5];
+  if (degree) {
+    *B_out = block_reduce_sum(bsum, sh.dred);
+    *nelig_out = (int64_t)block_reduce_sum((double)elig, sh.dred);
+  } else {
+    __syncthreads();
+  }
+  return total;
+}
+
+// Bitonic sort of n2 (power of two) 64-bit keys with a 32-bit payload,
+// ascending by (key, payload).
+__device__ void lb_sort_kv(unsigned long long* k, uint32_t* v, float* b, int n2) {
+  for (int kk = 2; kk <= n2; kk <<= 1) {
+    for (int jj = kk >> 1; jj > 0; jj >>= 1) {
+      for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+        const int ixj = i ^ jj;
+        if (ixj > i) {
+          const unsigned long long ka = k[i], kc = k[ixj];
+          const uint32_t va = v[i], vc = v[ixj];
+          const bool gt = ka > kc || (ka == kc && va > vc);
+          if (gt == ((i & kk) == 0)) {
+            k[i] = kc; k[ixj] = ka;
+            v[i] = vc; v[ixj] = va;
+            if (b) { const float t = b[i]; b[i] = b[ixj]; b[ixj] = t; }
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+__device__ __forceinline__ uint32_t lb_hash(uint32_t u) { return (u * 0x9E3779B1u) >> 19; }  // 13 bits
+
+__device__ __forceinline__ int lb_lookup(const int32_t* hk, const int32_t* hv, uint32_t u) {
+  uint32_t h = lb_hash(u);
+  while (true) {
+    const int32_t k = hk[h];
+    if (k == (int32_t)u) return hv[h];
+    if (k < 0) return -1;
+    h = (h + 1) & (LB_HS - 1);
+  }
+}
+
+__global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P) {
+  extern __shared__ __align__(16) unsigned char lb_dyn[];
+  __shared__ LBShared sh;
+  // dynamic smem: candidate buffer (keys, ids, biases; later the hash of S),
+  // S, per-column arrays, rank-group prefixes
+  unsigned long long* s_bk = (unsigned long long*)lb_dyn;            // [LB_CAP]
+  uint32_t* s_bu = (uint32_t*)(s_bk + LB_CAP);                       // [LB_CAP]
+  float* s_bb = (float*)(s_bu + LB_CAP);                             // [LB_CAP]
+  int32_t* s_hk = (int32_t*)lb_dyn;                                  // [LB_HS] (aliases)
+  int32_t* s_hv = s_hk + LB_HS;                                      // [LB_HS]
+  unsigned long long* s_sel = (unsigned long long*)(s_bb + LB_CAP);  // [LB_MAX_K] u<<32 | p
+  int64_t* s_off = (int64_t*)(s_sel + LB_MAX_K);                     // [maxT]
+  double* s_cs = (double*)(s_off + P.maxT);                          // [maxT]
+  int32_t* s_fstart = (int32_t*)(s_cs + P.maxT);                     // [maxT + 1]
+  int32_t* s_cnt = s_fstart + P.maxT + 1;                            // [maxT]
+  int32_t* s_gp = s_cnt + P.maxT;                                    // [ng + 1]
+
+  const int lane = threadIdx.x & 31;
+  uint32_t* bm = P.bm + (int64_t)blockIdx.x * P.n4 * 4;
+  const uint4* bm4 = (const uint4*)bm;
+  double* acc = P.acc ? P.acc + (int64_t)blockIdx.x * P.acc_cap : nullptr;
+  const bool degree = P.mode == GS_PROB_DEGREE;
+
+  for (int64_t b = blockIdx.x; b < P.num_batches; b += gridDim.x) {
+    const int64_t bstart = b * P.batch_size;
+    const int64_t nb = min(P.batch_size, P.num_seeds - bstart);
+    const uint32_t gb = (uint32_t)(P.batch_base + b);
+    const int32_t* F = P.seeds + bstart;
+    int64_t T = nb;
+    int64_t colbase = bstart;
+    for (int l = 0; l < P.L; ++l) {
+      const int K = P.K[l];
+      const int64_t rbase = b * (int64_t)K;
+      const int64_t ibase = colbase + b;
+      // ---- frontier: column starts in the flat edge order ----
+      {
+        int64_t run = 0;
+        for (int64_t j0 = 0; j0 < T; j0 += blockDim.x) {
+          const int64_t j = j0 + threadIdx.x;
+          int64_t d = 0, off = 0;
+          if (j < T) {
+            const int32_t v = __ldcg(F + j);
+            if (v < 0 || (int64_t)v >= P.N) {
+              atomicOr(P.err, ERR_SEED_RANGE);
+            } else {
+              off = __ldg(P.indptr + v);
+              d = __ldg(P.indptr + v + 1) - off;
+            }
+          }
+          unsigned long long tot;
+          const unsigned long long ex = block_exclusive_scan((unsigned long long)d, sh.scan, &tot);
+          if (j < T) {
+            s_fstart[j] = (int32_t)(run + (int64_t)ex);
+            s_off[j] = off;
+          }
+          run += (int64_t)tot;
+        }
+        if (threadIdx.x == 0) {
+          s_fstart[T] = (int32_t)run;
+          sh.u64[1] = (unsigned long long)run;
+        }
+      }
+      __syncthreads();
+      const int Ti = (int)T;
+      const int64_t nflat = T > 0 ? (int64_t)sh.u64[1] : 0;
+
+      // ---- L1: Extract, the rows' bits (one red.or per distinct row per warp round) ----
+      for (int64_t e0 = (int64_t)threadIdx.x - lane; e0 < nflat; e0 += (int64_t)blockDim.x * LB_ILP) {
+        uint32_t u[LB_ILP];
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          const int64_t e = e0 + (int64_t)q * blockDim.x + lane;
+          u[q] = 0xFFFFFFFFu;
+          if (e < nflat) {
+            const int c = lb_col(s_fstart, Ti, e);
+            u[q] = (uint32_t)__ldg(P.indices + s_off[c] + (e - s_fstart[c]));
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          const uint32_t peers = __match_any_sync(0xffffffffu, u[q]);
+          if (u[q] != 0xFFFFFFFFu && (__ffs(peers) - 1) == lane) atomicOr(bm + (u[q] >> 5), 1u << (u[q] & 31));
+        }
+      }
+      __syncthreads();
+
+      // ---- L2: rank groups (FastGCN: b(u) = in-degree, B, eligible) ----
+      double Btot = 0.0;
+      int64_t nelig = 0;
+      const int64_t nc = lb_ranks(P, sh, bm4, s_gp, degree, &Btot, &nelig);
+      bool acc_ok = true;
+      if (!degree && nc > P.acc_cap) {
+        if (threadIdx.x == 0) {
+          atomicOr(P.err, ERR_CAPACITY);
+          atomicMax(P.need_tab, (unsigned long long)nc);
+        }
+        acc_ok = false;
+      }
+
+      // ---- L3 (LADIES / COUNT): b(rank(u)) += fp32(w*w) / 1 in fp64 ----
+      if (!degree) {
+        if (acc_ok) {
+          for (int64_t e0 = threadIdx.x; e0 < nflat; e0 += (int64_t)blockDim.x * LB_ILP) {
+            uint32_t u[LB_ILP];
+            float w[LB_ILP];
+#pragma unroll
+            for (int q = 0; q < LB_ILP; ++q) {
+              const int64_t e = e0 + (int64_t)q * blockDim.x;
+              u[q] = 0xFFFFFFFFu;
+              w[q] = 1.0f;
+              if (e < nflat) {
+                const int c = lb_col(s_fstart, Ti, e);
+                const int64_t pos = s_off[c] + (e - s_fstart[c]);
+                u[q] = (uint32_t)__ldg(P.indices + pos);
+                if (P.mode == GS_PROB_LADIES && P.weights) w[q] = __ldg(P.weights + pos);
+              }
+            }
+#pragma unroll
+            for (int q = 0; q < LB_ILP; ++q) {
+              if (u[q] == 0xFFFFFFFFu) continue;
+              const int64_t r = lb_rank(P, bm, s_gp, u[q]);
+              atomicAdd(acc + r, P.mode == GS_PROB_LADIES ? (double)__fmul_rn(w[q], w[q]) : 1.0);
+            }
+          }
+        }
+        __syncthreads();
+        double bs = 0.0;
+        int el = 0;
+        for (int64_t r = threadIdx.x; r < nc && acc_ok; r += blockDim.x) {
+          const float bb = (float)__ldcg(acc + r);
+          bs += (double)bb;
+          el += bb > 0.0f ? 1 : 0;
+        }
+        Btot = block_reduce_sum(bs, sh.dred);
+        nelig = acc_ok ? (int64_t)block_reduce_sum((double)el, sh.dred) : 0;
+      }
+      const float B32 = (float)Btot;
+
+      // ---- L4: Select ----
+      auto bias_of = [&](uint32_t u, int64_t r) -> float {
+        return degree ? (float)__ldg(P.deg + u) : (float)__ldcg(acc + r);
+      };
+      if (threadIdx.x == 0) sh.misc[0] = 0;
+      __syncthreads();
+      int nsel = 0;
+      if (nelig <= K) {  // every eligible candidate (R24)
+        if (nelig > 0) {
+          lb_for_bits(P, bm4, s_gp, [&](uint32_t u, int64_t r) {
+            const float bb = bias_of(u, r);
+            if (bb > 0.0f) {
+              const int slot = atomicAdd(&sh.misc[0], 1);
+              s_bu[slot] = u;
+              s_bb[slot] = bb;
+            }
+          });
+        }
+        nsel = (int)nelig;
+        __syncthreads();
+      } else {
+        // threshold filter: keys below tau, ~2K of them (R6: exact fp64 key)
+        double tau = 2.0 * K / Btot, lo = 0.0, hi = 0.0;
+        int m = 0;
+        for (int it = 0; it < 64; ++it) {
+          if (threadIdx.x == 0) sh.misc[0] = 0;
+          __syncthreads();
+          lb_for_bits(P, bm4, s_gp, [&](uint32_t u, int64_t r) {
+            const float bb = bias_of(u, r);
+            if (!(bb > 0.0f)) return;
+            const U4 R = philox(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.key);
+            const float t = (float)(tau * (double)bb) * 1.01f;
+            if (!ares_maybe_below(R.x, t)) return;
+            const double kk = ares_key(R.x, (double)bb);
+            if (!(kk < tau)) return;
+            const int slot = atomicAdd(&sh.misc[0], 1);
+            if (slot < LB_CAP) {
+              s_bk[slot] = (unsigned long long)__double_as_longlong(kk);
+              s_bu[slot] = u;
+              s_bb[slot] = bb;
+            }
+          });
+          __syncthreads();
+          m = sh.misc[0];
+          __syncthreads();
+          if (m >= K && m <= LB_CAP) break;
+          if (m < K) lo = tau;
+          else hi = tau;
+          tau = (lo > 0.0 && hi > 0.0) ? sqrt(lo * hi) : (lo > 0.0 ? lo * 4.0 : hi * 0.25);
+          if (it == 63) {
+            if (threadIdx.x == 0) atomicOr(P.err, ERR_INTERNAL);
+            m = min(m, LB_CAP);
+          }
+        }
+        int n2 = 1;
+        while (n2 < m) n2 <<= 1;
+        for (int i = m + threadIdx.x; i < n2; i += blockDim.x) {
+          s_bk[i] = ~0ull;
+          s_bu[i] = 0xFFFFFFFFu;
+        }
+        __syncthreads();
+        lb_sort_kv(s_bk, s_bu, s_bb, n2);  // (key, u) ascending: the K smallest first
+        nsel = min(K, m);
+      }
+      // S sorted by node id (R3): (u << 32 | bias bits)
+      int n2 = 1;
+      while (n2 < nsel) n2 <<= 1;
+      for (int i = threadIdx.x; i < n2; i += blockDim.x)
+        s_sel[i] = i < nsel ? (((unsigned long long)s_bu[i] << 32) | __float_as_uint(s_bb[i])) : ~0ull;
+      __syncthreads();
+      for (int kk = 2; kk <= n2; kk <<= 1) {
+        for (int jj = kk >> 1; jj > 0; jj >>= 1) {
+          for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+            const int ixj = i ^ jj;
+            if (ixj > i) {
+              const unsigned long long a = s_sel[i], c = s_sel[ixj];
+              if ((a > c) == ((i & kk) == 0)) {
+                s_sel[i] = c;
+                s_sel[ixj] = a;
+              }
+            }
+          }
+          __syncthreads();
+        }
+      }
+      // p(u) = b(u) / B (R7); hash of S for the finalize
+      for (int i = threadIdx.x; i < LB_HS; i += blockDim.x) s_hk[i] = -1;
+      __syncthreads();
+      for (int i = threadIdx.x; i < nsel; i += blockDim.x) {
+        const uint32_t u = (uint32_t)(s_sel[i] >> 32);
+        const float p = __fdiv_rn(__uint_as_float((uint32_t)s_sel[i]), B32);
+        s_sel[i] = ((unsigned long long)u << 32) | __float_as_uint(p);
+        P.row_map[l][rbase + i] = (int32_t)u;
+        P.row_prob[l][rbase + i] = p;
+        uint32_t h = lb_hash(u);
+        while (atomicCAS(&s_hk[h], -1, (int32_t)u) != -1) h = (h + 1) & (LB_HS - 1);
+        s_hv[h] = i;
+      }
+      // clear C for the next batch-layer (bitmap, b(u))
+      for (int64_t i = threadIdx.x; i < P.n4; i += blockDim.x) ((uint4*)bm)[i] = make_uint4(0, 0, 0, 0);
+      if (!degree && acc_ok)
+        for (int64_t r = threadIdx.x; r < nc; r += blockDim.x) acc[r] = 0.0;
+      for (int j = threadIdx.x; j < Ti; j += blockDim.x) {
+        s_cnt[j] = 0;
+        s_cs[j] = 0.0;
+      }
+      __syncthreads();
+
+      // ---- L5a: per column kept count and c_j = sum_fp64 a (a = w / p(u)) ----
+      for (int64_t e0 = threadIdx.x; e0 < nflat && nsel > 0; e0 += (int64_t)blockDim.x * LB_ILP) {
+        uint32_t u[LB_ILP];
+        int c[LB_ILP];
+        int64_t pos[LB_ILP];
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          const int64_t e = e0 + (int64_t)q * blockDim.x;
+          u[q] = 0xFFFFFFFFu;
+          if (e < nflat) {
+            c[q] = lb_col(s_fstart, Ti, e);
+            pos[q] = s_off[c[q]] + (e - s_fstart[c[q]]);
+            u[q] = (uint32_t)__ldg(P.indices + pos[q]);
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          if (u[q] == 0xFFFFFFFFu) continue;
+          const int lid = lb_lookup(s_hk, s_hv, u[q]);
+          if (lid < 0) continue;
+          const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
+          const float p = __uint_as_float((uint32_t)s_sel[lid]);
+          atomicAdd(&s_cnt[c[q]], 1);
+          atomicAdd(&s_cs[c[q]], (double)__fdiv_rn(w, p));
+        }
+      }
+      __syncthreads();
+      int64_t E = 0;
+      for (int j0 = 0; j0 < Ti; j0 += blockDim.x) {
+        const int j = j0 + threadIdx.x;
+        const unsigned long long cv = j < Ti ? (unsigned long long)s_cnt[j] : 0ull;
+        unsigned long long tot;
+        const unsigned long long ex = block_exclusive_scan(cv, sh.scan, &tot);
+        if (j < Ti) P.indptr_out[l][ibase + j] = E + (int64_t)ex;
+        E += (int64_t)tot;
+      }
+      if (threadIdx.x == 0) sh.u64[0] = atomicAdd(P.edge_ctr + l, (unsigned long long)E);
+      for (int64_t j = threadIdx.x; j < T && l == 0; j += blockDim.x) P.col0[bstart + j] = __ldcg(F + j);
+      __syncthreads();
+      const int64_t ebase = (int64_t)sh.u64[0];
+      const bool fits = ebase + E <= P.edge_cap[l];
+      if (!fits && threadIdx.x == 0) atomicOr(P.err, ERR_CAPACITY);
+
+      // ---- L5b: emit in CSC order (flat order is column-major, positions
+      // ascending: an exclusive scan of the keep flags is the output index) ----
+      int64_t krun = 0;
+      for (int64_t e0 = 0; e0 < nflat && fits && E > 0; e0 += (int64_t)blockDim.x * LB_ILP) {
+        const int64_t eb = e0 + (int64_t)threadIdx.x * LB_ILP;
+        int lid[LB_ILP];
+        int c[LB_ILP];
+        int64_t pos[LB_ILP];
+        int kc = 0;
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          lid[q] = -1;
+          if (eb + q < nflat) {
+            c[q] = lb_col(s_fstart, Ti, eb + q);
+            pos[q] = s_off[c[q]] + (eb + q - s_fstart[c[q]]);
+            lid[q] = lb_lookup(s_hk, s_hv, (uint32_t)__ldg(P.indices + pos[q]));
+          }
+          kc += lid[q] >= 0 ? 1 : 0;
+        }
+        unsigned long long tot;
+        const unsigned long long ex = block_exclusive_scan((unsigned long long)kc, sh.scan, &tot);
+        int64_t o = ebase + krun + (int64_t)ex;
+#pragma unroll
+        for (int q = 0; q < LB_ILP; ++q) {
+          if (lid[q] < 0) continue;
+          const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
+          const float a = __fdiv_rn(w, __uint_as_float((uint32_t)s_sel[lid[q]]));
+          P.row_local[l][o] = lid[q];
+          P.eid[l][o] = pos[q];
+          P.val[l][o] = __fdiv_rn(a, (float)s_cs[c[q]]);
+          ++o;
+        }
+        krun += (int64_t)tot;
+      }
+      if (threadIdx.x == 0) {
+        P.indptr_out[l][ibase + T] = E;
+        long long* mt = (long long*)(P.meta + (b * P.L + l) * 8);
+        mt[0] = T; mt[1] = nsel; mt[2] = E; mt[3] = colbase; mt[4] = rbase; mt[5] = ibase;
+        mt[6] = ebase; mt[7] = 0;
+      }
+      __syncthreads();
+      F = P.row_map[l] + rbase;
+      colbase = rbase;
+      T = nsel;
+    }
+  }
+}
+
+// a0 pre-processing ("degree of each node in FastGCN"): deg[u] = in-degree.
+__global__ void degree_kernel(const int64_t* __restrict__ indptr, int64_t N, int32_t* __restrict__ deg) {
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < N; u += (int64_t)gridDim.x * blockDim.x)
+    deg[u] = (int32_t)(indptr[u + 1] - indptr[u]);
+}
+
+static int64_t a256(int64_t x) { return (x + 255) & ~int64_t(255); }
+
+// Shared-memory bytes of layerwise_bm_kernel for a graph of N nodes (0: does not fit).
+size_t layerwise_bm_smem(int64_t N, int maxT, int* gw_log_out, int* ng_out, int64_t* n4_out) {
+  const int64_t nwords = (N + 31) / 32;
+  int gw_log = 2;
+  while (((nwords >> gw_log) + 1) * 4 > 48 * 1024 && gw_log < 6) ++gw_log;
+  const int64_t gw = int64_t(1) << gw_log;
+  const int64_t ng = (nwords + gw - 1) / gw;
+  if ((ng + 1) * 4 > 48 * 1024) return 0;
+  const size_t s = (size_t)LB_CAP * (8 + 4 + 4) + (size_t)LB_MAX_K * 8 + (size_t)maxT * (8 + 8) +
+                   (size_t)(maxT + 1) * 4 + (size_t)maxT * 4 + (size_t)(ng + 1) * 4 + 16;
+  if (s + sizeof(LBShared) > 227 * 1024) return 0;
+  *gw_log_out = gw_log;
+  *ng_out = (int)ng;
+  *n4_out = ng * gw / 4;
+  return s;
+}
+
+gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                           int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
+                           int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk,
+                           size_t smem, int gw_log, int ng, int64_t n4) {
+  const Allocator& al = blk->al;
+  LBParams P = {};
+  P.indptr = g->indptr;
+  P.indices = g->indices;
+  P.weights = g->weights;
+  P.N = g->num_nodes;
+  P.seeds = seeds;
+  P.num_seeds = num_seeds;
+  P.batch_size = batch_size;
+  P.num_batches = (num_seeds + batch_size - 1) / batch_size;
+  P.batch_base = batch_base;
+  P.L = L;
+  P.mode = prob_mode;
+  P.key = key;
+  P.gw_log = gw_log;
+  P.ng = ng;
+  P.n4 = n4;
+  const int64_t nbatch = P.num_batches;
+  int maxK = 1;
+  for (int l = 0; l < L; ++l) {
+    P.K[l] = n_per_layer[l];
+    maxK = std::max(maxK, n_per_layer[l]);
+  }
+  P.maxT = (int)std::max<int64_t>(batch_size, maxK);
+  gs_graph* gm = const_cast<gs_graph*>(g);
+  if (prob_mode == GS_PROB_DEGREE && !gm->deg) {  // a0 pre-processing, once per graph
+    if (!gm->b_deg.ensure(gm->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
+      return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (degree array)");
+    gm->deg = (int32_t*)gm->b_deg.ptr;
+    const int64_t blocks = std::min<int64_t>((g->num_nodes + 255) / 256, 148 * 16);
+    if (g->num_nodes > 0) degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
+    GS_CUDA_TRY(cudaGetLastError());
+  }
+  P.deg = gm->deg;
+  blk->kind = gs_blocks::LAYERWISE;
+  blk->num_batches = nbatch;
+  blk->num_layers = L;
+  blk->stream = stream;
+  blk->synced = false;
+  auto need = [&](DevBuf& b, int64_t bytes) -> bool {
+    return b.ensure(al, (size_t)std::max<int64_t>(bytes, 256), stream);
+  };
+  bool ok = need(blk->b_col[0], num_seeds * 4);
+  int64_t edge_cap[MAX_LAYERS];
+  for (int l = 0; l < L && ok; ++l) {
+    const int64_t rows = nbatch * (int64_t)P.K[l];
+    const int64_t cols = l == 0 ? num_seeds : nbatch * (int64_t)P.K[l - 1];
+    int64_t ecap = std::max<int64_t>(int64_t(1) << 16, rows * 4);
+    ecap = std::max<int64_t>(ecap, blk->lw_edge_hint[l]);
+    ok = ok && need(blk->b_row[l], rows * 4) && need(blk->b_rprob[l], rows * 4) &&
+         need(blk->b_indptr[l], (cols + nbatch) * 8) && need(blk->b_rowl[l], ecap * 4) &&
+         need(blk->b_eid[l], ecap * 8) && need(blk->b_val[l], ecap * 4);
+    if (!ok) break;
+    edge_cap[l] = std::min<int64_t>({(int64_t)blk->b_rowl[l].bytes / 4, (int64_t)blk->b_eid[l].bytes / 8,
+                                     (int64_t)blk->b_val[l].bytes / 4});
+  }
+  ok = ok && need(blk->b_meta, nbatch * L * 8 * 8) && need(blk->b_err, 16) &&
+       need(blk->b_ctr, 8 * (MAX_LAYERS + 2));
+  if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (layer-wise blocks)");
+
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  GS_CUDA_TRY(cudaFuncSetAttribute(layerwise_bm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)smem));
+  const int nctas = (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, sms));
+  // per-CTA workspace: bitmap (kept zero), b(u) by rank (kept zero)
+  P.acc_cap = prob_mode == GS_PROB_DEGREE ? 0 : std::max<int64_t>(int64_t(1) << 15, blk->lw_tab_hint);
+  const int64_t bm_bytes = a256(n4 * 16);
+  const int64_t acc_bytes = a256(P.acc_cap * 8);
+  const int64_t stride = bm_bytes + acc_bytes;
+  const size_t ws_bytes = (size_t)stride * nctas;
+  const bool grow = blk->b_ws.bytes < ws_bytes;
+  if (!blk->b_ws.ensure(al, ws_bytes, stream))
+    return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (layer-wise workspace)");
+  if (grow || blk->ws_stride_prev != stride || blk->ws_kind_prev != 3)
+    GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, blk->b_ws.bytes, stream));
+  blk->ws_stride_prev = stride;
+  blk->ws_kind_prev = 3;
+  // bitmaps of every CTA first, then the b(u) arrays
+  P.bm = (uint32_t*)blk->b_ws.ptr;
+  P.acc = prob_mode == GS_PROB_DEGREE ? nullptr : (double*)((char*)blk->b_ws.ptr + bm_bytes * nctas);
+  P.col0 = (int32_t*)blk->b_col[0].ptr;
+  for (int l = 0; l < L; ++l) {
+    P.row_map[l] = (int32_t*)blk->b_row[l].ptr;
+    P.row_prob[l] = (float*)blk->b_rprob[l].ptr;
+    P.indptr_out[l] = (int64_t*)blk->b_indptr[l].ptr;
+    P.row_local[l] = (int32_t*)blk->b_rowl[l].ptr;
+    P.eid[l] = (int64_t*)blk->b_eid[l].ptr;
+    P.val[l] = (float*)blk->b_val[l].ptr;
+    P.edge_cap[l] = edge_cap[l];
+    gs_layer_buffers& lb = blk->layers[l];
+    lb = gs_layer_buffers{};
+    lb.col_map = l == 0 ? P.col0 : P.row_map[l - 1];
+    lb.col_capacity = l == 0 ? num_seeds : nbatch * (int64_t)P.K[l - 1];
+    lb.row_map = P.row_map[l];
+    lb.row_capacity = nbatch * (int64_t)P.K[l];
+    lb.indptr = P.indptr_out[l];
+    lb.indptr_capacity = lb.col_capacity + nbatch;
+    lb.row_local = P.row_local[l];
+    lb.eid = P.eid[l];
+    lb.val = P.val[l];
+    lb.edge_capacity = edge_cap[l];
+    lb.row_prob = P.row_prob[l];
+  }
+  P.edge_ctr = (unsigned long long*)blk->b_ctr.ptr;
+  P.need_tab = P.edge_ctr + MAX_LAYERS;
+  P.meta = (int64_t*)blk->b_meta.ptr;
+  P.err = (int*)blk->b_err.ptr;
+  GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
+  GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
+  if (nbatch == 0) return GS_OK;
+  layerwise_bm_kernel<<<nctas, LB_THREADS, smem, stream>>>(P);
+  GS_CUDA_TRY(cudaGetLastError());
+  return GS_OK;
+}
+
+}  // namespace gsb

@@ -32,7 +32,34 @@ struct WarpChunk {
   int32_t pre[32];                // exclusive prefix of the chunk's counts
   float csum[32];                 // PASS column sums
   int32_t cnt_all[32];            // count; bit 30: positions are 0..cnt-1
+  uint32_t smask[MAX_FANOUT];     // slot -> column map: bit f set iff slot f starts a column
+  uint8_t ne[32];                 // the chunk's non-empty columns, in order
 };
+
+// Builds the chunk's slot -> column map (warp-collective): slot f of the
+// chunk's flat slot space belongs to column ne[r], r = (number of column
+// starts <= f) - 1.  cnt / pre: this lane's column count and exclusive prefix.
+__device__ __forceinline__ void chunk_map_build(WarpChunk& C, int cnt, int pre) {
+  const int lane = threadIdx.x & 31;
+  C.smask[lane] = 0u;
+  __syncwarp();
+  const unsigned nem = __ballot_sync(0xffffffffu, cnt > 0);
+  if (cnt > 0) {
+    atomicOr(&C.smask[pre >> 5], 1u << (pre & 31));
+    C.ne[__popc(nem & ((1u << lane) - 1u))] = (uint8_t)lane;
+  }
+  __syncwarp();
+}
+
+// Column of slot f0 + lane in the round of slots [f0, f0 + 32) (f0 a multiple
+// of 32, rounds visited in order); `starts` = column starts before f0, advanced.
+__device__ __forceinline__ int chunk_map_col(const WarpChunk& C, int f0, int& starts) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t w = C.smask[f0 >> 5];
+  const int r = starts + __popc(w & ((2u << lane) - 1u)) - 1;
+  starts += __popc(w);
+  return C.ne[r < 0 ? 0 : r];
+}
 
 __device__ __forceinline__ uint32_t sel_word(const U4& r, int i) {
   return i == 0 ? r.x : (i == 1 ? r.y : (i == 2 ? r.z : r.w));

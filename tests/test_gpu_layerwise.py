@@ -20,6 +20,15 @@ def gs():
     return _gs
 
 
+@pytest.fixture(params=["bm", "old"], autouse=True)
+def lw_path(request, monkeypatch):
+    """Every test runs through both layer-wise kernels: the candidate-bitmap
+    kernel (layerwise_bm.cu, the default where it fits) and the hash-table
+    kernel (layerwise.cu, large graphs)."""
+    monkeypatch.setenv("GS_LW_PATH", request.param)
+    return request.param
+
+
 @pytest.fixture(scope="module")
 def ljlike(gs, oracle_lib):
     # LiveJournal-shaped (directed, GCN-normalised weights) at reduced size
@@ -81,3 +90,14 @@ def test_capacity_retry(gs, oracle_lib, ljlike):
     ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [2048], batch_size=2048, prob_mode=1,
                                       rng_key=1)
     compare_all(out.to_host(), ref, "fastgcn big")
+
+
+def test_ladies_bias_capacity_retry(gs, oracle_lib, ljlike):
+    """LADIES batch-layers with more candidates than the initial b(u) capacity
+    (32 Ki) overflow once; the binding grows the workspace and re-runs."""
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 10), 6000)
+    out = gs.sample_layerwise(G, seeds.cuda(), [3000, 3000], batch_size=3000, prob_mode=0, rng_key=2)
+    ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [3000, 3000], batch_size=3000, prob_mode=0,
+                                      rng_key=2)
+    compare_all(out.to_host(), ref, "ladies big")
