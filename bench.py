@@ -7,7 +7,7 @@ neighbour sampling, batch 1024, one full epoch of seeds (196,615 = the
 ogbn-products train-split size, 193 mini-batches) on an Ogbn-Products-shaped
 R-MAT graph (2,449,029 nodes, 61,859,140 undirected edges -> 123,718,280 CSC
 entries).  One step = one epoch (every batch, every hop: Extract, Select,
-Finalize) = one launch of the node-wise stream kernel.  Other configs of
+Finalize) = one launch of the node-wise wave kernel.  Other configs of
 BASELINE.json are selectable with --workload (parity cases / extra lines).
 
 Contract: python bench.py --gpus N --steps K --warmup W [--impl reference]
@@ -33,9 +33,13 @@ import torch  # noqa: E402
 
 METRIC = "sampled edges/s & epoch sampling time at 1/2/4/8 B200; % HBM roofline"
 UNIT = "sampled edges/s"
-# Random 32-byte-sector read ceiling of this B200's HBM, measured with
-# tools/microbench2.cu (profiles/r01_microbench.txt): ~55 G sectors/s.
-RANDOM_SECTOR_GBS = 1750.0
+# Random-access ceiling of this B200's HBM (profiles/r01_random_access_probe.md,
+# tools/microbench_l2fetch*.cu): every random load that misses L2 moves a
+# 128-byte line, ~36.9 G random loads/s on an 8 GB working set = 1181 GB/s of
+# useful 32-byte sectors.  The byte model counts 32 B per random sector, so a
+# gather-bound kernel's roofline.frac against the streaming peak cannot exceed
+# ~0.18; frac_of_random_sector_ceiling compares against this ceiling instead.
+RANDOM_SECTOR_GBS = 36.9e9 * 32 / 1e9
 
 WORKLOADS = {
     "graphsage_pd": dict(kind="nodewise", graph="PD", fanouts=[25, 10], batch=1024,

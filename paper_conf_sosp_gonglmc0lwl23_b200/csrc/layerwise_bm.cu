@@ -36,6 +36,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "gs_internal.h"
@@ -100,6 +101,29 @@ __device__ __forceinline__ int lb_col(const int32_t* fstart, int T, int64_t e) {
   }
   return lo;
 }
+
+// Flat-edge stream of one warp: a contiguous range of the batch-layer's flat
+// edge space (column-major, positions ascending), 32 * LB_ILP edges per round.
+// The column of each lane's edge is tracked incrementally (one binary search
+// per warp range, then a forward walk over the column starts).
+struct LBStream {
+  int64_t beg, end;
+  int c;
+  __device__ __forceinline__ LBStream(int64_t nflat) {
+    const int warp = threadIdx.x >> 5;
+    int64_t per = (nflat + LB_WARPS - 1) / LB_WARPS;
+    per = (per + 31) & ~int64_t(31);
+    beg = min((int64_t)warp * per, nflat);
+    end = min(beg + per, nflat);
+    c = -1;
+  }
+  // column of flat edge e (e < end, visited in increasing order per lane)
+  __device__ __forceinline__ int col(const int32_t* fstart, int T, int64_t e) {
+    if (c < 0) c = lb_col(fstart, T, e);
+    while (fstart[c + 1] <= e) ++c;
+    return c;
+  }
+};
 
 __device__ __forceinline__ int popc4(const uint4& x) {
   return __popc(x.x) + __popc(x.y) + __popc(x.z) + __popc(x.w);
@@ -308,21 +332,25 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       const int64_t nflat = T > 0 ? (int64_t)sh.u64[1] : 0;
 
       // ---- L1: Extract, the rows' bits (one red.or per distinct row per warp round) ----
-      for (int64_t e0 = (int64_t)threadIdx.x - lane; e0 < nflat; e0 += (int64_t)blockDim.x * LB_ILP) {
-        uint32_t u[LB_ILP];
+      {
+        LBStream st(nflat);
+        for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
+          uint32_t u[LB_ILP];
 #pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          const int64_t e = e0 + (int64_t)q * blockDim.x + lane;
-          u[q] = 0xFFFFFFFFu;
-          if (e < nflat) {
-            const int c = lb_col(s_fstart, Ti, e);
-            u[q] = (uint32_t)__ldg(P.indices + s_off[c] + (e - s_fstart[c]));
+          for (int q = 0; q < LB_ILP; ++q) {
+            const int64_t e = e0 + 32 * q + lane;
+            u[q] = 0xFFFFFFFFu;
+            if (e < st.end) {
+              const int c = st.col(s_fstart, Ti, e);
+              u[q] = (uint32_t)__ldg(P.indices + s_off[c] + (e - s_fstart[c]));
+            }
           }
-        }
 #pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          const uint32_t peers = __match_any_sync(0xffffffffu, u[q]);
-          if (u[q] != 0xFFFFFFFFu && (__ffs(peers) - 1) == lane) atomicOr(bm + (u[q] >> 5), 1u << (u[q] & 31));
+          for (int q = 0; q < LB_ILP; ++q) {
+            const uint32_t peers = __match_any_sync(0xffffffffu, u[q]);
+            if (u[q] != 0xFFFFFFFFu && (__ffs(peers) - 1) == lane)
+              atomicOr(bm + (u[q] >> 5), 1u << (u[q] & 31));
+          }
         }
       }
       __syncthreads();
@@ -487,33 +515,45 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       }
       __syncthreads();
 
-      // ---- L5a: per column kept count and c_j = sum_fp64 a (a = w / p(u)) ----
-      for (int64_t e0 = threadIdx.x; e0 < nflat && nsel > 0; e0 += (int64_t)blockDim.x * LB_ILP) {
-        uint32_t u[LB_ILP];
-        int c[LB_ILP];
-        int64_t pos[LB_ILP];
+      // ---- L5a: per column kept count and c_j = sum_fp64 a (a = w / p(u)),
+      // per warp kept count (the warp's offset in the CSC emit order) ----
+      int wkept = 0;
+      {
+        LBStream st(nflat);
+        for (int64_t e0 = st.beg; e0 < st.end && nsel > 0; e0 += 32 * LB_ILP) {
+          uint32_t u[LB_ILP];
+          int c[LB_ILP];
+          int64_t pos[LB_ILP];
 #pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          const int64_t e = e0 + (int64_t)q * blockDim.x;
-          u[q] = 0xFFFFFFFFu;
-          if (e < nflat) {
-            c[q] = lb_col(s_fstart, Ti, e);
-            pos[q] = s_off[c[q]] + (e - s_fstart[c[q]]);
-            u[q] = (uint32_t)__ldg(P.indices + pos[q]);
+          for (int q = 0; q < LB_ILP; ++q) {
+            const int64_t e = e0 + 32 * q + lane;
+            u[q] = 0xFFFFFFFFu;
+            c[q] = 0;
+            pos[q] = 0;
+            if (e < st.end) {
+              c[q] = st.col(s_fstart, Ti, e);
+              pos[q] = s_off[c[q]] + (e - s_fstart[c[q]]);
+              u[q] = (uint32_t)__ldg(P.indices + pos[q]);
+            }
+          }
+#pragma unroll
+          for (int q = 0; q < LB_ILP; ++q) {
+            const int lid = u[q] == 0xFFFFFFFFu ? -1 : lb_lookup(s_hk, s_hv, u[q]);
+            wkept += __popc(__ballot_sync(0xffffffffu, lid >= 0));
+            if (lid < 0) continue;
+            const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
+            const float p = __uint_as_float((uint32_t)s_sel[lid]);
+            atomicAdd(&s_cnt[c[q]], 1);
+            atomicAdd(&s_cs[c[q]], (double)__fdiv_rn(w, p));
           }
         }
-#pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          if (u[q] == 0xFFFFFFFFu) continue;
-          const int lid = lb_lookup(s_hk, s_hv, u[q]);
-          if (lid < 0) continue;
-          const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
-          const float p = __uint_as_float((uint32_t)s_sel[lid]);
-          atomicAdd(&s_cnt[c[q]], 1);
-          atomicAdd(&s_cs[c[q]], (double)__fdiv_rn(w, p));
-        }
       }
+      if (lane == 0) sh.wtot[threadIdx.x >> 5] = wkept;
       __syncthreads();
+      if (threadIdx.x < 32) {  // warps' exclusive offsets in the emit order
+        const int v = sh.wtot[lane];
+        sh.wtot[lane] = warp_inclusive_scan(v) - v;
+      }
       int64_t E = 0;
       for (int j0 = 0; j0 < Ti; j0 += blockDim.x) {
         const int j = j0 + threadIdx.x;
@@ -530,39 +570,41 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       const bool fits = ebase + E <= P.edge_cap[l];
       if (!fits && threadIdx.x == 0) atomicOr(P.err, ERR_CAPACITY);
 
-      // ---- L5b: emit in CSC order (flat order is column-major, positions
-      // ascending: an exclusive scan of the keep flags is the output index) ----
-      int64_t krun = 0;
-      for (int64_t e0 = 0; e0 < nflat && fits && E > 0; e0 += (int64_t)blockDim.x * LB_ILP) {
-        const int64_t eb = e0 + (int64_t)threadIdx.x * LB_ILP;
-        int lid[LB_ILP];
-        int c[LB_ILP];
-        int64_t pos[LB_ILP];
-        int kc = 0;
+      // ---- L5b: emit in CSC order (the flat order is column-major with
+      // ascending positions; warps own contiguous flat ranges in order) ----
+      if (fits && E > 0) {
+        LBStream st(nflat);
+        int64_t o = ebase + sh.wtot[threadIdx.x >> 5];
+        for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
+          int lid[LB_ILP];
+          int c[LB_ILP];
+          int64_t pos[LB_ILP];
 #pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          lid[q] = -1;
-          if (eb + q < nflat) {
-            c[q] = lb_col(s_fstart, Ti, eb + q);
-            pos[q] = s_off[c[q]] + (eb + q - s_fstart[c[q]]);
-            lid[q] = lb_lookup(s_hk, s_hv, (uint32_t)__ldg(P.indices + pos[q]));
+          for (int q = 0; q < LB_ILP; ++q) {
+            const int64_t e = e0 + 32 * q + lane;
+            lid[q] = -1;
+            c[q] = 0;
+            pos[q] = 0;
+            if (e < st.end) {
+              c[q] = st.col(s_fstart, Ti, e);
+              pos[q] = s_off[c[q]] + (e - s_fstart[c[q]]);
+              lid[q] = lb_lookup(s_hk, s_hv, (uint32_t)__ldg(P.indices + pos[q]));
+            }
           }
-          kc += lid[q] >= 0 ? 1 : 0;
-        }
-        unsigned long long tot;
-        const unsigned long long ex = block_exclusive_scan((unsigned long long)kc, sh.scan, &tot);
-        int64_t o = ebase + krun + (int64_t)ex;
 #pragma unroll
-        for (int q = 0; q < LB_ILP; ++q) {
-          if (lid[q] < 0) continue;
-          const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
-          const float a = __fdiv_rn(w, __uint_as_float((uint32_t)s_sel[lid[q]]));
-          P.row_local[l][o] = lid[q];
-          P.eid[l][o] = pos[q];
-          P.val[l][o] = __fdiv_rn(a, (float)s_cs[c[q]]);
-          ++o;
+          for (int q = 0; q < LB_ILP; ++q) {
+            const unsigned bal = __ballot_sync(0xffffffffu, lid[q] >= 0);
+            if (lid[q] >= 0) {
+              const int64_t oi = o + __popc(bal & ((1u << lane) - 1u));
+              const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
+              const float a = __fdiv_rn(w, __uint_as_float((uint32_t)s_sel[lid[q]]));
+              P.row_local[l][oi] = lid[q];
+              P.eid[l][oi] = pos[q];
+              P.val[l][oi] = __fdiv_rn(a, (float)s_cs[c[q]]);
+            }
+            o += __popc(bal);
+          }
         }
-        krun += (int64_t)tot;
       }
       if (threadIdx.x == 0) {
         P.indptr_out[l][ibase + T] = E;
@@ -672,7 +714,9 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   GS_CUDA_TRY(cudaFuncSetAttribute(layerwise_bm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)smem));
-  const int nctas = (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, sms));
+  int ctas = sms;
+  if (const char* e = getenv("GS_LW_CTAS")) ctas = std::max(1, std::min(atoi(e), sms));
+  const int nctas = (int)std::max<int64_t>(1, std::min<int64_t>(nbatch, ctas));
   // per-CTA workspace: bitmap (kept zero), b(u) by rank (kept zero)
   P.acc_cap = prob_mode == GS_PROB_DEGREE ? 0 : std::max<int64_t>(int64_t(1) << 15, blk->lw_tab_hint);
   const int64_t bm_bytes = a256(n4 * 16);

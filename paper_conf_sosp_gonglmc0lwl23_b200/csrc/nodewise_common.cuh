@@ -78,17 +78,6 @@ __device__ __forceinline__ int warp_excl(int v, int* total) {
   return inc - v;
 }
 
-// Last column c of the chunk with pre[c] <= f (the column holding flat slot f).
-__device__ __forceinline__ int chunk_col(const int32_t* pre, int f) {
-  int lo = 0, hi = 31;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (pre[mid] <= f) lo = mid;
-    else hi = mid - 1;
-  }
-  return lo;
-}
-
 // ---------------------------------------------------------------------------
 // A-Res by candidate filtering (R6).  The k smallest exact keys
 // key_i = -ln((r_i + 0.5) 2^-32) / w_i (fp64, as the oracle) are found among

@@ -253,6 +253,50 @@ __device__ __forceinline__ void nv_cols(const NVParams& P, WarpChunk& C, const N
   d_out = d;
 }
 
+// Uniform select (GraphSAGE Floyd, R5; KGCN replacement, R10), lane per column.
+// (v, d in registers: the Floyd loop stores into C.list, which would force
+// reloads of anything read back from the same shared-memory struct)
+__device__ void nv_select_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg, const int32_t v,
+                                  const int64_t d) {
+  const int lane = threadIdx.x & 31;
+  const int l = sg.l, k = P.k[l];
+  const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
+  int cnt = 0;
+  bool all = false;
+  if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
+    cnt = d > 0 ? k : 0;
+    for (int s = 0; s < cnt; ++s) {
+      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
+      C.list[s][lane] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
+    }
+  } else if (d <= k) {  // GraphSAGE, d <= k: every neighbour (R5)
+    cnt = (int)d;
+    all = true;
+  } else {  // GraphSAGE (R5): Floyd; the list stays sorted (m is always appended)
+    cnt = k;
+    int n = 0;
+    for (int s = 0; s < k; ++s) {
+      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.core.key);
+      const uint32_t m = (uint32_t)(d - k + s);
+      const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
+      int lo = 0, hi = n;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (C.list[mid][lane] < t) lo = mid + 1;
+        else hi = mid;
+      }
+      if (lo < n && C.list[lo][lane] == t) {
+        C.list[n][lane] = m;
+      } else {
+        for (int q = n; q > lo; --q) C.list[q][lane] = C.list[q - 1][lane];
+        C.list[lo][lane] = t;
+      }
+      ++n;
+    }
+  }
+  C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
+}
+
 // A-Res threshold search state: tau is widened / narrowed geometrically, or
 // bisected once both a too-small and a too-large value are known.
 struct TauSearch {
@@ -368,15 +412,16 @@ __device__ void nv_select_heavy(const NVParams& P, NVSmem& sm, NVWeighted& W, co
 }
 
 // Stage A, per warp after the select: stage the positions, gather every
-// sampled row of the chunk at once and set the rows' bits.  C.cnt_all, C.coff
-// and C.list are set; returns the chunk's edge count.
-__device__ __forceinline__ int nv_gather_rows(const NVParams& P, WarpChunk& C, const NVSeg& sg,
-                                              long long jb, int cnt) {
+// sampled row of the chunk at once and set the rows' bits.  Returns the
+// chunk's edge count.
+__device__ int nv_gather(const NVParams& P, WarpChunk& C, const NVSeg& sg, long long jb) {
   const int lane = threadIdx.x & 31;
-  const int k = P.k[sg.l];
-  const NVStage S = nv_stage(P, sg.j, sg.l, sg.g);
+  const int l = sg.l;
+  const int k = P.k[l];
+  const NVStage S = nv_stage(P, sg.j, l, sg.g);
   const uint64_t pf = pol_first(), pl = pol_last();
   const long long jcol = jb + lane;
+  const int cnt = C.cnt_all[lane] & ~(1 << 30);
   int total;
   const int pre = warp_excl(cnt, &total);
   C.pre[lane] = pre;
@@ -384,7 +429,8 @@ __device__ __forceinline__ int nv_gather_rows(const NVParams& P, WarpChunk& C, c
     sth(S.coff + jcol, C.coff[lane], pl);
     sth(S.cnt + jcol, cnt, pl);
   }
-  chunk_map_build(C, cnt, pre);
+  __syncwarp();
+  chunk_map_build(C, C.cnt_all[lane] & ~(1 << 30), C.pre[lane]);
   // (a) every sampled row of the chunk is requested at once: cp.async of the
   // gathered id straight into the position's own list cell (the position is
   // read, and staged, before its cell is overwritten)
@@ -392,20 +438,19 @@ __device__ __forceinline__ int nv_gather_rows(const NVParams& P, WarpChunk& C, c
   for (int f0 = 0; f0 < total; f0 += 32) {
     const int f = f0 + lane;
     const int c = chunk_map_col(C, f0, starts);
-    if (f < total) {
-      const int q = f - C.pre[c];
-      const uint32_t ps = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)q : C.list[q][c];
-      const uint32_t p = (uint32_t)((jb + c) * k + q);
-      sth(S.pos + p, ps, pl);
-      if (S.val) {
-        const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
-        sth(S.val + p, w / C.csum[c], pl);
-      }
-      const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
-      asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
-                   "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
-                   : "memory");
+    if (f >= total) continue;
+    const int q = f - C.pre[c];
+    const uint32_t ps = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)q : C.list[q][c];
+    const uint32_t p = (uint32_t)((jb + c) * k + q);
+    sth(S.pos + p, ps, pl);
+    if (S.val) {
+      const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
+      sth(S.val + p, w / C.csum[c], pl);
     }
+    const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
+                 "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
+                 : "memory");
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
   asm volatile("cp.async.wait_all;" ::: "memory");
@@ -415,8 +460,8 @@ __device__ __forceinline__ int nv_gather_rows(const NVParams& P, WarpChunk& C, c
   starts = 0;
   for (int f0 = 0; f0 < total; f0 += 32) {
     const int f = f0 + lane;
-    const int c = chunk_map_col(C, f0, starts);
     uint32_t u = 0xFFFFFFFFu;
+    const int c = chunk_map_col(C, f0, starts);
     if (f < total) {
       const int q = f - C.pre[c];
       u = C.list[q][c];
@@ -438,6 +483,8 @@ __device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg
   const int lane = threadIdx.x & 31;
   const int l = sg.l;
   const int k = P.k[l];
+  const NVStage S = nv_stage(P, sg.j, l, sg.g);
+  const uint64_t pf = pol_first(), pl = pol_last();
   const int32_t* F = nv_frontier(P, sg.b, l);
   const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
   const long long jcol = jb + lane;
@@ -450,6 +497,7 @@ __device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg
     off = __ldg(P.core.indptr + v);
     d = __ldg(P.core.indptr + v + 1) - off;
   }
+  const bool weighted = false;
   int cnt = 0;
   bool all = false;
   if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
@@ -483,9 +531,61 @@ __device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg
       ++n;
     }
   }
+  int total;
+  const int pre = warp_excl(cnt, &total);
   C.coff[lane] = off;
-  C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
-  return nv_gather_rows(P, C, sg, jb, cnt);
+  C.pre[lane] = pre;
+  if (!weighted) C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
+  if (active) {
+    sth(S.coff + jcol, off, pl);
+    sth(S.cnt + jcol, cnt, pl);
+  }
+  __syncwarp();
+  chunk_map_build(C, C.cnt_all[lane] & ~(1 << 30), C.pre[lane]);
+  // (a) every sampled row of the chunk is requested at once: cp.async of the
+  // gathered id straight into the position's own list cell (the position is
+  // read, and staged, before its cell is overwritten)
+  int starts = 0;
+  for (int f0 = 0; f0 < total; f0 += 32) {
+    const int f = f0 + lane;
+    const int c = chunk_map_col(C, f0, starts);
+    if (f >= total) continue;
+    const int q = f - C.pre[c];
+    const uint32_t ps = (C.cnt_all[c] & (1 << 30)) ? (uint32_t)q : C.list[q][c];
+    const uint32_t p = (uint32_t)((jb + c) * k + q);
+    sth(S.pos + p, ps, pl);
+    if (S.val) {
+      const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
+      sth(S.val + p, w / C.csum[c], pl);
+    }
+    const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
+                 "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  __syncwarp();
+  // (b) stage the rows and set their bits in the segment's row bitmap
+  // (fire-and-forget red.or; a row's bit is set once per warp round)
+  starts = 0;
+  for (int f0 = 0; f0 < total; f0 += 32) {
+    const int f = f0 + lane;
+    uint32_t u = 0xFFFFFFFFu;
+    const int c = chunk_map_col(C, f0, starts);
+    if (f < total) {
+      const int q = f - C.pre[c];
+      u = C.list[q][c];
+      sth(S.u + (jb + c) * k + q, (int32_t)u, pl);
+    }
+    const uint32_t peers = __match_any_sync(0xffffffffu, u);
+    if (f < total && (__ffs(peers) - 1) == lane)
+      asm volatile("red.global.or.b32 [%0], %1;" ::"l"((uint32_t*)(S.bm + (u >> 5))),
+                   "r"(1u << (u & 31))
+                   : "memory");
+  }
+  __syncwarp();
+  return total;
 }
 
 // Stage A tile: 512 columns, one 32-column chunk per warp; the tile's edge count.
@@ -508,7 +608,7 @@ __device__ void nv_stage_a(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
     }
     __syncthreads();
     nv_select_heavy(P, sm, W, sg);
-    if (has) e = nv_gather_rows(P, C, sg, jb, C.cnt_all[lane] & ~(1 << 30));
+    if (has) e = nv_gather(P, C, sg, jb);
   } else if (has) {
     e = nv_chunk_uniform(P, C, sg, jb);
   }

@@ -32,7 +32,7 @@ constexpr int SH_THREADS = 512;
 constexpr int SH_WARPS = SH_THREADS / 32;
 constexpr int SH_MAX_CS = 8;                      // portable cluster size
 constexpr int SH_ILP = 8;                         // column positions per lane in flight
-constexpr int64_t SH_SMEM_CAP = 200 * 1024;      // dynamic shared memory per CTA (bitmap + prefix)
+constexpr int64_t SH_SMEM_CAP = 220 * 1024;      // dynamic shared memory per CTA (bitmap + prefixes)
 
 struct SHParams {
   const int64_t* indptr;
@@ -56,6 +56,7 @@ struct SHParams {
   int* err;
   unsigned int* claim;
   int64_t bpc;                      // bitmap bits per CTA (multiple of 256)
+  uint32_t inv;                     // floor(2^32 / bpc)
 };
 
 struct SHShared {                   // static part; the bitmap + prefix are dynamic
@@ -66,24 +67,33 @@ struct SHShared {                   // static part; the bitmap + prefix are dyna
   int scr32[40];
 };
 
-__device__ __forceinline__ bool sh_member(const cg::cluster_group& cl, uint32_t* bm, int64_t bpc,
-                                          uint32_t u) {
-  const unsigned owner = (unsigned)(u / (uint64_t)bpc);
-  const uint32_t x = u - owner * (uint32_t)bpc;
+// Owner CTA of bit u: u / bpc by a 32-bit reciprocal (inv = floor(2^32 / bpc))
+// and one correction step (no 64-bit division on the per-edge path).
+__device__ __forceinline__ unsigned sh_owner(uint32_t u, uint32_t bpc, uint32_t inv) {
+  unsigned q = __umulhi(u, inv);
+  if ((q + 1u) * bpc <= u) ++q;
+  return q;
+}
+
+__device__ __forceinline__ bool sh_member(const cg::cluster_group& cl, uint32_t* bm, uint32_t bpc,
+                                          uint32_t inv, uint32_t u) {
+  const unsigned owner = sh_owner(u, bpc, inv);
+  const uint32_t x = u - owner * bpc;
   const uint32_t* w = cl.map_shared_rank(bm, owner);
   return (w[x >> 5] >> (x & 31)) & 1u;
 }
 
+// Rank of u in U: the owner's base + its 256-bit group prefix + the word's
+// offset inside the group (one byte per word) + the bits below u in its word.
 __device__ __forceinline__ long long sh_rank(const cg::cluster_group& cl, uint32_t* bm, int32_t* gp,
-                                             const SHShared& ss, int64_t bpc, uint32_t u) {
-  const unsigned owner = (unsigned)(u / (uint64_t)bpc);
-  const uint32_t x = u - owner * (uint32_t)bpc;
+                                             uint8_t* off8, const SHShared& ss, uint32_t bpc,
+                                             uint32_t inv, uint32_t u) {
+  const unsigned owner = sh_owner(u, bpc, inv);
+  const uint32_t x = u - owner * bpc;
   const uint32_t* w = cl.map_shared_rank(bm, owner);
   const int32_t* p = cl.map_shared_rank(gp, owner);
-  const uint32_t wi = x >> 5, g0 = (x >> 8) << 3;
-  long long r = ss.base[owner] + p[x >> 8];
-  for (uint32_t i = g0; i < wi; ++i) r += __popc(w[i]);
-  return r + __popc(w[wi] & ((1u << (x & 31)) - 1u));
+  const uint8_t* o = cl.map_shared_rank(off8, owner);
+  return ss.base[owner] + p[x >> 8] + o[x >> 5] + __popc(w[x >> 5] & ((1u << (x & 31)) - 1u));
 }
 
 __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P) {
@@ -96,6 +106,8 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
   const int nwords = (int)(bpc >> 5), ngroups = (int)(bpc >> 8);
   uint32_t* bm = (uint32_t*)smem_raw;
   int32_t* gp = (int32_t*)(smem_raw + (size_t)nwords * 4);
+  uint8_t* off8 = (uint8_t*)(gp + ngroups);
+  const uint32_t bpc32 = (uint32_t)bpc, inv = P.inv;
   const uint64_t pf = pol_first();
   while (true) {
     if (rank == 0 && tid == 0) ss.b = (long long)atomicAdd(P.claim, 1u);
@@ -129,8 +141,8 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
         atomicOr(P.err, ERR_SEED_RANGE);
         continue;
       }
-      const unsigned owner = (unsigned)((uint32_t)u / (uint64_t)bpc);
-      const uint32_t xb = (uint32_t)u - owner * (uint32_t)bpc;
+      const unsigned owner = sh_owner((uint32_t)u, bpc32, inv);
+      const uint32_t xb = (uint32_t)u - owner * bpc32;
       atomicOr(cl.map_shared_rank(bm, owner) + (xb >> 5), 1u << (xb & 31));
     }
     cl.sync();
@@ -141,7 +153,10 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       int c = 0;
       if (g < ngroups)
 #pragma unroll
-        for (int i = 0; i < 8; ++i) c += __popc(bm[g * 8 + i]);
+        for (int i = 0; i < 8; ++i) {
+          off8[g * 8 + i] = (uint8_t)c;
+          c += __popc(bm[g * 8 + i]);
+        }
       int tot;
       const int ex = block_exclusive_scan<int>(c, ss.scr32, &tot);
       if (g < ngroups) gp[g] = (int32_t)(run + ex);
@@ -190,7 +205,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
         }
 #pragma unroll
         for (int q = 0; q < SH_ILP; ++q)
-          cnt += __popc(__ballot_sync(0xffffffffu, u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc, u[q])));
+          cnt += __popc(__ballot_sync(0xffffffffu, u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q])));
       }
       if (lane == 0) ucnt[c] = cnt;
     }
@@ -246,13 +261,13 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
             u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
           }
 #pragma unroll
-          for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc, u[q]);
+          for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q]);
 #pragma unroll
           for (int q = 0; q < SH_ILP; ++q) {
             const uint32_t bal = __ballot_sync(0xffffffffu, m[q]);
             if (m[q]) {
               const long long e = pos + __popc(bal & ((1u << lane) - 1u));
-              sth(P.row_local + e, (int32_t)sh_rank(cl, bm, gp, ss, bpc, u[q]), pf);
+              sth(P.row_local + e, (int32_t)sh_rank(cl, bm, gp, off8, ss, bpc32, inv, u[q]), pf);
               sth(P.eid + e, (int64_t)(o + i0 + q * 32 + lane), pf);
             }
             pos += __popc(bal);
@@ -273,11 +288,11 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   int64_t bpc = 0;
   for (; CS <= SH_MAX_CS; CS *= 2) {
     bpc = ((N + CS - 1) / CS + 255) / 256 * 256;
-    if (bpc / 8 + bpc / 64 <= SH_SMEM_CAP) break;
+    if (bpc / 8 + bpc / 64 + bpc / 32 <= SH_SMEM_CAP) break;
   }
   if (CS > SH_MAX_CS)
     return fail(GS_ERR_NOT_SUPPORTED, "ShaDow: N = %lld exceeds the shared-memory bitmap envelope (%lld nodes)",
-                (long long)N, (long long)(SH_MAX_CS * (SH_SMEM_CAP * 64 / 9)));
+                (long long)N, (long long)(SH_MAX_CS * (SH_SMEM_CAP * 64 / 11)));
   // 1. node-wise sampling of every hop (internal result object)
   if (!blk->aux) {
     blk->aux = new (std::nothrow) gs_blocks();
@@ -350,13 +365,14 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   P.err = (int*)blk->b_err.ptr;
   P.claim = (unsigned int*)((char*)blk->b_ctr.ptr + 8 * (MAX_LAYERS + 1));
   P.bpc = bpc;
+  P.inv = (uint32_t)((uint64_t(1) << 32) / (uint64_t)bpc);
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
   // the node-wise kernel's error word (out-of-range seeds) is folded in
   GS_CUDA_TRY(cudaMemcpyAsync(blk->b_err.ptr, nw->b_err.ptr, 4, cudaMemcpyDeviceToDevice, stream));
 
-  const size_t smem = (size_t)(bpc / 8 + bpc / 64);
+  const size_t smem = (size_t)(bpc / 8 + bpc / 64 + bpc / 32);
   GS_CUDA_TRY(cudaFuncSetAttribute(shadow_induce_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)smem));
   cudaLaunchConfig_t cfg = {};
