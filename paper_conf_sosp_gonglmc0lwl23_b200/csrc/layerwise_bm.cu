@@ -89,6 +89,7 @@ struct LBShared {
   double dred[33];
   int misc[8];
   unsigned long long u64[4];
+  double tau_est[MAX_LAYERS];       // FastGCN: select threshold estimate per layer (previous batch)
   int wtot[LB_WARPS];
 };
 
@@ -175,10 +176,21 @@ __device__ __forceinline__ void lb_for_bits(const LBParams& P, const uint4* bm4,
   }
 }
 
+// Candidate buffer of the select (shared memory).
+struct LBBuf {
+  unsigned long long* k;  // exact fp64 key bits
+  uint32_t* u;
+  float* b;
+};
+
 // s_gp[g] = number of candidates before rank group g; returns |C|.  FastGCN:
-// also b(u) = deg(u) summed (B, fp64) and the eligible count.
+// also b(u) = deg(u) summed (B, fp64) and the eligible count, and -- with a
+// threshold estimate tau_est > 0 (from the CTA's previous batch at this
+// layer) -- every candidate with exact key < tau_est appended to the buffer
+// (counter sh.misc[6]), so that usually no second pass over C is needed.
 __device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, int32_t* s_gp,
-                            bool degree, double* B_out, int64_t* nelig_out) {
+                            bool degree, double* B_out, int64_t* nelig_out, double tau_est, int l,
+                            uint32_t gb, const LBBuf& buf) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gq = 1 << (P.gw_log - 2);
   const int gpw = (P.ng + LB_WARPS - 1) / LB_WARPS;
@@ -201,9 +213,25 @@ __device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, i
         while (w) {
           const int bpos = __ffs(w) - 1;
           w &= w - 1u;
-          const int32_t dg = __ldg(P.deg + (i * 4 + j) * 32 + bpos);
+          const uint32_t u = (uint32_t)((i * 4 + j) * 32 + bpos);
+          const int32_t dg = __ldg(P.deg + u);
           bsum += (double)(float)dg;
           elig += dg > 0 ? 1 : 0;
+          if (tau_est > 0.0 && dg > 0) {
+            const float bb = (float)dg;
+            const U4 R = philox(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.key);
+            if (ares_maybe_below(R.x, (float)(tau_est * (double)bb) * 1.01f)) {
+              const double kk = ares_key(R.x, (double)bb);
+              if (kk < tau_est) {
+                const int slot = atomicAdd(&sh.misc[6], 1);
+                if (slot < LB_CAP) {
+                  buf.k[slot] = (unsigned long long)__double_as_longlong(kk);
+                  buf.u[slot] = u;
+                  buf.b[slot] = bb;
+                }
+              }
+            }
+          }
         }
       }
     }
@@ -287,6 +315,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
   const uint4* bm4 = (const uint4*)bm;
   double* acc = P.acc ? P.acc + (int64_t)blockIdx.x * P.acc_cap : nullptr;
   const bool degree = P.mode == GS_PROB_DEGREE;
+  if (threadIdx.x < MAX_LAYERS) sh.tau_est[threadIdx.x] = 0.0;
 
   for (int64_t b = blockIdx.x; b < P.num_batches; b += gridDim.x) {
     const int64_t bstart = b * P.batch_size;
@@ -358,7 +387,12 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       // ---- L2: rank groups (FastGCN: b(u) = in-degree, B, eligible) ----
       double Btot = 0.0;
       int64_t nelig = 0;
-      const int64_t nc = lb_ranks(P, sh, bm4, s_gp, degree, &Btot, &nelig);
+      if (threadIdx.x == 0) sh.misc[6] = 0;
+      __syncthreads();
+      const double tau_est = degree ? sh.tau_est[l] : 0.0;
+      const int64_t nc = lb_ranks(P, sh, bm4, s_gp, degree, &Btot, &nelig, tau_est, l, gb,
+                                  LBBuf{s_bk, s_bu, s_bb});
+      const int m_fused = sh.misc[6];
       bool acc_ok = true;
       if (!degree && nc > P.acc_cap) {
         if (threadIdx.x == 0) {
@@ -431,7 +465,9 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
         // threshold filter: keys below tau, ~2K of them (R6: exact fp64 key)
         double tau = 2.0 * K / Btot, lo = 0.0, hi = 0.0;
         int m = 0;
-        for (int it = 0; it < 64; ++it) {
+        const bool fused = tau_est > 0.0 && m_fused >= K && m_fused <= LB_CAP;
+        if (fused) m = m_fused;
+        for (int it = 0; it < 64 && !fused; ++it) {
           if (threadIdx.x == 0) sh.misc[0] = 0;
           __syncthreads();
           lb_for_bits(P, bm4, s_gp, [&](uint32_t u, int64_t r) {
@@ -470,6 +506,8 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
         __syncthreads();
         lb_sort_kv(s_bk, s_bu, s_bb, n2);  // (key, u) ascending: the K smallest first
         nsel = min(K, m);
+        // next batch at this layer: ~3K expected candidates below the estimate
+        if (degree && threadIdx.x == 0) sh.tau_est[l] = 3.0 * K / Btot;
       }
       // S sorted by node id (R3): (u << 32 | bias bits)
       int n2 = 1;

@@ -40,7 +40,7 @@ namespace gsb {
 constexpr int NV_THREADS = 512;
 constexpr int NV_WARPS = NV_THREADS / 32;
 constexpr int NV_TC = 512;        // frontier columns per tile (stages A, C)
-constexpr int NV_MAXSEG = 256;    // live (stage, hop, batch) segments per super-step
+constexpr int NV_MAXSEG = 512;    // live (stage, hop, batch) segments per super-step (<= NV_THREADS)
 constexpr int NV_BW = 16;         // bitmap words per thread (stage B)
 constexpr int NV_BT = NV_THREADS * NV_BW;  // bitmap words per stage-B tile
 constexpr int NV_BT_LOG = 13;
@@ -855,11 +855,12 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   const int64_t nbatch = P.num_batches;
   P.nw = ((g->num_nodes + 31) / 32 + 1) & ~int64_t(1);  // even: 16-byte aligned bitmaps
   P.nbt = (int)((P.nw + NV_BT - 1) / NV_BT);
-  // batches per group: ~8 M padded slots in the deepest hop (measured on the
-  // PD-shaped GraphSAGE epoch: 32 batches of 1024 beat 16 / 8 / 4), <= 4 GB of bitmaps
+  // batches per group: ~16 M padded slots in the deepest hop (measured on the
+  // PD-shaped GraphSAGE epoch: 64 batches of 1024 1.47 ms, 48 1.49, 32 1.54,
+  // 16 2.7), <= 4 GB of bitmaps, <= NV_MAXSEG live segments
   {
     const int64_t deep = std::max<int64_t>(1, batch_size * P.K[L - 1]);
-    int64_t wb = std::max<int64_t>(1, (int64_t(8) << 20) / deep);
+    int64_t wb = std::max<int64_t>(1, (int64_t(16) << 20) / deep);
     wb = std::min<int64_t>(wb, std::max<int64_t>(1, (int64_t(4) << 30) / (4 * L * P.nw * 8)));
     wb = std::min<int64_t>(wb, NV_MAXSEG / (4 * L));
     if (const char* e = getenv("GS_WAVE")) wb = std::max(1, std::min(atoi(e), NV_MAXSEG / (4 * L)));
