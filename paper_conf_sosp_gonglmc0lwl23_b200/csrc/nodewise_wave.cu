@@ -41,6 +41,7 @@ constexpr int NV_THREADS = 512;
 constexpr int NV_WARPS = NV_THREADS / 32;
 constexpr int NV_TC = 512;        // frontier columns per tile (stages A, C)
 constexpr int NV_MAXSEG = 512;    // live (stage, hop, batch) segments per super-step (<= NV_THREADS)
+constexpr int NV_MAXSEG_W = 256;  // ... in the weighted (A-Res) kernel
 constexpr int NV_BW = 16;         // bitmap words per thread (stage B)
 constexpr int NV_BT = NV_THREADS * NV_BW;  // bitmap words per stage-B tile
 constexpr int NV_BT_LOG = 13;
@@ -67,6 +68,9 @@ struct NVParams {
   long long* T;                 // [num_batches][L] frontier sizes (l > 0 written by stage B)
   unsigned int* ctr;            // [S][4 + NV_MAXSEG] work counters, zeroed per launch
   unsigned long long* bm;       // row bitmaps: (j, l, g & 3) at bm + ((g&3)*L + l)*WB + j) * nw
+  uint32_t* sm;                 // summaries (hops with use_sum): bit w set iff bitmap word w is non-empty
+  int64_t nsw;                  // 32-bit summary words per bitmap
+  int use_sum[MAX_LAYERS];      // hop l's rows are sparse in N (B visits only non-empty words)
   int64_t nw;                   // 64-bit bitmap words per bitmap = ceil(N / 32)
   char* stg;                    // staging, per (j, l, g & 3)
   int64_t stg_off[MAX_LAYERS], stg_stride[MAX_LAYERS];
@@ -90,6 +94,7 @@ struct NVStage {
   int32_t* bcnt;             // [bitmap tile] rows of the tile (stage B)
   int32_t* bx;               // [bitmap tile] exclusive row prefix (stage B)
   unsigned long long* bm;    // [nw] row bitmap: bits (low) | row prefix (high)
+  uint32_t* sm;              // [nsw] summary of the bitmap's non-empty words
 };
 
 __device__ __forceinline__ NVStage nv_stage(const NVParams& P, int j, int l, int g) {
@@ -106,6 +111,7 @@ __device__ __forceinline__ NVStage nv_stage(const NVParams& P, int j, int l, int
   s.bcnt = (int32_t*)(base + P.o_bcnt[l]);
   s.bx = (int32_t*)(base + P.o_bx[l]);
   s.bm = P.bm + ((int64_t)(r * P.L + l) * P.WB + j) * P.nw;
+  s.sm = P.sm + ((int64_t)(r * P.L + l) * P.WB + j) * P.nsw;
   return s;
 }
 
@@ -132,12 +138,15 @@ struct NVTileC {            // stage C's per-tile arrays
 
 // Kept small: two CTAs per SM plus as much L1 as possible (the carveout is
 // the smallest that fits both CTAs' shared memory).
-struct NVSmem {
+// MAXSEG: the weighted kernel keeps 256 segments (its A-Res buffers follow in
+// dynamic smem and two CTAs per SM must still fit).
+template <int MAXSEG>
+struct NVSmemT {
   union {
     WarpChunk wc[NV_WARPS];  // stage A
     NVTileC tc;              // stage C (tasks never overlap inside a CTA)
   };
-  NVSeg seg[NV_MAXSEG];
+  NVSeg seg[MAXSEG];
   long long ntasks;
   int nseg;
   long long work;
@@ -168,7 +177,8 @@ struct NVWeighted {  // weighted mode only: placed after NVSmem in dynamic share
   int heavy[NV_TC];
 };
 
-__device__ __forceinline__ int nv_find_seg(const NVSmem& sm, long long x) {
+template <class SM>
+__device__ __forceinline__ int nv_find_seg(const SM& sm, long long x) {
   int lo = 0, hi = sm.nseg - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
@@ -192,7 +202,8 @@ __device__ __forceinline__ long long nv_z_tasks(const NVParams& P, long long R) 
 
 // Live segments of super-step s, stage-major in claim order (B, A, C, Z).
 // All threads; ends with __syncthreads.
-__device__ void nv_segments(const NVParams& P, NVSmem& sm, int s) {
+template <class SM>
+__device__ void nv_segments(const NVParams& P, SM& sm, int s) {
   const int tid = threadIdx.x;
   long long T = 0, nt = 0, b = -1;
   int j = 0, l = 0, st = 0, g = 0;
@@ -323,7 +334,8 @@ __device__ __forceinline__ float nv_tau0(const NVParams& P, int k, int32_t v, in
 // Weighted select (A-Res, R6), phase 1 (warp): columns with d <= k take every
 // eligible edge (lane per column); k < d <= NV_DHEAVY are filtered by the whole
 // warp one at a time; heavier columns are queued for the CTA (phase 2).
-__device__ void nv_select_weighted(const NVParams& P, NVSmem& sm, NVWeighted& W, WarpChunk& C,
+template <class SM>
+__device__ void nv_select_weighted(const NVParams& P, SM& sm, NVWeighted& W, WarpChunk& C,
                                    const NVSeg& sg) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int l = sg.l, k = P.k[l];
@@ -369,7 +381,8 @@ __device__ void nv_select_weighted(const NVParams& P, NVSmem& sm, NVWeighted& W,
 }
 
 // Weighted select, phase 2 (whole CTA): the queued heavy columns one by one.
-__device__ void nv_select_heavy(const NVParams& P, NVSmem& sm, NVWeighted& W, const NVSeg& sg) {
+template <class SM>
+__device__ void nv_select_heavy(const NVParams& P, SM& sm, NVWeighted& W, const NVSeg& sg) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int l = sg.l, k = P.k[l];
   const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
@@ -471,6 +484,9 @@ __device__ int nv_gather(const NVParams& P, WarpChunk& C, const NVSeg& sg, long 
     if (f < total && (__ffs(peers) - 1) == lane)
       asm volatile("red.global.or.b32 [%0], %1;" ::"l"((uint32_t*)(S.bm + (u >> 5))),
                    "r"(1u << (u & 31))
+                   : "memory");
+    if (P.use_sum[sg.l] && f < total && (__ffs(peers) - 1) == lane)
+      asm volatile("red.global.or.b32 [%0], %1;" ::"l"(S.sm + (u >> 10)), "r"(1u << ((u >> 5) & 31))
                    : "memory");
   }
   __syncwarp();
@@ -583,14 +599,17 @@ __device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg
       asm volatile("red.global.or.b32 [%0], %1;" ::"l"((uint32_t*)(S.bm + (u >> 5))),
                    "r"(1u << (u & 31))
                    : "memory");
+    if (P.use_sum[sg.l] && f < total && (__ffs(peers) - 1) == lane)
+      asm volatile("red.global.or.b32 [%0], %1;" ::"l"(S.sm + (u >> 10)), "r"(1u << ((u >> 5) & 31))
+                   : "memory");
   }
   __syncwarp();
   return total;
 }
 
 // Stage A tile: 512 columns, one 32-column chunk per warp; the tile's edge count.
-template <bool WEIGHTED>
-__device__ void nv_stage_a(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t) {
+template <bool WEIGHTED, class SM>
+__device__ void nv_stage_a(const NVParams& P, SM& sm, const NVSeg& sg, int t) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long jb = (long long)t * NV_TC + warp * 32;
   const bool has = jb < sg.T;
@@ -626,7 +645,8 @@ __device__ void nv_stage_a(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
 // word gets its in-tile row prefix in its high half.  The segment's last tile
 // scans the tile row counts (-> bx, R) and stage A's tile edge counts (-> tx,
 // E) and publishes the block's shape and the next hop's frontier size.
-__device__ void nv_stage_b(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t,
+template <class SM>
+__device__ void nv_stage_b(const NVParams& P, SM& sm, const NVSeg& sg, int t,
                            unsigned int* segdone) {
   const int l = sg.l;
   const NVStage S = nv_stage(P, sg.j, l, sg.g);
@@ -634,9 +654,11 @@ __device__ void nv_stage_b(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
   const int64_t wb = ((int64_t)t << NV_BT_LOG) + (int64_t)threadIdx.x * NV_BW;
   uint32_t bits[NV_BW];
   int c = 0;
+  // summary hops: only the non-empty words are read (NV_BW = 16 bits of one summary word)
+  const uint32_t smask = P.use_sum[l] ? (wb < P.nw ? (__ldcg(S.sm + (wb >> 5)) >> (wb & 31)) : 0u) : 0xFFFFu;
 #pragma unroll
   for (int i = 0; i < NV_BW; ++i) {
-    bits[i] = wb + i < P.nw ? (uint32_t)__ldcg(S.bm + wb + i) : 0u;
+    bits[i] = wb + i < P.nw && ((smask >> i) & 1u) ? (uint32_t)__ldcg(S.bm + wb + i) : 0u;
     c += __popc(bits[i]);
   }
   int tot;
@@ -689,7 +711,8 @@ __device__ void nv_stage_b(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t
 }
 
 // Stage C: relabel + compaction of one tile of 512 columns.
-__device__ void nv_stage_c(const NVParams& P, NVSmem& sm, const NVSeg& sg, int t) {
+template <class SM>
+__device__ void nv_stage_c(const NVParams& P, SM& sm, const NVSeg& sg, int t) {
   const int l = sg.l, k = P.k[l];
   const NVStage S = nv_stage(P, sg.j, l, sg.g);
   const uint64_t pf = pol_first(), pl = pol_last();
@@ -771,12 +794,18 @@ __device__ void nv_stage_z(const NVParams& P, const NVSeg& sg, int t) {
     for (int i = 0; i < NV_BW; i += 2)
       if (wb + i + 1 < P.nw) *(ulonglong2*)(S.bm + wb + i) = make_ulonglong2(0ull, 0ull);
       else if (wb + i < P.nw) S.bm[wb + i] = 0ull;
+    if (P.use_sum[l] && threadIdx.x < NV_BT / 32 && ((int64_t)t << (NV_BT_LOG - 5)) + threadIdx.x < P.nsw)
+      S.sm[((int64_t)t << (NV_BT_LOG - 5)) + threadIdx.x] = 0u;
     return;
   }
   const int32_t* rows = P.row_map[l] + b * P.batch_size * P.K[l];
   const long long hi = min(R, (long long)(t + 1) * NV_ZR);
   for (long long i = (long long)t * NV_ZR + threadIdx.x; i < hi; i += NV_THREADS)
-    S.bm[__ldcg(rows + i) >> 5] = 0ull;
+  {
+    const uint32_t u = (uint32_t)__ldcg(rows + i);
+    S.bm[u >> 5] = 0ull;
+    if (P.use_sum[l]) S.sm[u >> 10] = 0u;
+  }
 }
 
 // WEIGHTED: A-Res / PASS select (its own instantiation: the uniform kernel
@@ -784,7 +813,8 @@ __device__ void nv_stage_z(const NVParams& P, const NVSeg& sg, int t) {
 template <bool WEIGHTED>
 __global__ void __launch_bounds__(NV_THREADS, 2) nodewise_wave_kernel(NVParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  NVSmem& sm = *reinterpret_cast<NVSmem*>(smem_raw);
+  using SM = NVSmemT<WEIGHTED ? NV_MAXSEG_W : NV_MAXSEG>;
+  SM& sm = *reinterpret_cast<SM*>(smem_raw);
   cg::grid_group grid = cg::this_grid();
   for (int s = 0; s < P.S; ++s) {
     unsigned int* ctr = P.ctr + (int64_t)s * (4 + NV_MAXSEG);
@@ -860,10 +890,13 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   // 16 2.7), <= 4 GB of bitmaps, <= NV_MAXSEG live segments
   {
     const int64_t deep = std::max<int64_t>(1, batch_size * P.K[L - 1]);
-    int64_t wb = std::max<int64_t>(1, (int64_t(16) << 20) / deep);
+    const bool wsel = !replace && bias != GS_W_UNIFORM;  // A-Res: measured best at <= 32 (PASS PD 7.3 ms vs 8.5 at 64)
+    int64_t wb = std::max<int64_t>(1, (int64_t(wsel ? 8 : 16) << 20) / deep);
+    if (wsel) wb = std::min<int64_t>(wb, 32);
     wb = std::min<int64_t>(wb, std::max<int64_t>(1, (int64_t(4) << 30) / (4 * L * P.nw * 8)));
-    wb = std::min<int64_t>(wb, NV_MAXSEG / (4 * L));
-    if (const char* e = getenv("GS_WAVE")) wb = std::max(1, std::min(atoi(e), NV_MAXSEG / (4 * L)));
+    const int maxseg = wsel ? NV_MAXSEG_W : NV_MAXSEG;
+    wb = std::min<int64_t>(wb, maxseg / (4 * L));
+    if (const char* e = getenv("GS_WAVE")) wb = std::max(1, std::min(atoi(e), maxseg / (4 * L)));
     wb = std::min<int64_t>(wb, std::max<int64_t>(1, nbatch));
     P.WB = (int)wb;
   }
@@ -893,7 +926,12 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (blocks buffers)");
 
   // workspace: 4 * L * WB row bitmaps (rotating over groups), then staging
-  const int64_t bm_bytes = a256((int64_t)4 * L * P.WB * P.nw * 8);
+  // hops whose rows are sparse in N (PP-sized graphs) keep a summary bit per
+  // bitmap word, so stage B reads only the non-empty words
+  P.nsw = (P.nw + 31) / 32;
+  for (int l = 0; l < L; ++l) P.use_sum[l] = batch_size * P.K[l] * 8 < P.nw ? 1 : 0;
+  const int64_t sm_off = a256((int64_t)4 * L * P.WB * P.nw * 8);
+  const int64_t bm_bytes = a256(sm_off + (int64_t)4 * L * P.WB * P.nsw * 4);
   int64_t o = bm_bytes;
   for (int l = 0; l < L; ++l) {
     const int64_t slots = batch_size * P.K[l] + 64;
@@ -925,6 +963,7 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   blk->ws_kind_prev = 7;
   P.bm = (unsigned long long*)blk->b_ws.ptr;
   P.stg = (char*)blk->b_ws.ptr + bm_bytes;
+  P.sm = (uint32_t*)((char*)blk->b_ws.ptr + sm_off);
   P.ctr = (unsigned int*)blk->b_sched.ptr;
   P.T = (long long*)((char*)blk->b_sched.ptr + ctr_bytes);
 
@@ -957,7 +996,7 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   // dynamic shared memory: the A-Res candidate buffers only in weighted mode;
   // cooperative grid = every CTA co-resident
   const bool weighted = !replace && bias != GS_W_UNIFORM;
-  const size_t smem = sizeof(NVSmem) + (weighted ? sizeof(NVWeighted) : 0);
+  const size_t smem = weighted ? sizeof(NVSmemT<NV_MAXSEG_W>) + sizeof(NVWeighted) : sizeof(NVSmemT<NV_MAXSEG>);
   static int grid_for[2] = {0, 0};
   int& grid = grid_for[weighted ? 1 : 0];
   void* kfn = weighted ? (void*)nodewise_wave_kernel<true> : (void*)nodewise_wave_kernel<false>;
