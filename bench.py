@@ -157,16 +157,7 @@ def make_graph_dist(name, world, rank, device):
 def _layer_arrays(blocks, l):
     import ctypes
     from paper_conf_sosp_gonglmc0lwl23_b200 import gs
-
-    class LB(ctypes.Structure):
-        _fields_ = [("col_map", ctypes.c_void_p), ("col_capacity", ctypes.c_int64),
-                    ("row_map", ctypes.c_void_p), ("row_capacity", ctypes.c_int64),
-                    ("indptr", ctypes.c_void_p), ("indptr_capacity", ctypes.c_int64),
-                    ("row_local", ctypes.c_void_p), ("eid", ctypes.c_void_p),
-                    ("val", ctypes.c_void_p), ("edge_capacity", ctypes.c_int64),
-                    ("row_prob", ctypes.c_void_p)]
-    lb = LB()
-    gs._lib.gs_blocks_layer.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.POINTER(LB)]
+    lb = gs._LayerBuffers()
     gs._check(gs._lib.gs_blocks_layer(blocks._h, l, ctypes.byref(lb)))
     t = gs._dev_tensor
     d = {"col_map": t(lb.col_map, lb.col_capacity, torch.int32, blocks),
@@ -424,22 +415,23 @@ def run_gpu(args, wl, world, rank, device):
         dist.barrier()
     t_total_ms = sum(times)
 
-    # e2e: the same step through the C ABI with HOST buffers (pinned host
-    # inputs copied in, every output copied back, both inside the timed region)
+    # e2e: the same step through the C ABI with HOST buffers: pinned host
+    # inputs copied in; the sampled blocks packed densely on the device
+    # (gs_blocks_pack), their sizes read, and exactly the sampled data copied
+    # back -- all inside the timed region
     host_in = inputs.cpu().pin_memory()
     dev_in = torch.empty_like(inputs)
-    if kind == "walk":
-        outs = [traces]
-    else:
-        outs = []
-        for l in range(L):
-            la = _layer_arrays(out, l)
-            outs += [la[k2] for k2 in ("row_map", "indptr", "row_local", "eid") if k2 in la]
-        outs.append(out.device_meta())
-    host_out = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in outs]
     h2d = host_in.numel() * host_in.element_size()
-    d2h = sum(t.numel() * t.element_size() for t in host_out)
-    e2e_times = []
+    if kind == "walk":
+        host_tr = torch.empty(traces.shape, dtype=traces.dtype).pin_memory()
+    else:
+        packs = [out.pack(l) for l in range(L)]
+        meta_dev = out.device_meta()
+        host_meta = torch.empty(meta_dev.shape, dtype=meta_dev.dtype).pin_memory()
+        host_tot = torch.empty((L, 3), dtype=torch.int64).pin_memory()
+        host_pk = [{k2: torch.empty(v.shape, dtype=v.dtype).pin_memory() for k2, v in pk.items()
+                    if k2 != "totals"} for pk in packs]
+    e2e_times, d2h_all = [], []
     for i in range(max(2, min(args.steps, 5))):
         flush.zero_()
         torch.cuda.synchronize()
@@ -447,11 +439,26 @@ def run_gpu(args, wl, world, rank, device):
         ev0.record(stream)
         dev_in.copy_(host_in, non_blocking=True)
         step(args.warmup + i, dev_in)
-        for src, dst in zip(outs, host_out):
-            dst.copy_(src, non_blocking=True)
+        if kind == "walk":
+            host_tr.copy_(traces, non_blocking=True)
+            d2h = host_tr.numel() * 4
+        else:
+            for l in range(L):
+                out.pack(l, packs[l], stream=stream)
+                host_tot[l].copy_(packs[l]["totals"], non_blocking=True)
+            host_meta.copy_(meta_dev, non_blocking=True)
+            stream.synchronize()
+            d2h = host_tot.numel() * 8 + host_meta.numel() * 8
+            for l in range(L):
+                ne, ni, nr = (int(x) for x in host_tot[l])
+                for k2, n in (("row_local", ne), ("eid", ne), ("indptr", ni), ("row_map", nr)):
+                    host_pk[l][k2][:n].copy_(packs[l][k2][:n], non_blocking=True)
+                    d2h += n * packs[l][k2].element_size()
         ev1.record(stream)
         ev1.synchronize()
         e2e_times.append(ev0.elapsed_time(ev1))
+        d2h_all.append(d2h)
+    d2h = int(statistics.mean(d2h_all))
     e2e_ms = statistics.mean(e2e_times)
     if world > 1:
         t = torch.tensor([t_total_ms, e2e_ms], dtype=torch.float64, device=device)

@@ -140,6 +140,18 @@ typedef struct gs_layer_buffers {   /* whole-layer device arrays of one layer */
   float* row_prob;    /* [row_capacity] or NULL */
 } gs_layer_buffers;
 gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out);
+
+/* Packs layer `layer` of every batch into dense, batch-ordered DEVICE arrays
+ * (caller-owned, each at least the layer's capacity from gs_blocks_layer):
+ * batch b's edges (row_local, eid), its block indptr (n_cols + 1 entries,
+ * block-relative: starts at 0) and its row_map follow those of batch b - 1.
+ * totals: DEVICE int64[3] <- (edges, indptr entries, rows) of the layer.
+ * Stream-ordered, no host sync: the sampling kernels write every batch into a
+ * fixed padded region; this lets a host copy move only
+ * the sampled data (read `totals` first).  Errors: GS_ERR_INVALID_ARGUMENT
+ * (null pointer, bad layer), GS_ERR_OUT_OF_MEMORY, GS_ERR_CUDA. */
+gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
+                         int64_t* indptr, int32_t* row_map, int64_t* totals, cudaStream_t stream);
 void gs_blocks_destroy(gs_blocks* b);
 
 /* ------------------------------------------------------------------------ */

@@ -490,6 +490,7 @@ void gs_blocks_destroy(gs_blocks* b) {
   b->b_gen.reset(b->al, s);
   b->b_ctr.reset(b->al, s);
   b->b_sched.reset(b->al, s);
+  b->b_pack.reset(b->al, s);
   delete b;
 }
 

@@ -76,7 +76,7 @@ struct gs_blocks {
   gsb::DevBuf b_col[gsb::MAX_LAYERS], b_row[gsb::MAX_LAYERS], b_indptr[gsb::MAX_LAYERS],
       b_rowl[gsb::MAX_LAYERS], b_eid[gsb::MAX_LAYERS], b_val[gsb::MAX_LAYERS],
       b_rprob[gsb::MAX_LAYERS];
-  gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr, b_sched;
+  gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr, b_sched, b_pack;
   std::vector<int64_t> h_meta;
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch

@@ -898,6 +898,8 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
     wb = std::min<int64_t>(wb, maxseg / (4 * L));
     if (const char* e = getenv("GS_WAVE")) wb = std::max(1, std::min(atoi(e), maxseg / (4 * L)));
     wb = std::min<int64_t>(wb, std::max<int64_t>(1, nbatch));
+    // (balancing the groups -- 49+48+48+48 instead of 64+64+64+1 for the PD
+    // epoch -- measured 1.53 ms vs 1.51: the short last group is cheap)
     P.WB = (int)wb;
   }
   P.G = (int)((nbatch + P.WB - 1) / P.WB);

@@ -32,7 +32,7 @@ META_FIELDS = 8
 EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
-           "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_layerwise",
+           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check"]
 
 
@@ -54,6 +54,15 @@ class _GraphInfo(ctypes.Structure):
                 ("weighted", ctypes.c_int), ("sorted", ctypes.c_int),
                 ("max_in_degree", ctypes.c_int64), ("indptr", ctypes.c_void_p),
                 ("indices", ctypes.c_void_p), ("weights", ctypes.c_void_p)]
+
+
+class _LayerBuffers(ctypes.Structure):
+    _fields_ = [("col_map", ctypes.c_void_p), ("col_capacity", ctypes.c_int64),
+                ("row_map", ctypes.c_void_p), ("row_capacity", ctypes.c_int64),
+                ("indptr", ctypes.c_void_p), ("indptr_capacity", ctypes.c_int64),
+                ("row_local", ctypes.c_void_p), ("eid", ctypes.c_void_p),
+                ("val", ctypes.c_void_p), ("edge_capacity", ctypes.c_int64),
+                ("row_prob", ctypes.c_void_p)]
 
 
 _ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
@@ -116,6 +125,8 @@ def load_library(path: str = LIB_PATH):
     L.gs_blocks_shape.argtypes = [vp, ctypes.POINTER(i64), ctypes.POINTER(i32)]
     L.gs_blocks_view.argtypes = [vp, i64, i32, ctypes.POINTER(_BlockView)]
     L.gs_blocks_device_meta.argtypes = [vp, ctypes.POINTER(vp)]
+    L.gs_blocks_layer.argtypes = [vp, i32, ctypes.POINTER(_LayerBuffers)]
+    L.gs_blocks_pack.argtypes = [vp, i32, vp, vp, vp, vp, vp, vp]
     L.gs_blocks_destroy.argtypes = [vp]
     L.gs_blocks_destroy.restype = None
     _lib = L
@@ -258,6 +269,29 @@ class Blocks:
         _check(_lib.gs_blocks_shape(self._h, ctypes.byref(nb), ctypes.byref(nl)))
         t = _dev_tensor(p.value, nb.value * nl.value * META_FIELDS, torch.int64, self)
         return t.view(nb.value, nl.value, META_FIELDS)
+
+    def layer_capacity(self, layer: int) -> dict:
+        """Capacities of layer `layer`'s whole-layer arrays (gs_blocks_layer)."""
+        lb = _LayerBuffers()
+        _check(_lib.gs_blocks_layer(self._h, layer, ctypes.byref(lb)), "gs_blocks_layer")
+        return {"edges": lb.edge_capacity, "indptr": lb.indptr_capacity, "rows": lb.row_capacity}
+
+    def pack(self, layer: int, out: dict = None, stream=None) -> dict:
+        """gs_blocks_pack: layer `layer` of every batch packed densely on the
+        device (batch order).  Returns device tensors (capacity-sized; the used
+        prefix lengths are in `totals` = device int64 [edges, indptr entries, rows])."""
+        if out is None:
+            cap = self.layer_capacity(layer)
+            dev = torch.device("cuda", torch.cuda.current_device())
+            out = {"row_local": torch.empty(cap["edges"], dtype=torch.int32, device=dev),
+                   "eid": torch.empty(cap["edges"], dtype=torch.int64, device=dev),
+                   "indptr": torch.empty(cap["indptr"], dtype=torch.int64, device=dev),
+                   "row_map": torch.empty(cap["rows"], dtype=torch.int32, device=dev),
+                   "totals": torch.empty(3, dtype=torch.int64, device=dev)}
+        _check(_lib.gs_blocks_pack(self._h, layer, _ptr(out["row_local"]), _ptr(out["eid"]),
+                                   _ptr(out["indptr"]), _ptr(out["row_map"]), _ptr(out["totals"]),
+                                   _stream_ptr(stream)), "gs_blocks_pack")
+        return out
 
     def to_host(self) -> list:
         """blocks[batch][layer] -> dict of numpy arrays (tests / e2e)."""

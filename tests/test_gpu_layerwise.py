@@ -101,3 +101,19 @@ def test_ladies_bias_capacity_retry(gs, oracle_lib, ljlike):
     ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [3000, 3000], batch_size=3000, prob_mode=0,
                                       rng_key=2)
     compare_all(out.to_host(), ref, "ladies big")
+
+
+def test_fastgcn_threshold_reuse(gs, oracle_lib, ljlike, monkeypatch, lw_path):
+    """One CTA walks every batch, so from the second batch on the bitmap
+    kernel's rank pass filters against the previous batch's threshold (the
+    fused select); the result must not depend on it."""
+    if lw_path != "bm":
+        pytest.skip("bitmap-kernel path")
+    monkeypatch.setenv("GS_LW_CTAS", "1")
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 11), 512 * 12)
+    for K in (64, 512):
+        out = gs.sample_layerwise(G, seeds.cuda(), [K, K, K], batch_size=512, prob_mode=1, rng_key=K)
+        ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [K, K, K], batch_size=512, prob_mode=1,
+                                          rng_key=K)
+        compare_all(out.to_host(), ref, f"fastgcn one CTA K={K}")

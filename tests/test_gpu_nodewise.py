@@ -136,3 +136,30 @@ def test_shadow(gs, oracle_lib, medium, mode):
                            rng_key=21).to_host()
     ref = oracle_lib.shadow(O, seeds.numpy(), [10, 5], batch_size=256, bias_mode=mode, rng_key=21)
     compare_all(out, [[r] for r in ref], f"shadow {mode}")
+
+
+@pytest.mark.parametrize("kind", ["nodewise", "layerwise"])
+def test_pack_matches_views(gs, medium, kind):
+    """gs_blocks_pack: every batch's block, packed densely in batch order, is
+    exactly its view (indptr block-relative), and `totals` are the sums."""
+    g, G, O = medium
+    seeds = synth.make_seeds(synth.GraphSpec("m", 200_000, 1, False, None, 12), 5000).cuda()
+    if kind == "nodewise":
+        out = gs.sample_neighbors(G, seeds, [7, 3], batch_size=700, rng_key=21)
+    else:
+        out = gs.sample_layerwise(G, seeds, [300, 300], batch_size=700, prob_mode=1, rng_key=21)
+    out.sync()
+    for l in range(2):
+        pk = out.pack(l)
+        torch.cuda.synchronize()
+        tot = pk["totals"].cpu().tolist()
+        e = i = r = 0
+        for b in range(out.num_batches):
+            v = out.view(b, l)
+            ne, nc, nr = v["eid"].numel(), v["indptr"].numel(), v["row_map"].numel()
+            assert torch.equal(pk["row_local"][e:e + ne], v["row_local"])
+            assert torch.equal(pk["eid"][e:e + ne], v["eid"])
+            assert torch.equal(pk["indptr"][i:i + nc], v["indptr"])
+            assert torch.equal(pk["row_map"][r:r + nr], v["row_map"])
+            e, i, r = e + ne, i + nc, r + nr
+        assert tot == [e, i, r]

@@ -7,7 +7,7 @@ d=/tmp/var_$name/a/b; rm -rf /tmp/var_$name; mkdir -p $d /tmp/var_$name/include;
 cp paper_conf_sosp_gonglmc0lwl23_b200/csrc/*.cu paper_conf_sosp_gonglmc0lwl23_b200/csrc/*.cuh paper_conf_sosp_gonglmc0lwl23_b200/csrc/*.h $d/
 cp $ov/* $d/
 objs=""
-for f in capi nodewise_wave shadow layerwise layerwise_bm walk; do
+for f in capi nodewise_wave shadow layerwise layerwise_bm walk pack; do
   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -fmad=false -std=c++17 -Xcompiler -fPIC -I include -c $d/$f.cu -o $d/$f.o &
   objs="$objs $d/$f.o"
 done
