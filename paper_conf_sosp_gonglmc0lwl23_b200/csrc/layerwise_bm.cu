@@ -666,6 +666,20 @@ __global__ void degree_kernel(const int64_t* __restrict__ indptr, int64_t N, int
 
 static int64_t a256(int64_t x) { return (x + 255) & ~int64_t(255); }
 
+// The a0 degree array of a graph (FastGCN), built once on first use.
+gs_status layerwise_degree_array(const gs_graph* g, cudaStream_t stream) {
+  gs_graph* gm = const_cast<gs_graph*>(g);
+  if (gm->deg) return GS_OK;
+  if (!gm->b_deg.ensure(gm->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
+    return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (degree array)");
+  gm->deg = (int32_t*)gm->b_deg.ptr;
+  const int64_t blocks = std::min<int64_t>((g->num_nodes + 255) / 256, 148 * 16);
+  if (g->num_nodes > 0)
+    degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
+  GS_CUDA_TRY(cudaGetLastError());
+  return GS_OK;
+}
+
 // Shared-memory bytes of layerwise_bm_kernel for a graph of N nodes (0: does not fit).
 size_t layerwise_bm_smem(int64_t N, int maxT, int* gw_log_out, int* ng_out, int64_t* n4_out) {
   const int64_t nwords = (N + 31) / 32;
@@ -711,16 +725,11 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
     maxK = std::max(maxK, n_per_layer[l]);
   }
   P.maxT = (int)std::max<int64_t>(batch_size, maxK);
-  gs_graph* gm = const_cast<gs_graph*>(g);
-  if (prob_mode == GS_PROB_DEGREE && !gm->deg) {  // a0 pre-processing, once per graph
-    if (!gm->b_deg.ensure(gm->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
-      return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (degree array)");
-    gm->deg = (int32_t*)gm->b_deg.ptr;
-    const int64_t blocks = std::min<int64_t>((g->num_nodes + 255) / 256, 148 * 16);
-    if (g->num_nodes > 0) degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
-    GS_CUDA_TRY(cudaGetLastError());
+  if (prob_mode == GS_PROB_DEGREE) {
+    const gs_status st = layerwise_degree_array(g, stream);
+    if (st) return st;
   }
-  P.deg = gm->deg;
+  P.deg = g->deg;
   blk->kind = gs_blocks::LAYERWISE;
   blk->num_batches = nbatch;
   blk->num_layers = L;
