@@ -377,12 +377,17 @@ def run_gpu(args, wl, world, rank, device):
 
     def account():
         if kind == "walk":
+            # walk index (walk_kernel): per step one 32-byte sector
+            # holding the 16-byte record of the chosen neighbour + 4 bytes of
+            # trace; per walker the start's indptr pair (32(1+straddle)) and
+            # its trace entry.  Node2Vec's extra trials and membership probes
+            # are not counted (a lower bound).
             nxt = traces[:, 1:]
-            moved = nxt >= 0
-            edges = int(moved.sum())
-            prev = traces[:, :-1].to(torch.int64)
-            straddle = int((((prev & 3) == 3) & moved).sum())
-            return edges * (32 + 32 + 4) + 32 * straddle, edges
+            edges = int((nxt >= 0).sum())
+            st = traces[:, 0].to(torch.int64)
+            walkers = int((st >= 0).sum())
+            straddle = int(((st & 3) == 3).sum())
+            return edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges
         out.sync()
         return _blocks_byte_model(out, g, kind, g["weights"] is not None and wl.get("mode") == 0,
                                   L, weighted_select=kind == "nodewise" and wl.get("bias", 0) != 0)

@@ -214,7 +214,8 @@ gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t n
 /* ------------------------------------------------------------------------ */
 /* Random walks (a5): DeepWalk / Node2Vec.                                   */
 /* ------------------------------------------------------------------------ */
-enum { GS_WALK_FORCE_NODE2VEC = 1 }; /* use the Node2Vec sampler even at p == q == 1 */
+enum { GS_WALK_FORCE_NODE2VEC = 1,  /* use the Node2Vec sampler even at p == q == 1 */
+       GS_WALK_PLAIN_CSC = 2 };     /* walk the plain CSC: do not build / use the walk index */
 /* One walker per start node.  traces: caller-owned device
  * int32 [num_walkers][length + 1]; traces[i][0] = starts[i]; a walker at a
  * node with no in-neighbours stops and the rest of its row is -1 (R13).
@@ -222,7 +223,11 @@ enum { GS_WALK_FORCE_NODE2VEC = 1 }; /* use the Node2Vec sampler even at p == q 
  * Otherwise Node2Vec with bias 1/p (x == prev), 1 (x in column(prev)), 1/q
  * (else), by rejection sampling (R14); needs a sorted graph
  * (GS_ERR_UNSORTED_GRAPH otherwise).  walker_index_base keys the RNG by the
- * global walker index (R4).  p, q > 0; 0 <= length < 2^24. */
+ * global walker index (R4).  p, q > 0; 0 <= length < 2^24.
+ * The first walk on a graph builds a walk index (16 bytes per CSC entry: each
+ * position's neighbour with that neighbour's column range, a0 pre-processing)
+ * when memory allows, so that a step is one dependent random read instead of
+ * two; results are identical either way (GS_WALK_PLAIN_CSC disables it). */
 gs_status gs_random_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
                          int64_t walker_index_base, int length, float p, float q,
                          uint64_t rng_key, uint32_t flags, void* stream, int32_t* traces);

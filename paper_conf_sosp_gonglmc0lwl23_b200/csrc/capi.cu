@@ -93,7 +93,7 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
 gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
                       int64_t walker_base, int length, float p, float q, uint64_t key,
-                      bool node2vec, cudaStream_t stream, int32_t* traces);
+                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces);
 
 // ---------------------------------------------------------------------------
 // a0: CSC validation (indptr monotone and in range, indices in [0, N),
@@ -281,6 +281,7 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_weights.reset(g->al, s);
   g->b_colsum.reset(g->al, s);
   g->b_deg.reset(g->al, s);
+  g->b_walk.reset(g->al, s);
   g->b_err.reset(g->al, s);
   delete g;
 }
@@ -387,7 +388,7 @@ gs_status gs_random_walk(const gs_graph* g, const int32_t* starts, int64_t num_w
   if (n2v && !g->sorted)
     return fail(GS_ERR_UNSORTED_GRAPH, "gs_random_walk: Node2Vec needs ascending CSC columns");
   return launch_walk(g, starts, num_walkers, walker_index_base, length, p, q, rng_key, n2v,
-                     (cudaStream_t)stream_, traces);
+                     (flags & GS_WALK_PLAIN_CSC) != 0, (cudaStream_t)stream_, traces);
 }
 
 gs_status gs_walk_check(const gs_graph* g, void* stream_) {

@@ -60,6 +60,9 @@ struct gs_graph {
   gsb::Allocator al;
   gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_err, b_deg;
   int32_t* deg = nullptr;    // FastGCN a0 pre-processing: in-degree per node (built on first use)
+  gsb::DevBuf b_walk;        // walk index (walk.cu): 16 B per CSC entry, built on the first walk
+  const int4* walk_rec = nullptr;
+  bool walk_index_failed = false;
   int* d_err = nullptr;  // walk error word
 };
 

@@ -264,50 +264,6 @@ __device__ __forceinline__ void nv_cols(const NVParams& P, WarpChunk& C, const N
   d_out = d;
 }
 
-// Uniform select (GraphSAGE Floyd, R5; KGCN replacement, R10), lane per column.
-// (v, d in registers: the Floyd loop stores into C.list, which would force
-// reloads of anything read back from the same shared-memory struct)
-__device__ void nv_select_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg, const int32_t v,
-                                  const int64_t d) {
-  const int lane = threadIdx.x & 31;
-  const int l = sg.l, k = P.k[l];
-  const uint32_t gb = (uint32_t)(P.batch_base + sg.b);
-  int cnt = 0;
-  bool all = false;
-  if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
-    cnt = d > 0 ? k : 0;
-    for (int s = 0; s < cnt; ++s) {
-      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
-      C.list[s][lane] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
-    }
-  } else if (d <= k) {  // GraphSAGE, d <= k: every neighbour (R5)
-    cnt = (int)d;
-    all = true;
-  } else {  // GraphSAGE (R5): Floyd; the list stays sorted (m is always appended)
-    cnt = k;
-    int n = 0;
-    for (int s = 0; s < k; ++s) {
-      const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.core.key);
-      const uint32_t m = (uint32_t)(d - k + s);
-      const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
-      int lo = 0, hi = n;
-      while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (C.list[mid][lane] < t) lo = mid + 1;
-        else hi = mid;
-      }
-      if (lo < n && C.list[lo][lane] == t) {
-        C.list[n][lane] = m;
-      } else {
-        for (int q = n; q > lo; --q) C.list[q][lane] = C.list[q - 1][lane];
-        C.list[lo][lane] = t;
-      }
-      ++n;
-    }
-  }
-  C.cnt_all[lane] = cnt | (all ? (1 << 30) : 0);
-}
-
 // A-Res threshold search state: tau is widened / narrowed geometrically, or
 // bisected once both a too-small and a too-large value are known.
 struct TauSearch {

@@ -17,6 +17,14 @@ def gs():
     return _gs
 
 
+@pytest.fixture(params=["index", "plain"], autouse=True)
+def walk_layout(request, monkeypatch):
+    """Every walk test runs on the walk index (one random 16-byte record per
+    step) and on the plain CSC (GS_WALK_INDEX=0): identical traces."""
+    monkeypatch.setenv("GS_WALK_INDEX", "1" if request.param == "index" else "0")
+    return request.param
+
+
 @pytest.fixture(scope="module")
 def graph(gs, oracle_lib):
     g = synth.small_graph(100_000, 1_500_000, undirected=True, weights=None, seed=9, device="cuda")
