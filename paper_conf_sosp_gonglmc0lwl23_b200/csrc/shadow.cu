@@ -8,9 +8,12 @@
 // a popcount prefix per 256 bits, so the membership test of every streamed
 // edge -- the hot loop, Sum of in-degrees over U per batch -- and the rank of a
 // kept row are shared-memory reads (local or a peer's), never L2/HBM probes.
-// Per batch: mark U -> scan (U ascending) -> count kept edges per column ->
-// scan (CSC indptr, bump-allocated edge range) -> write kept edges in CSC order.
+// Per batch: mark U -> scan (U ascending) -> count kept edges per column,
+// staging each kept edge (row rank, eid) in a per-warp region -> scan (CSC
+// indptr, bump-allocated edge range) -> copy the staged edges to their CSC
+// positions (a column whose edges did not fit the region is streamed again).
 #include <algorithm>
+#include <cstdlib>
 #include <new>
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
@@ -55,6 +58,10 @@ struct SHParams {
   int64_t* meta;
   int* err;
   unsigned int* claim;
+  int64_t* ustart;                  // [b * stride] staged start of a column's kept edges, -1: re-stream
+  int32_t* stage_row;               // [CTA][warp][wcap] kept edges staged by the count pass
+  int64_t* stage_eid;
+  int64_t wcap;
   int64_t bpc;                      // bitmap bits per CTA (multiple of 256)
   uint32_t inv;                     // floor(2^32 / bpc)
 };
@@ -189,13 +196,22 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     }
     __threadfence();
     cl.sync();
-    // ---- count kept edges per column (this CTA's share of U) ----
+    // ---- count kept edges per column (this CTA's share of U), staging every
+    // kept edge (row rank, eid) in this warp's private region so that the
+    // emit below is a copy, not a second stream of the columns ----
     const long long c_lo = nU * rank / CS, c_hi = nU * (rank + 1) / CS;
     int32_t* ucnt = P.ucnt + b * P.stride;
+    int64_t* ustart = P.ustart + b * P.stride;
+    const int64_t wreg = ((int64_t)blockIdx.x * SH_WARPS + warp) * P.wcap;
+    int32_t* wst_r = P.stage_row + wreg;
+    int64_t* wst_e = P.stage_eid + wreg;
+    long long wfill = 0;
     for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
       const int32_t v = __ldcg(U + c);
       const int64_t o = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - o;
       int cnt = 0;
+      const long long start = wfill;
+      bool staged = true;
       for (int64_t i0 = 0; i0 < d; i0 += 32 * SH_ILP) {  // SH_ILP loads, then tests, in flight
         uint32_t u[SH_ILP];
 #pragma unroll
@@ -203,11 +219,30 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
           const int64_t i = i0 + q * 32 + lane;
           u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
         }
+        bool m[SH_ILP];
 #pragma unroll
-        for (int q = 0; q < SH_ILP; ++q)
-          cnt += __popc(__ballot_sync(0xffffffffu, u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q])));
+        for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q]);
+#pragma unroll
+        for (int q = 0; q < SH_ILP; ++q) {
+          const uint32_t bal = __ballot_sync(0xffffffffu, m[q]);
+          const int n = __popc(bal);
+          cnt += n;
+          if (staged && wfill + n > P.wcap) staged = false;  // this column is re-streamed below
+          if (staged) {
+            if (m[q]) {
+              const long long idx = wfill + __popc(bal & ((1u << lane) - 1u));
+              wst_r[idx] = (int32_t)sh_rank(cl, bm, gp, off8, ss, bpc32, inv, u[q]);
+              wst_e[idx] = o + i0 + q * 32 + lane;
+            }
+            wfill += n;
+          }
+        }
       }
-      if (lane == 0) ucnt[c] = cnt;
+      if (!staged) wfill = start;
+      if (lane == 0) {
+        ucnt[c] = cnt;
+        ustart[c] = staged ? start : -1;
+      }
     }
     __threadfence();
     cl.sync();
@@ -246,9 +281,21 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       m[5] = b * P.stride + b; m[6] = fits ? eoff : 0; m[7] = 0;
       if (!fits) atomicOr(P.err, ERR_CAPACITY);
     }
-    // ---- write kept edges in CSC order ----
+    // ---- write kept edges in CSC order: a copy of the staged edges (the
+    // same warp staged this column); columns that did not fit re-stream ----
     if (fits) {
       for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
+        const long long st = __ldcg(ustart + c);
+        if (st >= 0) {
+          const long long p0 = __ldcg(ucnt + c);
+          const long long n = (c + 1 < c_hi ? (long long)__ldcg(ucnt + c + 1) : ss.etotal) - p0;
+          const long long dst = eoff + ebase + p0;
+          for (long long i = lane; i < n; i += 32) {
+            sth(P.row_local + dst + i, wst_r[st + i], pf);
+            sth(P.eid + dst + i, wst_e[st + i], pf);
+          }
+          continue;
+        }
         const int32_t v = __ldcg(U + c);
         const int64_t o = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - o;
         long long pos = eoff + ebase + __ldcg(ucnt + c);
@@ -391,6 +438,20 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   GS_CUDA_TRY(cudaOccupancyMaxActiveClusters(&nclusters, (void*)shadow_induce_kernel, &cfg));
   nclusters = (int)std::max<int64_t>(1, std::min<int64_t>(nclusters, nbatch));
   cfg.gridDim = dim3((unsigned)(nclusters * CS));
+  // staging of kept edges: a fixed region per warp (columns that do not fit
+  // fall back to a second stream), then the per-column staged starts
+  P.wcap = int64_t(1) << 17;
+  if (const char* e = getenv("GS_SH_WCAP")) P.wcap = std::max<int64_t>(1, atoll(e));  // tests: force re-streams
+  {
+    const int64_t nw = (int64_t)nclusters * CS * SH_WARPS;
+    const int64_t o_e = ((nw * P.wcap * 4) + 255) & ~int64_t(255);
+    const int64_t o_s = o_e + nw * P.wcap * 8;
+    if (!blk->b_ws.ensure(al, (size_t)(o_s + std::max<int64_t>(nodes, 1) * 8), stream))
+      return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (ShaDow staging)");
+    P.stage_row = (int32_t*)blk->b_ws.ptr;
+    P.stage_eid = (int64_t*)((char*)blk->b_ws.ptr + o_e);
+    P.ustart = (int64_t*)((char*)blk->b_ws.ptr + o_s);
+  }
   GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, shadow_induce_kernel, P));
   return GS_OK;
 }
