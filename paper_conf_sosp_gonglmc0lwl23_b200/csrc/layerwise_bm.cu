@@ -50,6 +50,7 @@ constexpr int LB_CAP = 4096;        // A-Res candidate buffer (select), >= max K
 constexpr int LB_HS = 8192;         // hash of S (aliases the candidate buffer)
 constexpr int LB_ILP = 4;           // flat edges per thread in flight
 constexpr int LB_MAX_K = 4096;
+constexpr int LB_SCAP = 512;        // kept edges a warp stages in L5a (more: L5b streams again)
 
 struct LBParams {
   const int64_t* indptr;
@@ -79,6 +80,11 @@ struct LBParams {
   int64_t n4;                       // uint4 per bitmap (a multiple of GW / 4)
   double* acc;                      // [CTA][acc_cap] b(u) by rank (zero between uses)
   int64_t acc_cap;
+  int64_t* stg_pos;                 // [CTA][warp][LB_SCAP] kept edges staged by L5a: position,
+  int32_t* stg_lid;                 //   local row, column, a = w / p(u)
+  int32_t* stg_col;
+  float* stg_a;
+  int scap;                         // staged kept edges per warp (<= LB_SCAP)
   int gw_log;                       // log2 words per rank group (>= 2)
   int ng;                           // rank groups per bitmap
   int maxT;
@@ -556,6 +562,13 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       // ---- L5a: per column kept count and c_j = sum_fp64 a (a = w / p(u)),
       // per warp kept count (the warp's offset in the CSC emit order) ----
       int wkept = 0;
+      const int64_t sreg = ((int64_t)blockIdx.x * LB_WARPS + (threadIdx.x >> 5)) * LB_SCAP;
+      int64_t* stg_pos = P.stg_pos + sreg;
+      int32_t* stg_lid = P.stg_lid + sreg;
+      int32_t* stg_col = P.stg_col + sreg;
+      float* stg_a = P.stg_a + sreg;
+      if (threadIdx.x == 0) sh.misc[7] = 0;
+      __syncthreads();
       {
         LBStream st(nflat);
         for (int64_t e0 = st.beg; e0 < st.end && nsel > 0; e0 += 32 * LB_ILP) {
@@ -577,16 +590,26 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
 #pragma unroll
           for (int q = 0; q < LB_ILP; ++q) {
             const int lid = u[q] == 0xFFFFFFFFu ? -1 : lb_lookup(s_hk, s_hv, u[q]);
-            wkept += __popc(__ballot_sync(0xffffffffu, lid >= 0));
-            if (lid < 0) continue;
-            const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
-            const float p = __uint_as_float((uint32_t)s_sel[lid]);
-            atomicAdd(&s_cnt[c[q]], 1);
-            atomicAdd(&s_cs[c[q]], (double)__fdiv_rn(w, p));
+            const unsigned bal = __ballot_sync(0xffffffffu, lid >= 0);
+            if (lid >= 0) {
+              const float w = P.weights ? __ldg(P.weights + pos[q]) : 1.0f;
+              const float a = __fdiv_rn(w, __uint_as_float((uint32_t)s_sel[lid]));
+              atomicAdd(&s_cnt[c[q]], 1);
+              atomicAdd(&s_cs[c[q]], (double)a);
+              const int idx = wkept + __popc(bal & ((1u << lane) - 1u));
+              if (idx < P.scap) {
+                stg_pos[idx] = pos[q];
+                stg_lid[idx] = lid;
+                stg_col[idx] = c[q];
+                stg_a[idx] = a;
+              }
+            }
+            wkept += __popc(bal);
           }
         }
       }
       if (lane == 0) sh.wtot[threadIdx.x >> 5] = wkept;
+      if (lane == 0 && wkept > P.scap) sh.misc[7] = 1;  // some warp streams again in L5b
       __syncthreads();
       if (threadIdx.x < 32) {  // warps' exclusive offsets in the emit order
         const int v = sh.wtot[lane];
@@ -610,7 +633,14 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
 
       // ---- L5b: emit in CSC order (the flat order is column-major with
       // ascending positions; warps own contiguous flat ranges in order) ----
-      if (fits && E > 0) {
+      if (fits && E > 0 && !sh.misc[7]) {  // every warp's kept edges are staged: copy them
+        const int64_t o = ebase + sh.wtot[threadIdx.x >> 5];
+        for (int i = lane; i < wkept; i += 32) {
+          P.row_local[l][o + i] = stg_lid[i];
+          P.eid[l][o + i] = stg_pos[i];
+          P.val[l][o + i] = __fdiv_rn(stg_a[i], (float)s_cs[stg_col[i]]);
+        }
+      } else if (fits && E > 0) {
         LBStream st(nflat);
         int64_t o = ebase + sh.wtot[threadIdx.x >> 5];
         for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
@@ -768,7 +798,8 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.acc_cap = prob_mode == GS_PROB_DEGREE ? 0 : std::max<int64_t>(int64_t(1) << 15, blk->lw_tab_hint);
   const int64_t bm_bytes = a256(n4 * 16);
   const int64_t acc_bytes = a256(P.acc_cap * 8);
-  const int64_t stride = bm_bytes + acc_bytes;
+  const int64_t stg_bytes = a256((int64_t)LB_WARPS * LB_SCAP * (8 + 4 + 4 + 4));
+  const int64_t stride = bm_bytes + acc_bytes + stg_bytes;
   const size_t ws_bytes = (size_t)stride * nctas;
   const bool grow = blk->b_ws.bytes < ws_bytes;
   if (!blk->b_ws.ensure(al, ws_bytes, stream))
@@ -780,6 +811,16 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   // bitmaps of every CTA first, then the b(u) arrays
   P.bm = (uint32_t*)blk->b_ws.ptr;
   P.acc = prob_mode == GS_PROB_DEGREE ? nullptr : (double*)((char*)blk->b_ws.ptr + bm_bytes * nctas);
+  P.scap = LB_SCAP;
+  if (const char* e = getenv("GS_LW_SCAP")) P.scap = std::max(0, std::min(atoi(e), LB_SCAP));  // tests
+  {
+    char* sb = (char*)blk->b_ws.ptr + (bm_bytes + acc_bytes) * nctas;
+    const int64_t ne = (int64_t)nctas * LB_WARPS * LB_SCAP;
+    P.stg_pos = (int64_t*)sb;
+    P.stg_lid = (int32_t*)(sb + ne * 8);
+    P.stg_col = (int32_t*)(sb + ne * 12);
+    P.stg_a = (float*)(sb + ne * 16);
+  }
   P.col0 = (int32_t*)blk->b_col[0].ptr;
   for (int l = 0; l < L; ++l) {
     P.row_map[l] = (int32_t*)blk->b_row[l].ptr;

@@ -290,9 +290,25 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
           const long long p0 = __ldcg(ucnt + c);
           const long long n = (c + 1 < c_hi ? (long long)__ldcg(ucnt + c + 1) : ss.etotal) - p0;
           const long long dst = eoff + ebase + p0;
-          for (long long i = lane; i < n; i += 32) {
-            sth(P.row_local + dst + i, wst_r[st + i], pf);
-            sth(P.eid + dst + i, wst_e[st + i], pf);
+          for (long long i0 = lane; i0 < n; i0 += 32 * SH_ILP) {  // SH_ILP loads in flight
+            int32_t r[SH_ILP];
+            int64_t e[SH_ILP];
+#pragma unroll
+            for (int q = 0; q < SH_ILP; ++q) {
+              const long long i = i0 + 32 * q;
+              if (i < n) {
+                r[q] = __ldcs(wst_r + st + i);
+                e[q] = __ldcs(wst_e + st + i);
+              }
+            }
+#pragma unroll
+            for (int q = 0; q < SH_ILP; ++q) {
+              const long long i = i0 + 32 * q;
+              if (i < n) {
+                sth(P.row_local + dst + i, r[q], pf);
+                sth(P.eid + dst + i, e[q], pf);
+              }
+            }
           }
           continue;
         }

@@ -117,3 +117,19 @@ def test_fastgcn_threshold_reuse(gs, oracle_lib, ljlike, monkeypatch, lw_path):
         ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [K, K, K], batch_size=512, prob_mode=1,
                                           rng_key=K)
         compare_all(out.to_host(), ref, f"fastgcn one CTA K={K}")
+
+
+def test_fastgcn_emit_restream(gs, oracle_lib, ljlike, monkeypatch, lw_path):
+    """The bitmap kernel copies the kept edges its L5a pass staged; with a
+    staging capacity of 2 edges per warp every batch-layer takes the
+    re-stream emit instead -- same blocks."""
+    if lw_path != "bm":
+        pytest.skip("bitmap-kernel path")
+    monkeypatch.setenv("GS_LW_SCAP", "2")
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 14), 2048)
+    for mode in (1, 0):
+        out = gs.sample_layerwise(G, seeds.cuda(), [512, 512], batch_size=512, prob_mode=mode, rng_key=5)
+        ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [512, 512], batch_size=512, prob_mode=mode,
+                                          rng_key=5)
+        compare_all(out.to_host(), ref, f"restream emit mode {mode}")
