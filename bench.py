@@ -184,10 +184,13 @@ def _blocks_byte_model(blocks, g, kind, weighted, L, weighted_select=False):
     shadow: per U node the whole column streamed once (4 + 32(1+straddle) +
       32 secs(off, d)) + 12 per induced edge + 4 per node.
     layer-wise: every frontier column streamed twice (indices, + weights for
-      LADIES) + 32(1+straddle) + 4; per block edge 16; per row 8."""
+      LADIES) + 32(1+straddle) + 4; per block edge 16; per row 8.
+    Also returns the number of those 32-byte sectors that are RANDOM accesses
+    (indptr pairs, sampled positions, the first sector of a streamed column):
+    on this B200 each moves a 128-byte HBM line (the line model)."""
     indptr = g["indptr"]
     meta = blocks.device_meta()
-    total, edges = 0, 0
+    total, edges, rnd = 0, 0, 0
     for l in range(L):
         view = _layer_arrays(blocks, l)
         m = meta[:, l, :].cpu()
@@ -215,14 +218,18 @@ def _blocks_byte_model(blocks, g, kind, weighted, L, weighted_select=False):
                 cid = torch.repeat_interleave(torch.arange(cnt.numel(), device=cnt.device), cnt)
                 sec += torch.unique(cid * (1 << 40) + (eids >> 3)).numel()
             total += ncols * 12 + 32 * (ncols + straddle) + 32 * sec
+            rnd += ncols + straddle + sec
             if weighted_select:  # A-Res streams every weight of the column
                 total += 32 * int(_secs(off, d).sum())
+                rnd += int((d > 0).sum())
         elif kind == "shadow":
             total += ncols * 4 + 32 * (ncols + straddle) + 32 * int(_secs(off, d).sum())
+            rnd += ncols + straddle + int((d > 0).sum())
         else:
             s = int(_secs(off, d).sum())
             total += 2 * (ncols * 4 + 32 * (ncols + straddle) + 32 * s * (2 if weighted else 1))
-    return total, edges
+            rnd += 2 * (ncols + straddle + int((d > 0).sum()) * (2 if weighted else 1))
+    return total, edges, rnd
 
 
 # ---------------------------------------------------------------------------
@@ -387,7 +394,8 @@ def run_gpu(args, wl, world, rank, device):
             st = traces[:, 0].to(torch.int64)
             walkers = int((st >= 0).sum())
             straddle = int(((st & 3) == 3).sum())
-            return edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges
+            return (edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges,
+                    edges + walkers + straddle)
         out.sync()
         return _blocks_byte_model(out, g, kind, g["weights"] is not None and wl.get("mode") == 0,
                                   L, weighted_select=kind == "nodewise" and wl.get("bias", 0) != 0)
@@ -399,7 +407,7 @@ def run_gpu(args, wl, world, rank, device):
     if kind != "walk":
         out.sync()
     torch.cuda.synchronize()
-    times, edges, model_bytes = [], 0, 0
+    times, edges, model_bytes, rnd_secs = [], 0, 0, 0
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -412,9 +420,10 @@ def run_gpu(args, wl, world, rank, device):
             ev1.record(stream)
             ev1.synchronize()
             times.append(ev0.elapsed_time(ev1))
-            mb, e = account()
+            mb, e, rs = account()
             model_bytes += mb
             edges += e
+            rnd_secs += rs
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -477,11 +486,14 @@ def run_gpu(args, wl, world, rank, device):
     peak, peak_src = measured_peak_hbm()
     bytes_per_launch = model_bytes / args.steps  # this rank, one launch = one step
     achieved = bytes_per_launch / (statistics.mean(times) / 1000.0) / 1e9
+    line_bytes = (model_bytes + 96 * rnd_secs) / args.steps  # random 32-B sectors as 128-B lines
+    line_achieved = line_bytes / (statistics.mean(times) / 1000.0) / 1e9
     return {"value": edges_all / (t_total_ms / 1000.0), "ms_per_step": t_total_ms / args.steps,
             "edges_per_step": edges_all / args.steps,
             "e2e_value": (edges / args.steps) * world / (e2e_ms / 1000.0), "h2d": h2d, "d2h": d2h,
             "achieved": achieved, "peak": peak, "peak_src": peak_src,
-            "bytes_per_launch": bytes_per_launch, "clocks": clk.summary(), "gen_s": gen_s,
+            "bytes_per_launch": bytes_per_launch, "line_bytes": line_bytes,
+            "line_achieved": line_achieved, "clocks": clk.summary(), "gen_s": gen_s,
             "units": nunits, "graph": g, "inputs": inputs}
 
 
@@ -544,7 +556,13 @@ def main():
                          "kernel": KERNEL_OF[kind] + " (1 launch = 1 step)",
                          "algorithmic_bytes_per_launch": r["bytes_per_launch"],
                          "random_sector_ceiling_gbs": RANDOM_SECTOR_GBS,
-                         "frac_of_random_sector_ceiling": r["achieved"] / RANDOM_SECTOR_GBS},
+                         "frac_of_random_sector_ceiling": r["achieved"] / RANDOM_SECTOR_GBS,
+                         "line_model": {
+                             "bytes_per_launch": r["line_bytes"], "achieved": r["line_achieved"],
+                             "frac": r["line_achieved"] / r["peak"],
+                             "note": "the same accesses with every random 32-B sector counted as "
+                                     "the 128-B HBM line this B200 moves per random access "
+                                     "(profiles/r01_random_access_probe.md)"}},
             "e2e": {"value": r["e2e_value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d"],
                     "d2h_bytes_per_step": r["d2h"]},
             "gpu_launches": args.steps * (2 if kind == "shadow" else 1),
