@@ -71,6 +71,7 @@ def lib():
                                            ctypes.POINTER(vp)]
         L.gso_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, i32,
                                  ctypes.POINTER(vp)]
+        L.gso_saint_rw.argtypes = [vp, vp, i64, i64, i64, i32, u64, i32, ctypes.POINTER(vp)]
         L.gso_random_walk.argtypes = [vp, vp, i64, i64, i32, ctypes.c_float, ctypes.c_float,
                                       u64, i32, i32, vp]
         L.gso_result_num_batches.argtypes = [vp]
@@ -199,6 +200,20 @@ def shadow(g: Graph, seeds, fanouts, batch_size=None, batch_index_base=0, bias_m
                           len(f), bias_mode, rng_key, num_threads, ctypes.byref(res))
     if st:
         raise OracleError(st, "gso_shadow")
+    return [blocks[0] for blocks in _collect(res)]
+
+
+def saint_rw(g: Graph, roots, walk_length, batch_size=None, batch_index_base=0, rng_key=0,
+             num_threads=0):
+    """GraphSAINT-RW (Table 2; DESIGN R26): DeepWalk walks from the roots,
+    then per batch the subgraph induced on the visited nodes (one block per batch)."""
+    s = _seeds(roots)
+    bs = batch_size or max(1, len(s))
+    res = ctypes.c_void_p()
+    st = lib().gso_saint_rw(g.ptr, s.ctypes.data, len(s), bs, batch_index_base, walk_length,
+                            rng_key, num_threads, ctypes.byref(res))
+    if st:
+        raise OracleError(st, "gso_saint_rw")
     return [blocks[0] for blocks in _collect(res)]
 
 

@@ -375,6 +375,30 @@ int gso_sample_layerwise(const gso_graph* g, const int32_t* seeds, int64_t num_s
   return GSO_OK;
 }
 
+// Induce (R12): U = unique(nodes) in ascending order, then
+// every edge u->v of A with u, v in U, columns in U order, CSC order inside.
+static Block induce(const Graph& gg, std::vector<int32_t> all) {
+  Block ind;
+  std::sort(all.begin(), all.end());
+  all.erase(std::unique(all.begin(), all.end()), all.end());
+  ind.row_map = all;
+  std::unordered_map<int32_t, int32_t> local;
+  for (size_t i = 0; i < all.size(); ++i) local[all[i]] = (int32_t)i;
+  ind.col_map = ind.row_map;
+  ind.indptr.push_back(0);
+  for (int32_t v : ind.col_map) {
+    int64_t off = gg.off(v);
+    for (int64_t i = 0; i < gg.deg(v); ++i) {
+      auto it = local.find(gg.indices[off + i]);
+      if (it == local.end()) continue;
+      ind.row_local.push_back(it->second);
+      ind.eid.push_back(off + i);
+    }
+    ind.indptr.push_back((int64_t)ind.eid.size());
+  }
+  return ind;
+}
+
 int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int64_t batch_size,
                int64_t batch_index_base, const int32_t* fanouts, int num_layers, int bias_mode,
                uint64_t rng_key, int num_threads, gso_result** out) {
@@ -399,25 +423,7 @@ int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int6
       frontier = blk.row_map;
       all.insert(all.end(), blk.row_map.begin(), blk.row_map.end());
     }
-    Block ind;
-    std::sort(all.begin(), all.end());
-    all.erase(std::unique(all.begin(), all.end()), all.end());
-    ind.row_map = all;
-    std::unordered_map<int32_t, int32_t> local;
-    for (size_t i = 0; i < all.size(); ++i) local[all[i]] = (int32_t)i;
-    ind.col_map = ind.row_map;
-    ind.indptr.push_back(0);
-    // Induce: every edge u->v of A with u, v in U, CSC order.
-    for (int32_t v : ind.col_map) {
-      int64_t off = gg.off(v);
-      for (int64_t i = 0; i < gg.deg(v); ++i) {
-        auto it = local.find(gg.indices[off + i]);
-        if (it == local.end()) continue;
-        ind.row_local.push_back(it->second);
-        ind.eid.push_back(off + i);
-      }
-      ind.indptr.push_back((int64_t)ind.eid.size());
-    }
+    Block ind = induce(gg, std::move(all));
     r->blocks[(size_t)b] = std::move(ind);
   }
   *out = r;
@@ -506,3 +512,36 @@ int gso_result_view(const gso_result* r, int64_t batch, int layer, gso_block_vie
 void gso_result_free(gso_result* r) { delete r; }
 
 }  // extern "C"
+
+int gso_saint_rw(const gso_graph* g, const int32_t* roots, int64_t num_roots, int64_t batch_size,
+                 int64_t batch_index_base, int walk_length, uint64_t rng_key, int num_threads,
+                 gso_result** out) {
+  if (!g || !out || (!roots && num_roots > 0) || num_roots < 0 || batch_size <= 0 ||
+      batch_index_base < 0 || walk_length < 0)
+    return GSO_ERR_INVALID_ARGUMENT;
+  Graph gg{g->num_nodes, g->num_edges, g->indptr, g->indices, g->weights};
+  if (!frontier_in_range(gg, roots, num_roots)) return GSO_ERR_INDEX_OUT_OF_RANGE;
+  // GraphSAINT-RW (Table 2; R26): a DeepWalk walk from every root,
+  // keyed by the global walker index (batch_index_base * batch_size + i) ...
+  const int64_t L1 = (int64_t)walk_length + 1;
+  std::vector<int32_t> traces((size_t)(num_roots * L1));
+  int st = gso_random_walk(g, roots, num_roots, batch_index_base * batch_size, walk_length, 1.0f,
+                           1.0f, rng_key, 0, num_threads, traces.data());
+  if (st) return st;
+  gso_result* r = new gso_result();
+  r->num_batches = (num_roots + batch_size - 1) / batch_size;
+  r->num_layers = 1;
+  r->blocks.resize((size_t)r->num_batches);
+  set_threads(num_threads);
+  // ... then per batch the subgraph induced on the nodes its walks visited.
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t b = 0; b < r->num_batches; ++b) {
+    int64_t lo = b * batch_size, hi = std::min(num_roots, lo + batch_size);
+    std::vector<int32_t> all;
+    for (int64_t i = lo * L1; i < hi * L1; ++i)
+      if (traces[(size_t)i] >= 0) all.push_back(traces[(size_t)i]);  // -1: after a dead end (R13)
+    r->blocks[(size_t)b] = induce(gg, std::move(all));
+  }
+  *out = r;
+  return GSO_OK;
+}

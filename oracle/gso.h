@@ -14,7 +14,8 @@
  *              collective_sample (layer-wise),
  *              random walks (DeepWalk P:75, Node2Vec P:82)
  *   - Finalize row()/column() + relabel/compaction,
- *              ShaDow induced subgraph
+ *              ShaDow induced subgraph,
+ *              GraphSAINT-RW walk + induce
  * The paper does not fix the sampling algorithms, the RNG or the output order;
  * the readings used here are DESIGN.md section "Readings" (R1..R25), which
  * follow SURVEY.md section 8(c).  Every random draw is Philox4x32-10 keyed by
@@ -96,6 +97,14 @@ int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds,
                int64_t batch_size, int64_t batch_index_base,
                const int32_t* fanouts, int num_layers, int bias_mode,
                uint64_t rng_key, int num_threads, gso_result** out);
+
+/* GraphSAINT-RW (Table 2; R26): a DeepWalk walk of walk_length steps
+ * from every root (global walker index batch_index_base * batch_size + i),
+ * then per batch of batch_size roots the subgraph induced on the visited nodes
+ * (as ShaDow: U ascending, one block per batch). */
+int gso_saint_rw(const gso_graph* g, const int32_t* roots, int64_t num_roots, int64_t batch_size,
+                 int64_t batch_index_base, int walk_length, uint64_t rng_key, int num_threads,
+                 gso_result** out);
 
 /* DeepWalk (p == q == 1 and !force_node2vec) / Node2Vec random walks.
  * traces: caller-owned int32 [num_walkers][length+1], -1 after a dead end. */

@@ -130,3 +130,71 @@ def test_shadow_brute_force(oracle_lib, tiny, bias_mode):
             lo, hi = blk["indptr"][c], blk["indptr"][c + 1]
             assert np.all((blk["eid"][lo:hi] >= ip[v]) & (blk["eid"][lo:hi] < ip[v + 1]))
         assert np.all(np.array(U)[blk["row_local"]] == ix[blk["eid"]])
+
+
+# ---- GraphSAINT-RW (Table 2; DESIGN R26): walk, then induce on the visited nodes ----
+
+def test_saint_rw_visited_set_law(oracle_lib):
+    """One root per batch on the 5-node graph: U's law is the DeepWalk path law
+    (prod 1/deg) pushed through path -> set of visited nodes; every block's edges
+    are exactly {u -> v in E : u, v in U} read off the column lists."""
+    ip, ix, _ = csc_from_columns(5, WALK5)
+    og = oracle_lib.Graph(ip, ix)
+    n = 20_000
+    blocks = oracle_lib.saint_rw(og, np.zeros(n, np.int32), 3, batch_size=1, rng_key=77)
+    assert len(blocks) == n
+    law = Counter()
+    for path, p in path_law(WALK5, 0, 3).items():
+        law[tuple(sorted(set(x for x in path if x >= 0)))] += p
+    cnt = Counter(tuple(b["row_map"].tolist()) for b in blocks)
+    assert chi_square_p(cnt, dict(law), n) > 1e-3
+    edges = {(u, v) for v, col in WALK5.items() for u, _ in col}
+    for b in blocks[:500]:
+        U = b["row_map"].tolist()
+        assert b["col_map"].tolist() == U
+        got = {(U[r], U[c]) for c in range(len(U))
+               for r in b["row_local"][b["indptr"][c]:b["indptr"][c + 1]].tolist()}
+        assert got == {(u, v) for (u, v) in edges if u in U and v in U}
+
+
+def test_saint_rw_special_cases(oracle_lib):
+    # walk_length 0: U = the batch's distinct roots; complete digraph K_6:
+    # the induced block has |U| (|U| - 1) edges
+    n = 6
+    ip, ix, _ = csc_from_columns(n, {v: [(u, 1.0) for u in range(n) if u != v] for v in range(n)})
+    og = oracle_lib.Graph(ip, ix)
+    roots = np.array([4, 1, 4, 0, 5, 5], np.int32)
+    blocks = oracle_lib.saint_rw(og, roots, 0, batch_size=3)
+    assert [b["row_map"].tolist() for b in blocks] == [[1, 4], [0, 5]]
+    assert [len(b["eid"]) for b in blocks] == [2, 2]
+    # walks on K_6 never stop: U covers every visited node, edges |U|(|U|-1)
+    blocks = oracle_lib.saint_rw(og, roots, 4, batch_size=2, rng_key=9)
+    for b in blocks:
+        k = len(b["row_map"])
+        assert 1 <= k <= 2 * 5 and len(b["eid"]) == k * (k - 1)
+    # a root with no in-neighbours: its walk stops at once (R13)
+    ip, ix, _ = csc_from_columns(5, WALK5)
+    blocks = oracle_lib.saint_rw(oracle_lib.Graph(ip, ix), np.array([4], np.int32), 5)
+    assert blocks[0]["row_map"].tolist() == [4] and len(blocks[0]["eid"]) == 0
+
+
+def test_saint_rw_brute_force_tiny(oracle_lib, tiny):
+    roots = synth.make_seeds("tiny", 600).numpy()
+    bs, L = 200, 4
+    blocks = oracle_lib.saint_rw(tiny, roots, L, batch_size=bs, rng_key=12)
+    tr = oracle_lib.random_walk(tiny, roots, L, rng_key=12)   # DeepWalk, global walker ids
+    ip, ix = tiny.indptr, tiny.indices
+    for b, blk in enumerate(blocks):
+        t = tr[b * bs:(b + 1) * bs].ravel()
+        U = sorted(set(t[t >= 0].tolist()))
+        assert blk["row_map"].tolist() == U
+        Uset = set(U)
+        want = [e for v in U for e in range(ip[v], ip[v + 1]) if ix[e] in Uset]
+        assert blk["eid"].tolist() == want   # CSC order: columns in U order, positions ascending
+        assert np.all(np.array(U)[blk["row_local"]] == ix[blk["eid"]])
+        assert np.all(np.diff(blk["indptr"]) >= 0) and blk["indptr"][-1] == len(want)
+    # global batch index keying: batch 2 alone, based at 2, is the same block
+    part = oracle_lib.saint_rw(tiny, roots[2 * bs:], L, batch_size=bs, batch_index_base=2,
+                               rng_key=12)
+    for k in ["row_map", "indptr", "row_local", "eid"]:
+        assert np.array_equal(part[0][k], blocks[2][k])
