@@ -59,6 +59,9 @@ WORKLOADS = {
                     desc="GraphSAGE [15,10,5] weighted A-Res, Papers100M-shaped"),
     "shadow_pd": dict(kind="shadow", graph="PD", fanouts=[10, 5], batch=1024, seeds=196_615,
                       bias=0, desc="ShaDow [10,5] uniform + induce, PD-shaped"),
+    "saint_pd": dict(kind="saint", graph="PD", walk_length=2, batch=3000, seeds=None,
+                     desc="GraphSAINT-RW 3000 roots x walk length 2 + induce per subgraph, every "
+                          "node a root once per epoch (817 subgraphs), PD-shaped"),
     "ladies_lj": dict(kind="layerwise", graph="LJ", n_per_layer=[512, 512, 512], batch=512,
                       seeds=None, mode=0, desc="LADIES 512x3, LJ-shaped, all nodes as seeds"),
     "fastgcn_lj": dict(kind="layerwise", graph="LJ", n_per_layer=[512, 512, 512], batch=512,
@@ -263,6 +266,9 @@ def oracle_rate(g, inputs, wl, budget_s=15.0):
             return oracle.sample_neighbors(O, s[:nbat * bs], wl["fanouts"], batch_size=bs,
                                            replace=wl["replace"], bias_mode=wl["bias"], rng_key=1,
                                            num_threads=threads)
+        if kind == "saint":
+            return [[x] for x in oracle.saint_rw(O, s[:nbat * bs], wl["walk_length"],
+                                                 batch_size=bs, rng_key=1, num_threads=threads)]
         if kind == "shadow":
             return [[x] for x in oracle.shadow(O, s[:nbat * bs], wl["fanouts"], batch_size=bs,
                                                bias_mode=wl["bias"], rng_key=1,
@@ -348,7 +354,7 @@ def run_gpu(args, wl, world, rank, device):
         bs = wl["batch"]
         nunits = (inputs.numel() + bs - 1) // bs
         wbase = gdist.weak_batch_base(rank, nunits)
-        L = 1 if kind == "shadow" else len(wl.get("fanouts") or wl.get("n_per_layer"))
+        L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer"))
 
     def step(i, x=None):
         x = inputs if x is None else x
@@ -361,6 +367,9 @@ def run_gpu(args, wl, world, rank, device):
             gs.sample_shadow(G, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
                              bias_mode=wl["bias"], rng_key=key, stream=stream, out=out,
                              retry=False)
+        elif kind == "saint":
+            gs.sample_saint_rw(G, x, wl["walk_length"], batch_size=bs, batch_index_base=wbase,
+                               rng_key=key, stream=stream, out=out, retry=False)
         elif kind == "layerwise":
             gs.sample_layerwise(G, x, wl["n_per_layer"], batch_size=bs, batch_index_base=wbase,
                                 prob_mode=wl["mode"], rng_key=key, stream=stream, out=out,
@@ -368,6 +377,8 @@ def run_gpu(args, wl, world, rank, device):
         else:
             gs.random_walk(G, x, wl["length"], p=wl["p"], q=wl["q"], walker_index_base=wbase,
                            rng_key=key, stream=stream, out=traces)
+
+    cur = [0]  # the step index account() describes
 
     def grow_until_fits():
         # layer-wise / ShaDow outputs are sized on the device: every rng key the
@@ -397,10 +408,23 @@ def run_gpu(args, wl, world, rank, device):
             return (edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges,
                     edges + walkers + straddle)
         out.sync()
+        if kind == "saint":
+            # induce as ShaDow (per U node its column streamed once, 12 per
+            # induced edge, 4 per node) + the walks: per root 32(1+straddle) + 4,
+            # per step one 32-B record sector + 4 written + 4 read back (the
+            # traces, recomputed here outside the timed region for the count)
+            tot, e, rnd = _blocks_byte_model(out, g, "shadow", False, 1)
+            tr = gs.random_walk(G, inputs, wl["walk_length"], walker_index_base=wbase * bs,
+                                rng_key=base_key + 7919 * cur[0], stream=stream)
+            steps = int((tr[:, 1:] >= 0).sum())
+            st = inputs.to(torch.int64)
+            straddle = int(((st & 3) == 3).sum())
+            tot += steps * 40 + st.numel() * 36 + 32 * straddle
+            return tot, e, rnd + steps + st.numel() + straddle
         return _blocks_byte_model(out, g, kind, g["weights"] is not None and wl.get("mode") == 0,
                                   L, weighted_select=kind == "nodewise" and wl.get("bias", 0) != 0)
 
-    if kind in ("shadow", "layerwise"):
+    if kind in ("shadow", "saint", "layerwise"):
         grow_until_fits()
     for i in range(args.warmup):
         step(i)
@@ -416,6 +440,7 @@ def run_gpu(args, wl, world, rank, device):
             flush.zero_()
             ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             ev0.record(stream)
+            cur[0] = args.warmup + i
             step(args.warmup + i)
             ev1.record(stream)
             ev1.synchronize()
@@ -498,6 +523,7 @@ def run_gpu(args, wl, world, rank, device):
 
 
 KERNEL_OF = {"nodewise": "gsb::nodewise_wave_kernel", "shadow": "gsb::shadow_induce_kernel",
+             "saint": "gsb::shadow_induce_kernel",
              "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
 
 
@@ -565,7 +591,7 @@ def main():
                                      "(profiles/r01_random_access_probe.md)"}},
             "e2e": {"value": r["e2e_value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d"],
                     "d2h_bytes_per_step": r["d2h"]},
-            "gpu_launches": args.steps * (2 if kind == "shadow" else 1),
+            "gpu_launches": args.steps * (2 if kind in ("shadow", "saint") else 1),
             "clocks": r["clocks"],
         }
         if kind == "nodewise":

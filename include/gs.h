@@ -191,6 +191,25 @@ gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_
                            int num_layers, int bias_mode, uint64_t rng_key, void* stream,
                            gs_blocks** out);
 
+/* GraphSAINT-RW (Table 2: "conduct vanilla random walk and induce
+ * subgraph according to sampled nodes"; DESIGN R26).
+ *   roots       device int32[num_roots], cut into batches of batch_size (the
+ *               last may be shorter); root i walks walk_length DeepWalk steps
+ *               (R13) keyed by the global walker index
+ *               batch_index_base * batch_size + i (Philox tag 5, R4)
+ *   walk_length >= 0; batch_size * (walk_length + 1) <= 2^25 and the global
+ *               walker ids must fit 32 bits (else GS_ERR_NOT_SUPPORTED)
+ * Output: one block per batch (num_layers == 1), exactly as gs_sample_shadow:
+ * col_map == row_map == U = the distinct nodes the batch's walks visited,
+ * ascending; edges u->v of A with u, v in U in CSC order.  Roots outside
+ * [0, N) are reported by gs_blocks_sync (GS_ERR_INDEX_OUT_OF_RANGE); edge
+ * overflow as GS_ERR_CAPACITY (the object has grown: call again).
+ * Two launches: the walk kernel (traces kept in the result object) and the
+ * cluster induce kernel. */
+gs_status gs_sample_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_roots,
+                             int64_t batch_size, int64_t batch_index_base, int walk_length,
+                             uint64_t rng_key, void* stream, gs_blocks** out);
+
 /* ------------------------------------------------------------------------ */
 /* Layer-wise sampling (a1 + a2 + a4 + a6): FastGCN / LADIES.                 */
 /* ------------------------------------------------------------------------ */

@@ -93,7 +93,11 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
 gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
                       int64_t walker_base, int length, float p, float q, uint64_t key,
-                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces);
+                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces,
+                      int* err = nullptr);
+gs_status run_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_roots,
+                       int64_t batch_size, int64_t batch_base, int walk_length, uint64_t key,
+                       cudaStream_t stream, gs_blocks* blk);
 
 // ---------------------------------------------------------------------------
 // a0: CSC validation (indptr monotone and in range, indices in [0, N),
@@ -359,6 +363,25 @@ gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_
                     bias_mode, rng_key, stream, *out);
 }
 
+gs_status gs_sample_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_roots,
+                             int64_t batch_size, int64_t batch_index_base, int walk_length,
+                             uint64_t rng_key, void* stream_, gs_blocks** out) {
+  if (!g || !out || (!roots && num_roots > 0))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_saint_rw: null pointer argument");
+  if (num_roots < 0 || batch_size <= 0 || batch_index_base < 0 || walk_length < 0 ||
+      walk_length >= (1 << 24))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_saint_rw: bad num_roots/batch_size/base/walk_length");
+  if (num_roots >= (int64_t(1) << 31) || batch_size * ((int64_t)walk_length + 1) > MAX_SLOTS_PER_BATCH)
+    return fail(GS_ERR_NOT_SUPPORTED, "gs_sample_saint_rw: batch_size * (walk_length + 1) must be <= 2^25");
+  if ((batch_index_base + (num_roots + batch_size - 1) / batch_size) * batch_size > (int64_t(1) << 32))
+    return fail(GS_ERR_NOT_SUPPORTED, "gs_sample_saint_rw: global walker ids must fit 32 bits");
+  cudaStream_t stream = (cudaStream_t)stream_;
+  gs_status st = prepare_blocks(out, stream);
+  if (st) return st;
+  return run_saint_rw(g, roots, num_roots, batch_size, batch_index_base, walk_length, rng_key,
+                      stream, *out);
+}
+
 gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                               int64_t batch_size, int64_t batch_index_base,
                               const int32_t* n_per_layer, int num_layers, int prob_mode,
@@ -492,6 +515,7 @@ void gs_blocks_destroy(gs_blocks* b) {
   b->b_ctr.reset(b->al, s);
   b->b_sched.reset(b->al, s);
   b->b_pack.reset(b->al, s);
+  b->b_trace.reset(b->al, s);
   delete b;
 }
 

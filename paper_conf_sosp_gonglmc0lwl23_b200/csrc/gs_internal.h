@@ -80,6 +80,7 @@ struct gs_blocks {
       b_rowl[gsb::MAX_LAYERS], b_eid[gsb::MAX_LAYERS], b_val[gsb::MAX_LAYERS],
       b_rprob[gsb::MAX_LAYERS];
   gsb::DevBuf b_meta, b_err, b_ws, b_gen, b_ctr, b_sched, b_pack;
+  gsb::DevBuf b_trace;         // GraphSAINT-RW: walk traces between the walk and the induce launch
   std::vector<int64_t> h_meta;
   int64_t sh_edge_hint = 0;    // ShaDow edge capacity learnt from an overflow
   int64_t ws_stride_prev = -1; // workspace layout of the previous launch

@@ -1,6 +1,8 @@
-// shadow.cu -- ShaDow (R12): node-wise sampling of every hop
-// (nodewise_wave.cu), then per mini-batch the subgraph of A induced on
-// U = unique(seeds, rows of every hop), ascending (R3/R12).
+// shadow.cu -- induced subgraphs: ShaDow (R12): node-wise
+// sampling of every hop (nodewise_wave.cu), then per mini-batch the subgraph of
+// A induced on U = unique(seeds, rows of every hop), ascending (R3/R12); and
+// GraphSAINT-RW (R26): DeepWalk walks (walk.cu), then the subgraph
+// induced on U = the nodes each batch's walks visited.
 //
 // Induce is one persistent kernel of thread-block CLUSTERS, one cluster per
 // mini-batch at a time.  U's membership bitmap (N bits) is split across the
@@ -30,6 +32,10 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
                             int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                             int replace, int bias, uint64_t key, cudaStream_t stream,
                             gs_blocks* blk);
+gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
+                      int64_t walker_base, int length, float p, float q, uint64_t key,
+                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces,
+                      int* err = nullptr);
 
 constexpr int SH_THREADS = 512;
 constexpr int SH_WARPS = SH_THREADS / 32;
@@ -47,6 +53,8 @@ struct SHParams {
   const int32_t* rows[MAX_LAYERS];  // node-wise row_map of every hop
   int64_t K[MAX_LAYERS];
   const int64_t* nmeta;             // node-wise meta [b][L][8]
+  const int32_t* traces;            // GraphSAINT-RW: walk traces [root][L1] (U source instead of seeds + rows)
+  int64_t L1;                       // walk_length + 1
   int64_t stride;                   // U capacity per batch
   int32_t* U;                       // [b * stride] U ascending (col_map == row_map)
   int64_t* indptr_out;              // [b * stride + b] CSC over U
@@ -129,14 +137,21 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     const long long T0 = min(P.batch_size, P.num_seeds - bstart);
     long long nitems = T0;
     long long cnt_l[MAX_LAYERS];
-    for (int l = 0; l < P.L; ++l) {
-      cnt_l[l] = __ldcg(P.nmeta + (b * P.L + l) * 8 + 1);
-      nitems += cnt_l[l];
+    if (P.traces) {
+      nitems = T0 * P.L1;  // every visited node of the batch's walks (R26)
+    } else {
+      for (int l = 0; l < P.L; ++l) {
+        cnt_l[l] = __ldcg(P.nmeta + (b * P.L + l) * 8 + 1);
+        nitems += cnt_l[l];
+      }
     }
     for (long long i = (long long)rank * SH_THREADS + tid; i < nitems; i += (long long)CS * SH_THREADS) {
       long long x = i;
       int32_t u;
-      if (x < T0) {
+      if (P.traces) {
+        u = __ldcg(P.traces + bstart * P.L1 + x);
+        if (u == -1 && x % P.L1 != 0) continue;  // padding after a dead end (R13)
+      } else if (x < T0) {
         u = __ldg(P.seeds + bstart + x);
       } else {
         x -= T0;
@@ -342,11 +357,9 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
   }
 }
 
-gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
-                     int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
-                     int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
-  // cluster size: the N-bit bitmap (+ 1/64 prefix) split over at most 8 CTAs
-  const int64_t N = g->num_nodes;
+// Cluster size for an N-bit membership bitmap (+ 1/64 prefix + 1/32 offsets)
+// split over at most 8 CTAs' shared memory.
+static gs_status induce_envelope(int64_t N, int* CS_out, int64_t* bpc_out) {
   int CS = 1;
   int64_t bpc = 0;
   for (; CS <= SH_MAX_CS; CS *= 2) {
@@ -354,28 +367,20 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
     if (bpc / 8 + bpc / 64 + bpc / 32 <= SH_SMEM_CAP) break;
   }
   if (CS > SH_MAX_CS)
-    return fail(GS_ERR_NOT_SUPPORTED, "ShaDow: N = %lld exceeds the shared-memory bitmap envelope (%lld nodes)",
+    return fail(GS_ERR_NOT_SUPPORTED, "induce: N = %lld exceeds the shared-memory bitmap envelope (%lld nodes)",
                 (long long)N, (long long)(SH_MAX_CS * (SH_SMEM_CAP * 64 / 11)));
-  // 1. node-wise sampling of every hop (internal result object)
-  if (!blk->aux) {
-    blk->aux = new (std::nothrow) gs_blocks();
-    if (!blk->aux) return fail(GS_ERR_OUT_OF_MEMORY, "host allocation failed");
-    blk->aux->al = blk->al;
-  }
-  blk->aux->stream = stream;
-  gs_status st = run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias,
-                                   key, stream, blk->aux);
-  if (st) return st;
-  const gs_blocks* nw = blk->aux;
-  // 2. induce
+  *CS_out = CS;
+  *bpc_out = bpc;
+  return GS_OK;
+}
+
+// Induce on U (one block per batch) -- P carries the U sources (seeds + node-wise
+// rows, or walk traces); stride = U capacity per batch; err_src = the device
+// error word of the producing kernel, folded into the result's.
+static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bpc, int64_t nbatch,
+                               int64_t stride, const int* err_src, cudaStream_t stream,
+                               gs_blocks* blk) {
   const Allocator& al = blk->al;
-  const int64_t nbatch = (num_seeds + batch_size - 1) / batch_size;
-  int64_t sumK = 0, prod = 1;
-  for (int l = 0; l < L; ++l) {
-    prod *= fanouts[l];
-    sumK += prod;
-  }
-  const int64_t stride = batch_size * (1 + sumK);
   const int64_t nodes = nbatch * stride;
   blk->kind = gs_blocks::SHADOW;
   blk->num_batches = nbatch;
@@ -390,7 +395,7 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
             need(blk->b_rowl[0], edges * 4) && need(blk->b_eid[0], edges * 8) &&
             need(blk->b_row[0], nodes * 4) && need(blk->b_meta, std::max<int64_t>(nbatch, 1) * 64) &&
             need(blk->b_err, 16) && need(blk->b_ctr, 8 * (MAX_LAYERS + 2));
-  if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (ShaDow buffers)");
+  if (!ok) return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (induce buffers)");
   edges = (int64_t)std::min(blk->b_rowl[0].bytes / 4, blk->b_eid[0].bytes / 8);
   gs_layer_buffers& lb = blk->layers[0];
   lb = gs_layer_buffers{};
@@ -402,20 +407,10 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   lb.eid = (int64_t*)blk->b_eid[0].ptr;
   lb.edge_capacity = edges;
 
-  SHParams P = {};
   P.indptr = g->indptr;
   P.indices = g->indices;
-  P.N = N;
-  P.seeds = seeds;
-  P.num_seeds = num_seeds;
-  P.batch_size = batch_size;
+  P.N = g->num_nodes;
   P.num_batches = nbatch;
-  P.L = L;
-  for (int l = 0; l < L; ++l) {
-    P.rows[l] = nw->layers[l].row_map;
-    P.K[l] = l == 0 ? fanouts[0] : P.K[l - 1] * fanouts[l];
-  }
-  P.nmeta = (const int64_t*)nw->b_meta.ptr;
   P.stride = stride;
   P.U = lb.row_map;
   P.indptr_out = lb.indptr;
@@ -432,8 +427,8 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
-  // the node-wise kernel's error word (out-of-range seeds) is folded in
-  GS_CUDA_TRY(cudaMemcpyAsync(blk->b_err.ptr, nw->b_err.ptr, 4, cudaMemcpyDeviceToDevice, stream));
+  if (err_src)
+    GS_CUDA_TRY(cudaMemcpyAsync(blk->b_err.ptr, err_src, 4, cudaMemcpyDeviceToDevice, stream));
 
   const size_t smem = (size_t)(bpc / 8 + bpc / 64 + bpc / 32);
   GS_CUDA_TRY(cudaFuncSetAttribute(shadow_induce_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -463,13 +458,82 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
     const int64_t o_e = ((nw * P.wcap * 4) + 255) & ~int64_t(255);
     const int64_t o_s = o_e + nw * P.wcap * 8;
     if (!blk->b_ws.ensure(al, (size_t)(o_s + std::max<int64_t>(nodes, 1) * 8), stream))
-      return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (ShaDow staging)");
+      return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (induce staging)");
     P.stage_row = (int32_t*)blk->b_ws.ptr;
     P.stage_eid = (int64_t*)((char*)blk->b_ws.ptr + o_e);
     P.ustart = (int64_t*)((char*)blk->b_ws.ptr + o_s);
   }
   GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, shadow_induce_kernel, P));
   return GS_OK;
+}
+
+gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                     int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                     int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  int CS = 1;
+  int64_t bpc = 0;
+  gs_status st = induce_envelope(g->num_nodes, &CS, &bpc);
+  if (st) return st;
+  // 1. node-wise sampling of every hop (internal result object)
+  if (!blk->aux) {
+    blk->aux = new (std::nothrow) gs_blocks();
+    if (!blk->aux) return fail(GS_ERR_OUT_OF_MEMORY, "host allocation failed");
+    blk->aux->al = blk->al;
+  }
+  blk->aux->stream = stream;
+  st = run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias, key,
+                         stream, blk->aux);
+  if (st) return st;
+  const gs_blocks* nw = blk->aux;
+  // 2. induce on U = seeds + every hop's rows
+  const int64_t nbatch = (num_seeds + batch_size - 1) / batch_size;
+  int64_t sumK = 0, prod = 1;
+  for (int l = 0; l < L; ++l) {
+    prod *= fanouts[l];
+    sumK += prod;
+  }
+  SHParams P = {};
+  P.seeds = seeds;
+  P.num_seeds = num_seeds;
+  P.batch_size = batch_size;
+  P.L = L;
+  for (int l = 0; l < L; ++l) {
+    P.rows[l] = nw->layers[l].row_map;
+    P.K[l] = l == 0 ? fanouts[0] : P.K[l - 1] * fanouts[l];
+  }
+  P.nmeta = (const int64_t*)nw->b_meta.ptr;
+  return launch_induce(g, P, CS, bpc, nbatch, batch_size * (1 + sumK), (const int*)nw->b_err.ptr,
+                       stream, blk);
+}
+
+// GraphSAINT-RW (Table 2; R26): a DeepWalk walk from every root
+// (walk.cu, global walker ids batch_base * batch_size + i), then per batch the
+// subgraph induced on the nodes its walks visited.  The traces stay in HBM
+// between the two launches (4 B per visited slot, written once, read once).
+gs_status run_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_roots,
+                       int64_t batch_size, int64_t batch_base, int walk_length, uint64_t key,
+                       cudaStream_t stream, gs_blocks* blk) {
+  int CS = 1;
+  int64_t bpc = 0;
+  gs_status st = induce_envelope(g->num_nodes, &CS, &bpc);
+  if (st) return st;
+  const int64_t L1 = (int64_t)walk_length + 1;
+  const int64_t nbatch = (num_roots + batch_size - 1) / batch_size;
+  const int64_t tr_bytes = (num_roots * L1 * 4 + 255) & ~int64_t(255);
+  if (!blk->b_trace.ensure(blk->al, (size_t)(tr_bytes + 256), stream))
+    return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (GraphSAINT-RW traces)");
+  int* werr = (int*)((char*)blk->b_trace.ptr + tr_bytes);  // the walk's own error word (not the graph's)
+  GS_CUDA_TRY(cudaMemsetAsync(werr, 0, 4, stream));
+  st = launch_walk(g, roots, num_roots, batch_base * batch_size, walk_length, 1.0f, 1.0f, key,
+                   false, false, stream, (int32_t*)blk->b_trace.ptr, werr);
+  if (st) return st;
+  SHParams P = {};
+  P.seeds = roots;
+  P.num_seeds = num_roots;
+  P.batch_size = batch_size;
+  P.traces = (const int32_t*)blk->b_trace.ptr;
+  P.L1 = L1;
+  return launch_induce(g, P, CS, bpc, nbatch, batch_size * L1, werr, stream, blk);
 }
 
 }  // namespace gsb

@@ -163,7 +163,8 @@ static const int4* walk_index(const gs_graph* g, cudaStream_t stream, bool plain
 
 gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
                       int64_t walker_base, int length, float p, float q, uint64_t key,
-                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces) {
+                      bool node2vec, bool plain, cudaStream_t stream, int32_t* traces,
+                      int* err) {
   WalkParams P;
   P.rec = num_walkers > 0 && length > 0 ? walk_index(g, stream, plain) : nullptr;
   P.indptr = g->indptr;
@@ -179,7 +180,7 @@ gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walk
   P.bmax = fmaxf(P.bp, fmaxf(1.0f, P.bq));
   P.key = key;
   P.traces = traces;
-  P.err = g->d_err;
+  P.err = err ? err : g->d_err;
   if (num_walkers == 0) return GS_OK;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);

@@ -32,7 +32,8 @@ META_FIELDS = 8
 EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
-           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_layerwise",
+           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_saint_rw",
+           "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check"]
 
 
@@ -116,6 +117,7 @@ def load_library(path: str = LIB_PATH):
     L.gs_sample_neighbors.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
     L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
+    L.gs_sample_saint_rw.argtypes = [vp, vp, i64, i64, i64, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_layerwise.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
     L.gs_random_walk.argtypes = [vp, vp, i64, i64, i32, ctypes.c_float, ctypes.c_float, u64, u32,
@@ -360,6 +362,32 @@ def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch
             if e.status != 7 or attempt == 2:
                 raise
     out._seeds = seeds
+    return out
+
+
+def sample_saint_rw(g: Graph, roots: torch.Tensor, walk_length: int, batch_size=None,
+                    batch_index_base=0, rng_key=0, stream=None, out: Blocks = None, retry=True):
+    """GraphSAINT-RW (Table 2; DESIGN R26) through gs_sample_saint_rw:
+    one induced block per batch of roots."""
+    L = load_library()
+    _drain()
+    roots = roots.to(torch.int32).contiguous()
+    bs = int(batch_size or max(1, roots.numel()))
+    out = out or Blocks()
+    for attempt in range(3):
+        _check(L.gs_sample_saint_rw(g.handle, _ptr(roots), roots.numel(), bs, int(batch_index_base),
+                                    int(walk_length), ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                                    ctypes.byref(out._h)), "gs_sample_saint_rw")
+        out.synced = False
+        if not retry:
+            break
+        try:
+            out.sync()
+            break
+        except GSError as e:
+            if e.status != 7 or attempt == 2:
+                raise
+    out._seeds = roots
     return out
 
 

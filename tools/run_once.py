@@ -25,6 +25,10 @@ if wl["kind"] in ("nodewise", "shadow"):
         else:
             gs.sample_shadow(G, seeds, wl["fanouts"], batch_size=wl["batch"], bias_mode=wl["bias"],
                              rng_key=i, out=out)
+elif wl["kind"] == "saint":
+    roots = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
+    for i in range(reps):
+        gs.sample_saint_rw(G, roots, wl["walk_length"], batch_size=wl["batch"], rng_key=i, out=out)
 elif wl["kind"] == "layerwise":
     seeds = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
     for i in range(reps):
