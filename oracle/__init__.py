@@ -72,6 +72,8 @@ def lib():
         L.gso_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, i32,
                                  ctypes.POINTER(vp)]
         L.gso_saint_rw.argtypes = [vp, vp, i64, i64, i64, i32, u64, i32, ctypes.POINTER(vp)]
+        L.gso_pinsage.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, ctypes.c_float, u64,
+                                  i32, ctypes.POINTER(vp)]
         L.gso_random_walk.argtypes = [vp, vp, i64, i64, i32, ctypes.c_float, ctypes.c_float,
                                       u64, i32, i32, vp]
         L.gso_result_num_batches.argtypes = [vp]
@@ -215,6 +217,22 @@ def saint_rw(g: Graph, roots, walk_length, batch_size=None, batch_index_base=0, 
     if st:
         raise OracleError(st, "gso_saint_rw")
     return [blocks[0] for blocks in _collect(res)]
+
+
+def pinsage(g: Graph, seeds, topk, num_walks, walk_length, restart_prob, batch_size=None,
+            batch_index_base=0, rng_key=0, num_threads=0):
+    """PinSAGE-style sampling (Table 2; DESIGN R27): restart walks from every
+    frontier, its topk[l] most visited nodes as neighbours (val = visit count)."""
+    s = _seeds(seeds)
+    f = np.ascontiguousarray(topk, dtype=np.int32)
+    bs = batch_size or max(1, len(s))
+    res = ctypes.c_void_p()
+    st = lib().gso_pinsage(g.ptr, s.ctypes.data, len(s), bs, batch_index_base, f.ctypes.data,
+                           len(f), num_walks, walk_length, restart_prob, rng_key, num_threads,
+                           ctypes.byref(res))
+    if st:
+        raise OracleError(st, "gso_pinsage")
+    return _collect(res)
 
 
 def random_walk(g: Graph, starts, length, p=1.0, q=1.0, walker_index_base=0, rng_key=0,

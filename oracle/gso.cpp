@@ -12,6 +12,7 @@
 #include <cstring>
 #include <unordered_map>
 #include <utility>
+#include <map>
 #include <vector>
 #ifdef _OPENMP
 #include <omp.h>
@@ -49,7 +50,7 @@ Word4 philox(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3, uint64_t rng_ke
 
 // Tags of the counter word c2 = layer_or_step | tag << 24 (R4).
 enum { TAG_FLOYD = 1, TAG_REPLACE = 2, TAG_ARES_NODE = 3, TAG_ARES_LAYER = 4,
-       TAG_DEEPWALK = 5, TAG_NODE2VEC = 6 };
+       TAG_DEEPWALK = 5, TAG_NODE2VEC = 6, TAG_PINSAGE = 7 };
 
 uint32_t c2_of(int layer, int tag) { return (uint32_t)layer | ((uint32_t)tag << 24); }
 
@@ -541,6 +542,97 @@ int gso_saint_rw(const gso_graph* g, const int32_t* roots, int64_t num_roots, in
     for (int64_t i = lo * L1; i < hi * L1; ++i)
       if (traces[(size_t)i] >= 0) all.push_back(traces[(size_t)i]);  // -1: after a dead end (R13)
     r->blocks[(size_t)b] = induce(gg, std::move(all));
+  }
+  *out = r;
+  return GSO_OK;
+}
+
+// PinSAGE-style (Table 2: "random walks ... using restarts, select
+// top-k visited neighbors as sampled nodes"; R27).  For every frontier v:
+// num_walks walks from v of at most walk_length steps; before each step the
+// walk ends with probability restart_prob (the next walk restarts at v), or at
+// a node with no in-neighbours; draw r = philox(v, w * walk_length + t - 1,
+// layer | 7<<24, b): end if fp32((r2 >> 8) * 2^-24) < restart_prob, else step
+// to in-neighbour draw_below(d, r0, r1).  Every visit of a node x != v counts;
+// the k most visited (count descending, node id ascending) are v's sampled
+// neighbours, in that rank order, with val = fp32(count).  eid = -1: these
+// are not edges of A.  row_map = the selected nodes, unique ascending (R3).
+static Block pinsage_layer(const Graph& gg, const std::vector<int32_t>& F, int k, int num_walks,
+                           int walk_length, float restart_prob, int layer, uint32_t batch,
+                           uint64_t key) {
+  Block blk;
+  blk.col_map = F;
+  blk.has_val = true;
+  std::vector<std::vector<std::pair<int64_t, int32_t>>> sel(F.size());  // (count, node)
+  for (size_t j = 0; j < F.size(); ++j) {
+    const int32_t v = F[j];
+    std::map<int32_t, int64_t> count;
+    for (int w = 0; w < num_walks; ++w) {
+      int32_t x = v;
+      for (int t = 1; t <= walk_length; ++t) {
+        Word4 r = philox((uint32_t)v, (uint32_t)(w * walk_length + t - 1), c2_of(layer, TAG_PINSAGE),
+                         batch, key);
+        float y = (float)(r.v[2] >> 8) * 0x1p-24f;
+        if (y < restart_prob) break;  // restart: the next walk starts at v again
+        if (gg.deg(x) == 0) break;    // dead end (R13)
+        x = gg.indices[gg.off(x) + (int64_t)uniform_below((uint64_t)gg.deg(x), r.v[0], r.v[1])];
+        if (x != v) count[x] += 1;
+      }
+    }
+    std::vector<std::pair<int64_t, int32_t>> ranked;
+    for (auto& kv : count) ranked.push_back({kv.second, kv.first});
+    std::sort(ranked.begin(), ranked.end(), [](const std::pair<int64_t, int32_t>& a,
+                                               const std::pair<int64_t, int32_t>& b) {
+      return a.first != b.first ? a.first > b.first : a.second < b.second;
+    });
+    if ((int)ranked.size() > k) ranked.resize((size_t)k);
+    sel[j] = ranked;
+  }
+  std::vector<int32_t> rows;
+  for (auto& sj : sel)
+    for (auto& cx : sj) rows.push_back(cx.second);
+  std::sort(rows.begin(), rows.end());
+  rows.erase(std::unique(rows.begin(), rows.end()), rows.end());
+  blk.row_map = rows;
+  std::unordered_map<int32_t, int32_t> local;
+  for (size_t i = 0; i < rows.size(); ++i) local[rows[i]] = (int32_t)i;
+  blk.indptr.push_back(0);
+  for (auto& sj : sel) {
+    for (auto& cx : sj) {
+      blk.row_local.push_back(local[cx.second]);
+      blk.eid.push_back(-1);
+      blk.val.push_back((float)cx.first);
+    }
+    blk.indptr.push_back((int64_t)blk.eid.size());
+  }
+  return blk;
+}
+
+int gso_pinsage(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int64_t batch_size,
+                int64_t batch_index_base, const int32_t* topk, int num_layers, int num_walks,
+                int walk_length, float restart_prob, uint64_t rng_key, int num_threads,
+                gso_result** out) {
+  int st = check_common(g, seeds, num_seeds, batch_size, num_layers, topk, out);
+  if (st) return st;
+  if (num_walks < 1 || walk_length < 1 || !(restart_prob >= 0.0f) || !(restart_prob <= 1.0f))
+    return GSO_ERR_INVALID_ARGUMENT;
+  Graph gg{g->num_nodes, g->num_edges, g->indptr, g->indices, g->weights};
+  gso_result* r = new gso_result();
+  r->num_batches = (num_seeds + batch_size - 1) / batch_size;
+  r->num_layers = num_layers;
+  r->blocks.resize((size_t)r->num_batches * num_layers);
+  set_threads(num_threads);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t b = 0; b < r->num_batches; ++b) {
+    int64_t lo = b * batch_size, hi = std::min(num_seeds, lo + batch_size);
+    std::vector<int32_t> frontier(seeds + lo, seeds + hi);
+    uint32_t gb = (uint32_t)(batch_index_base + b);
+    for (int l = 0; l < num_layers; ++l) {
+      Block blk = pinsage_layer(gg, frontier, topk[l], num_walks, walk_length, restart_prob, l, gb,
+                                rng_key);
+      frontier = blk.row_map;  // next frontier = the selected nodes (R2)
+      r->blocks[(size_t)b * num_layers + l] = std::move(blk);
+    }
   }
   *out = r;
   return GSO_OK;

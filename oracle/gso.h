@@ -15,7 +15,8 @@
  *              random walks (DeepWalk P:75, Node2Vec P:82)
  *   - Finalize row()/column() + relabel/compaction,
  *              ShaDow induced subgraph,
- *              GraphSAINT-RW walk + induce
+ *              GraphSAINT-RW walk + induce,
+ *              PinSAGE-style restart walks + top-k visited
  * The paper does not fix the sampling algorithms, the RNG or the output order;
  * the readings used here are DESIGN.md section "Readings" (R1..R25), which
  * follow SURVEY.md section 8(c).  Every random draw is Philox4x32-10 keyed by
@@ -105,6 +106,16 @@ int gso_shadow(const gso_graph* g, const int32_t* seeds, int64_t num_seeds,
 int gso_saint_rw(const gso_graph* g, const int32_t* roots, int64_t num_roots, int64_t batch_size,
                  int64_t batch_index_base, int walk_length, uint64_t rng_key, int num_threads,
                  gso_result** out);
+
+/* PinSAGE-style (Table 2; R27): per frontier v, num_walks walks of at
+ * most walk_length steps, each step preceded by an end-with-probability
+ * restart_prob test; the topk[l] most visited nodes != v (count descending,
+ * id ascending) are v's neighbours (val = visit count, eid = -1).  Next
+ * frontier = row_map (the selected nodes, ascending). */
+int gso_pinsage(const gso_graph* g, const int32_t* seeds, int64_t num_seeds, int64_t batch_size,
+                int64_t batch_index_base, const int32_t* topk, int num_layers, int num_walks,
+                int walk_length, float restart_prob, uint64_t rng_key, int num_threads,
+                gso_result** out);
 
 /* DeepWalk (p == q == 1 and !force_node2vec) / Node2Vec random walks.
  * traces: caller-owned int32 [num_walkers][length+1], -1 after a dead end. */
