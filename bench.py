@@ -62,6 +62,10 @@ WORKLOADS = {
     "saint_pd": dict(kind="saint", graph="PD", walk_length=2, batch=3000, seeds=None,
                      desc="GraphSAINT-RW 3000 roots x walk length 2 + induce per subgraph, every "
                           "node a root once per epoch (817 subgraphs), PD-shaped"),
+    "pinsage_pd": dict(kind="pinsage", graph="PD", topk=[10, 10], num_walks=10, walk_length=3,
+                       restart=0.5, batch=1024, seeds=196_615,
+                       desc="PinSAGE-style top-k [10,10] of 10 restart walks (<= 3 steps, restart "
+                            "0.5), batch 1024, full epoch (196,615 seeds), PD-shaped"),
     "ladies_lj": dict(kind="layerwise", graph="LJ", n_per_layer=[512, 512, 512], batch=512,
                       seeds=None, mode=0, desc="LADIES 512x3, LJ-shaped, all nodes as seeds"),
     "fastgcn_lj": dict(kind="layerwise", graph="LJ", n_per_layer=[512, 512, 512], batch=512,
@@ -266,6 +270,9 @@ def oracle_rate(g, inputs, wl, budget_s=15.0):
             return oracle.sample_neighbors(O, s[:nbat * bs], wl["fanouts"], batch_size=bs,
                                            replace=wl["replace"], bias_mode=wl["bias"], rng_key=1,
                                            num_threads=threads)
+        if kind == "pinsage":
+            return oracle.pinsage(O, s[:nbat * bs], wl["topk"], wl["num_walks"], wl["walk_length"],
+                                  wl["restart"], batch_size=bs, rng_key=1, num_threads=threads)
         if kind == "saint":
             return [[x] for x in oracle.saint_rw(O, s[:nbat * bs], wl["walk_length"],
                                                  batch_size=bs, rng_key=1, num_threads=threads)]
@@ -354,7 +361,8 @@ def run_gpu(args, wl, world, rank, device):
         bs = wl["batch"]
         nunits = (inputs.numel() + bs - 1) // bs
         wbase = gdist.weak_batch_base(rank, nunits)
-        L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer"))
+        L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer")
+                                                       or wl.get("topk"))
 
     def step(i, x=None):
         x = inputs if x is None else x
@@ -367,6 +375,10 @@ def run_gpu(args, wl, world, rank, device):
             gs.sample_shadow(G, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
                              bias_mode=wl["bias"], rng_key=key, stream=stream, out=out,
                              retry=False)
+        elif kind == "pinsage":
+            gs.sample_pinsage(G, x, wl["topk"], wl["num_walks"], wl["walk_length"], wl["restart"],
+                              batch_size=bs, batch_index_base=wbase, rng_key=key, stream=stream,
+                              out=out)
         elif kind == "saint":
             gs.sample_saint_rw(G, x, wl["walk_length"], batch_size=bs, batch_index_base=wbase,
                                rng_key=key, stream=stream, out=out, retry=False)
@@ -408,6 +420,20 @@ def run_gpu(args, wl, world, rank, device):
             return (edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges,
                     edges + walkers + straddle)
         out.sync()
+        if kind == "pinsage":
+            # per frontier column: 4 (id) + its walks' steps, each one random
+            # indptr-pair sector + one random index sector (32 + 32); the steps
+            # are counted by their expectation W * sum_t (1-r)^t (the restart
+            # law); per selected neighbour 16 (row_local + val + eid) + 8
+            # (indptr); per row 4
+            meta = out.device_meta().cpu()
+            cols = int(meta[:, :, 0].sum())
+            rows = int(meta[:, :, 1].sum())
+            e = int(meta[:, :, 2].sum())
+            r = wl["restart"]
+            steps = cols * wl["num_walks"] * sum((1 - r) ** t for t in range(1, wl["walk_length"] + 1))
+            tot = cols * (4 + 8) + int(steps * 64) + e * 16 + rows * 4
+            return tot, e, int(2 * steps)
         if kind == "saint":
             # induce as ShaDow (per U node its column streamed once, 12 per
             # induced edge, 4 per node) + the walks: per root 32(1+straddle) + 4,
@@ -523,7 +549,7 @@ def run_gpu(args, wl, world, rank, device):
 
 
 KERNEL_OF = {"nodewise": "gsb::nodewise_wave_kernel", "shadow": "gsb::shadow_induce_kernel",
-             "saint": "gsb::shadow_induce_kernel",
+             "saint": "gsb::shadow_induce_kernel", "pinsage": "gsb::pinsage_kernel",
              "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
 
 

@@ -210,6 +210,30 @@ gs_status gs_sample_saint_rw(const gs_graph* g, const int32_t* roots, int64_t nu
                              int64_t batch_size, int64_t batch_index_base, int walk_length,
                              uint64_t rng_key, void* stream, gs_blocks** out);
 
+/* PinSAGE-style (Table 2: "random walks ... using restarts, select
+ * top-k visited neighbors as sampled nodes"; DESIGN R27).
+ * Per (batch b, layer l) and frontier column v: num_walks walks from v of at
+ * most walk_length steps; before step t of walk w, r = philox(v,
+ * w*walk_length + t-1, l | 7<<24, batch_index_base + b): the walk ends if
+ * fp32((r2>>8) 2^-24) < restart_prob (the next walk restarts at v) or at a
+ * node with no in-neighbours, else it moves to in-neighbour draw_below(d).
+ * Every visit of a node x != v counts; v's neighbours are its topk[l] most
+ * visited nodes (count descending, id ascending), in that order.
+ *   seeds       device int32[num_seeds], batches of batch_size (last ragged)
+ *   topk        host int32[num_layers], 1..32; 1 <= num_layers <= 8
+ *   num_walks, walk_length >= 1, num_walks * walk_length <= 2048
+ *   restart_prob in [0, 1]
+ * Output per (b, l) like gs_sample_neighbors: col_map = frontier (l = 0 the
+ * seeds, else the previous layer's row_map, R2), row_map = the selected nodes
+ * ascending (R3), CSC over local ids with each column in rank order,
+ * val = fp32(visit count), eid = -1 (these are not edges of A).
+ * Envelope: batch_size * prod(topk[0..l]) <= 2^25.  Seeds outside [0, N) are
+ * reported by gs_blocks_sync; their columns are empty.  One kernel launch. */
+gs_status gs_sample_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_index_base, const int32_t* topk,
+                            int num_layers, int num_walks, int walk_length, float restart_prob,
+                            uint64_t rng_key, void* stream, gs_blocks** out);
+
 /* ------------------------------------------------------------------------ */
 /* Layer-wise sampling (a1 + a2 + a4 + a6): FastGCN / LADIES.                 */
 /* ------------------------------------------------------------------------ */

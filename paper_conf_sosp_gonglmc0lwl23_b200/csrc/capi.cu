@@ -95,6 +95,10 @@ gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walk
                       int64_t walker_base, int length, float p, float q, uint64_t key,
                       bool node2vec, bool plain, cudaStream_t stream, int32_t* traces,
                       int* err = nullptr);
+gs_status run_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                      int64_t batch_size, int64_t batch_base, const int32_t* topk, int L,
+                      int num_walks, int walk_length, float restart, uint64_t key,
+                      cudaStream_t stream, gs_blocks* blk);
 gs_status run_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_roots,
                        int64_t batch_size, int64_t batch_base, int walk_length, uint64_t key,
                        cudaStream_t stream, gs_blocks* blk);
@@ -380,6 +384,30 @@ gs_status gs_sample_saint_rw(const gs_graph* g, const int32_t* roots, int64_t nu
   if (st) return st;
   return run_saint_rw(g, roots, num_roots, batch_size, batch_index_base, walk_length, rng_key,
                       stream, *out);
+}
+
+gs_status gs_sample_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                            int64_t batch_size, int64_t batch_index_base, const int32_t* topk,
+                            int num_layers, int num_walks, int walk_length, float restart_prob,
+                            uint64_t rng_key, void* stream_, gs_blocks** out) {
+  gs_status st = check_batches(g, seeds, num_seeds, batch_size, batch_index_base, topk,
+                               num_layers, out);
+  if (st) return st;
+  if (num_walks < 1 || walk_length < 1 || !(restart_prob >= 0.0f) || !(restart_prob <= 1.0f))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_pinsage: num_walks, walk_length >= 1 and restart_prob in [0, 1] required");
+  if ((int64_t)num_walks * walk_length > 2048)
+    return fail(GS_ERR_NOT_SUPPORTED, "gs_sample_pinsage: num_walks * walk_length must be <= 2048");
+  int64_t prod = batch_size;
+  for (int l = 0; l < num_layers; ++l) {
+    if (topk[l] > MAX_FANOUT) return fail(GS_ERR_NOT_SUPPORTED, "top-k must be <= %d", MAX_FANOUT);
+    prod *= topk[l];
+    if (prod > MAX_SLOTS_PER_BATCH)
+      return fail(GS_ERR_NOT_SUPPORTED, "batch_size * prod(topk) must be <= 2^25");
+  }
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if ((st = prepare_blocks(out, stream))) return st;
+  return run_pinsage(g, seeds, num_seeds, batch_size, batch_index_base, topk, num_layers, num_walks,
+                     walk_length, restart_prob, rng_key, stream, *out);
 }
 
 gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,

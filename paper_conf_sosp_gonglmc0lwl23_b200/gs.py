@@ -32,7 +32,7 @@ META_FIELDS = 8
 EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
-           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_saint_rw",
+           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_saint_rw", "gs_sample_pinsage",
            "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check"]
 
@@ -117,6 +117,8 @@ def load_library(path: str = LIB_PATH):
     L.gs_sample_neighbors.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
     L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
+    L.gs_sample_pinsage.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, ctypes.c_float, u64,
+                                    vp, ctypes.POINTER(vp)]
     L.gs_sample_saint_rw.argtypes = [vp, vp, i64, i64, i64, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_layerwise.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
@@ -361,6 +363,24 @@ def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch
         except GSError as e:
             if e.status != 7 or attempt == 2:
                 raise
+    out._seeds = seeds
+    return out
+
+
+def sample_pinsage(g: Graph, seeds: torch.Tensor, topk, num_walks: int, walk_length: int,
+                   restart_prob: float, batch_size=None, batch_index_base=0, rng_key=0,
+                   stream=None, out: Blocks = None):
+    """PinSAGE-style sampling (Table 2; DESIGN R27) through gs_sample_pinsage."""
+    L = load_library()
+    _drain()
+    seeds = seeds.to(torch.int32).contiguous()
+    bs = int(batch_size or max(1, seeds.numel()))
+    out = out or Blocks()
+    _check(L.gs_sample_pinsage(g.handle, _ptr(seeds), seeds.numel(), bs, int(batch_index_base),
+                               _host_i32(topk), len(topk), int(num_walks), int(walk_length),
+                               float(restart_prob), ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                               ctypes.byref(out._h)), "gs_sample_pinsage")
+    out.synced = False
     out._seeds = seeds
     return out
 

@@ -25,6 +25,11 @@ if wl["kind"] in ("nodewise", "shadow"):
         else:
             gs.sample_shadow(G, seeds, wl["fanouts"], batch_size=wl["batch"], bias_mode=wl["bias"],
                              rng_key=i, out=out)
+elif wl["kind"] == "pinsage":
+    seeds = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
+    for i in range(reps):
+        gs.sample_pinsage(G, seeds, wl["topk"], wl["num_walks"], wl["walk_length"], wl["restart"],
+                          batch_size=wl["batch"], rng_key=i, out=out)
 elif wl["kind"] == "saint":
     roots = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
     for i in range(reps):
