@@ -15,7 +15,7 @@
 //      positions j*k + r, and marks the ids in the CTA's N-bit row bitmap
 //      (global memory, L2-resident, left cleared after every layer);
 //   F  finalize: CSC indptr by a block scan of the per-column counts; a
-//      popcount prefix per 16 bitmap words (global, per CTA); row_local =
+//      popcount prefix per 4 bitmap words (global, per CTA); row_local =
 //      rank of the id (prefix + popc of the words before it in its group +
 //      popc below it in its word), val = fp32(count); row_map = the set bits
 //      in ascending order (R3), clearing the bitmap as it goes; eid = -1.
@@ -35,7 +35,8 @@ constexpr uint32_t TAG_PINSAGE = 7;
 constexpr int PS_THREADS = 512;
 constexpr int PS_WARPS = PS_THREADS / 32;
 constexpr int PS_SMEM = 48 * 1024;   // hash tables of one chunk (4 CTAs per SM fit)
-constexpr int PS_GROUP = 16;         // bitmap words per prefix entry
+constexpr int PS_GROUP = 4;          // bitmap words per prefix entry
+constexpr int PS_ILP = 2;            // walks per thread in lockstep
 
 struct PSParams {
   const int64_t* indptr;
@@ -119,29 +120,55 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
       for (long long c0 = 0; c0 < nF; c0 += C) {
         const int nc = (int)min((long long)C, nF - c0);
         const int npairs = nc * W;
-        for (int i = tid; i < npairs; i += PS_THREADS) {
-          const int cj = i / W, w = i - cj * W;
-          const int32_t v = __ldcg(F + c0 + cj);
-          if (v < 0 || (int64_t)v >= P.N) continue;
-          int32_t* tk = hkey + cj * HCAP;
-          int32_t* tc = hcnt + cj * HCAP;
-          int32_t x = v;
+        // PS_ILP independent walks per thread advance in lockstep, so their
+        // dependent loads (indptr pair, then the index) overlap
+        for (int i = tid; i < npairs; i += PS_ILP * PS_THREADS) {
+          int32_t wv[PS_ILP], wx[PS_ILP];
+          int wcol[PS_ILP], ww[PS_ILP];
+          bool alive[PS_ILP];
+#pragma unroll
+          for (int a = 0; a < PS_ILP; ++a) {
+            const int ia = i + a * PS_THREADS;
+            alive[a] = ia < npairs;
+            wcol[a] = alive[a] ? ia / W : 0;
+            ww[a] = ia - wcol[a] * W;
+            wv[a] = alive[a] ? __ldcg(F + c0 + wcol[a]) : 0;
+            if (wv[a] < 0 || (int64_t)wv[a] >= P.N) alive[a] = false;
+            wx[a] = wv[a];
+          }
           for (int t = 1; t <= T; ++t) {
-            const U4 r = philox((uint32_t)v, (uint32_t)(w * T + t - 1), ctr2(l, TAG_PINSAGE), gb, P.key);
-            const float y = (float)(r.z >> 8) * 0x1p-24f;
-            if (y < P.restart) break;                    // restart at v (R27)
-            const int64_t off = __ldg(P.indptr + x), d = __ldg(P.indptr + x + 1) - off;
-            if (d == 0) break;                           // dead end (R13)
-            x = __ldg(P.indices + off + (int64_t)draw_below((uint64_t)d, r.x, r.y));
-            if (x == v) continue;
-            uint32_t h = ps_hash((uint32_t)x) & (uint32_t)(HCAP - 1);
-            while (true) {
-              const int32_t old = atomicCAS(tk + h, -1, x);
-              if (old == -1 || old == x) {
-                atomicAdd(tc + h, 1);
-                break;
+            U4 r[PS_ILP];
+            int64_t off[PS_ILP], d[PS_ILP];
+#pragma unroll
+            for (int a = 0; a < PS_ILP; ++a) {
+              r[a] = philox((uint32_t)wv[a], (uint32_t)(ww[a] * T + t - 1), ctr2(l, TAG_PINSAGE), gb, P.key);
+              if ((float)(r[a].z >> 8) * 0x1p-24f < P.restart) alive[a] = false;  // restart at v (R27)
+              off[a] = alive[a] ? __ldg(P.indptr + wx[a]) : 0;
+              d[a] = alive[a] ? __ldg(P.indptr + wx[a] + 1) : 0;
+            }
+            bool any = false;
+#pragma unroll
+            for (int a = 0; a < PS_ILP; ++a) {
+              d[a] -= off[a];
+              if (d[a] == 0) alive[a] = false;            // dead end (R13)
+              if (alive[a]) wx[a] = __ldg(P.indices + off[a] + (int64_t)draw_below((uint64_t)d[a], r[a].x, r[a].y));
+              any |= alive[a];
+            }
+            if (!any) break;
+#pragma unroll
+            for (int a = 0; a < PS_ILP; ++a) {
+              if (!alive[a] || wx[a] == wv[a]) continue;
+              int32_t* tk = hkey + wcol[a] * HCAP;
+              int32_t* tc = hcnt + wcol[a] * HCAP;
+              uint32_t h = ps_hash((uint32_t)wx[a]) & (uint32_t)(HCAP - 1);
+              while (true) {
+                const int32_t old = atomicCAS(tk + h, -1, wx[a]);
+                if (old == -1 || old == wx[a]) {
+                  atomicAdd(tc + h, 1);
+                  break;
+                }
+                h = (h + 1) & (uint32_t)(HCAP - 1);
               }
-              h = (h + 1) & (uint32_t)(HCAP - 1);
             }
           }
         }
@@ -201,7 +228,7 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
       }
       if (tid == 0) ip[0] = 0;
       const long long E = run;
-      // ---- popcount prefix per group of 16 bitmap words ----
+      // ---- popcount prefix per group of PS_GROUP bitmap words ----
       long long rrun = 0;
       for (long long g0 = 0; g0 < P.ngroups; g0 += PS_THREADS) {
         const long long g = g0 + tid;
@@ -229,7 +256,7 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
         if (lane < n) {
           const int64_t s = scratch[j * k + lane];
           const int32_t id = (int32_t)(uint32_t)s;
-          const long long g = id >> 9;  // 16 words x 32 bits
+          const long long g = id >> 7;  // PS_GROUP words x 32 bits
           int rank = __ldcg(gp + g);
           const int wi = id >> 5;
           for (int q = (int)(g * PS_GROUP); q < wi; ++q) rank += __popc(__ldcg(bm + q));

@@ -10,8 +10,9 @@
 // a popcount prefix per 256 bits, so the membership test of every streamed
 // edge -- the hot loop, Sum of in-degrees over U per batch -- and the rank of a
 // kept row are shared-memory reads (local or a peer's), never L2/HBM probes.
-// Per batch: mark U -> scan (U ascending) -> count kept edges per column,
-// staging each kept edge (row rank, eid) in a per-warp region -> scan (CSC
+// Per batch: mark U -> scan (U ascending) -> count kept edges per column
+// (columns claimed dynamically by every warp of the cluster from a DSMEM
+// counter), staging each kept edge (row rank, eid) in a per-warp region -> scan (CSC
 // indptr, bump-allocated edge range) -> copy the staged edges to their CSC
 // positions (a column whose edges did not fit the region is streamed again).
 #include <algorithm>
@@ -41,6 +42,7 @@ constexpr int SH_THREADS = 512;
 constexpr int SH_WARPS = SH_THREADS / 32;
 constexpr int SH_MAX_CS = 8;                      // portable cluster size
 constexpr int SH_ILP = 8;                         // column positions per lane in flight
+constexpr int SH_CLAIM = 4;                       // columns per claim of the count pass
 constexpr int64_t SH_SMEM_CAP = 220 * 1024;      // dynamic shared memory per CTA (bitmap + prefixes)
 
 struct SHParams {
@@ -78,6 +80,7 @@ struct SHShared {                   // static part; the bitmap + prefix are dyna
   long long b;
   long long total, base[SH_MAX_CS];
   long long etotal, ebase, eoff, E, nU;
+  unsigned long long next;          // rank 0: the cluster's column claim counter (count pass)
   long long scr64[40];
   int scr32[40];
 };
@@ -184,7 +187,10 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       if (g < ngroups) gp[g] = (int32_t)(run + ex);
       run += tot;
     }
-    if (tid == 0) ss.total = run;
+    if (tid == 0) {
+      ss.total = run;
+      ss.next = 0;
+    }
     cl.sync();
     if (tid < (int)CS) ss.base[tid] = 0;
     if (tid == 0) {
@@ -221,7 +227,17 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     int32_t* wst_r = P.stage_row + wreg;
     int64_t* wst_e = P.stage_eid + wreg;
     long long wfill = 0;
-    for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
+    // columns are claimed dynamically, SH_CLAIM at a time, from a counter in
+    // rank 0's shared memory by every warp of the cluster (hub columns no
+    // longer pin one warp / one CTA while the others wait at the barrier)
+    unsigned long long* next = cl.map_shared_rank(&ss.next, 0);
+    for (;;) {
+    long long cb = 0;
+    if (lane == 0) cb = (long long)atomicAdd(next, (unsigned long long)SH_CLAIM);
+    cb = __shfl_sync(0xffffffffu, cb, 0);
+    if (cb >= nU) break;
+    const long long ce = min(cb + SH_CLAIM, nU);
+    for (long long c = cb; c < ce; ++c) {
       const int32_t v = __ldcg(U + c);
       const int64_t o = __ldg(P.indptr + v), d = __ldg(P.indptr + v + 1) - o;
       int cnt = 0;
@@ -256,8 +272,9 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       if (!staged) wfill = start;
       if (lane == 0) {
         ucnt[c] = cnt;
-        ustart[c] = staged ? start : -1;
+        ustart[c] = staged ? wreg + start : -1;  // absolute staging index
       }
+    }
     }
     __threadfence();
     cl.sync();
@@ -297,7 +314,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       if (!fits) atomicOr(P.err, ERR_CAPACITY);
     }
     // ---- write kept edges in CSC order: a copy of the staged edges (the
-    // same warp staged this column); columns that did not fit re-stream ----
+    // claiming warp staged it, ustart is absolute); columns that did not fit re-stream ----
     if (fits) {
       for (long long c = c_lo + warp; c < c_hi; c += SH_WARPS) {
         const long long st = __ldcg(ustart + c);
@@ -312,8 +329,8 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
             for (int q = 0; q < SH_ILP; ++q) {
               const long long i = i0 + 32 * q;
               if (i < n) {
-                r[q] = __ldcs(wst_r + st + i);
-                e[q] = __ldcs(wst_e + st + i);
+                r[q] = __ldcs(P.stage_row + st + i);
+                e[q] = __ldcs(P.stage_eid + st + i);
               }
             }
 #pragma unroll
