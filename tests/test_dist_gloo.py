@@ -42,6 +42,14 @@ def _worker(rank, world, port, out_dir):
     O = oracle.Graph(g["indptr"].numpy(), g["indices"].numpy(), g["weights"].numpy())
     res = oracle.sample_neighbors(O, seeds[s0:s1].numpy(), [5, 3], batch_size=bs,
                                   batch_index_base=lo, rng_key=77)
+    # GraphSAINT-RW and PinSAGE-style shard the same way (global batch ids)
+    sa = oracle.saint_rw(O, seeds[s0:s1].numpy(), 3, batch_size=bs, batch_index_base=lo,
+                         rng_key=78)
+    np.save(os.path.join(out_dir, f"saint_{rank}.npy"), np.concatenate([b["eid"] for b in sa]))
+    ps = oracle.pinsage(O, seeds[s0:s1].numpy(), [4, 2], 6, 3, 0.4, batch_size=bs,
+                        batch_index_base=lo, rng_key=79)
+    np.save(os.path.join(out_dir, f"pinsage_{rank}.npy"),
+            np.concatenate([blk["row_map"][blk["row_local"]] for layers in ps for blk in layers]))
     edges = sum(len(blk["eid"]) for layers in res for blk in layers)
     tot_edges, max_ms = gdist.reduce_measurement(edges, 10.0 + rank, torch.device("cpu"))
     np.save(os.path.join(out_dir, f"eids_{rank}.npy"),
@@ -74,6 +82,13 @@ def test_two_rank_gloo_shard_invariance(tmp_path, oracle_lib):
     want = np.concatenate([blk["eid"] for layers in full for blk in layers])
     got = np.concatenate([np.load(tmp_path / f"eids_{r}.npy") for r in range(world)])
     assert np.array_equal(got, want)
+    sa = oracle_lib.saint_rw(O, seeds, 3, batch_size=64, rng_key=78)
+    got = np.concatenate([np.load(tmp_path / f"saint_{r}.npy") for r in range(world)])
+    assert np.array_equal(got, np.concatenate([b["eid"] for b in sa]))
+    ps = oracle_lib.pinsage(O, seeds, [4, 2], 6, 3, 0.4, batch_size=64, rng_key=79)
+    got = np.concatenate([np.load(tmp_path / f"pinsage_{r}.npy") for r in range(world)])
+    assert np.array_equal(got, np.concatenate([blk["row_map"][blk["row_local"]]
+                                               for layers in ps for blk in layers]))
     m0, m1 = np.load(tmp_path / "meta_0.npy"), np.load(tmp_path / "meta_1.npy")
     assert m0[2] == m1[2] == len(want)          # all-reduce SUM of edges
     assert m0[3] == m1[3] == 11.0               # all-reduce MAX of time
