@@ -68,9 +68,7 @@ typedef struct gs_graph gs_graph;
 
 enum {
   GS_GRAPH_HOST_PTRS = 1, /* indptr/indices/weights are host pointers (copied to HBM)      */
-  GS_GRAPH_BORROW = 2     /* device pointers are used in place; caller keeps them alive
-                             (an index array not 16-byte aligned or whose length is not a
-                             multiple of 4 is copied: the induce kernel reads 16-B vectors) */
+  GS_GRAPH_BORROW = 2     /* device pointers are used in place; caller keeps them alive    */
 };                        /* default (0): device pointers, copied into library-owned HBM  */
 
 /* Validates the CSC on the device (indptr[0] == 0, monotone, indptr[N] ==

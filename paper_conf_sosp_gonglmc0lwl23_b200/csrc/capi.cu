@@ -211,12 +211,7 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
     gs_graph_destroy(g);
     return st;
   };
-  // the induce kernel streams indices in 16-byte vectors: a borrowed index
-  // array must be 16-byte aligned with a length that is a multiple of 4
-  // (else it is copied; owned buffers carry slack past the end)
-  const bool borrow = (flags & GS_GRAPH_BORROW) && ((uintptr_t)indices & 15) == 0 &&
-                      (num_edges & 3) == 0;
-  if (borrow) {
+  if (flags & GS_GRAPH_BORROW) {
     g->indptr = const_cast<int64_t*>(indptr);
     g->indices = const_cast<int32_t*>(indices);
     g->weights = const_cast<float*>(weights);
@@ -224,7 +219,7 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
     const cudaMemcpyKind kind =
         (flags & GS_GRAPH_HOST_PTRS) ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
     if (!g->b_indptr.ensure(g->al, (num_nodes + 1) * 8, stream) ||
-        !g->b_indices.ensure(g->al, std::max<int64_t>(num_edges, 1) * 4 + 16, stream) ||
+        !g->b_indices.ensure(g->al, std::max<int64_t>(num_edges, 1) * 4, stream) ||
         (weights && !g->b_weights.ensure(g->al, std::max<int64_t>(num_edges, 1) * 4, stream)))
       return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_create: device allocation failed"));
     g->owns = true;

@@ -229,13 +229,6 @@ __device__ __forceinline__ float ldg_h(const float* a, uint64_t p) {
   asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(a), "l"(p));
   return v;
 }
-// 16-byte vector of read-only graph data (a must be 16-byte aligned)
-__device__ __forceinline__ uint4 ldg_h4(const int32_t* a, uint64_t p) {
-  uint4 v;
-  asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
-               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a), "l"(p));
-  return v;
-}
 __device__ __forceinline__ void sth(int32_t* a, int32_t v, uint64_t p) {
   asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(p) : "memory");
 }

@@ -10,7 +10,8 @@
 //      current node's indptr pair and one index gather per step -- and counts
 //      each visit of x != v with a shared-memory atomicAdd;
 //   S  select: a warp per column takes the k most visited entries (count
-//      descending, id ascending) by k rounds of a warp arg-max, writes them
+//      descending, id ascending) -- a warp bitonic sort of the (<= 32)
+//      visited nodes, else k rounds of a warp arg-max -- writes them
 //      (count, id) to the layer's eid region as scratch at column-major
 //      positions j*k + r, and marks the ids in the CTA's N-bit row bitmap
 //      (global memory, L2-resident, left cleared after every layer);
@@ -81,6 +82,7 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
   __shared__ long long s_b;
   __shared__ int scr[40];
   __shared__ long long scr64[40];
+  __shared__ unsigned long long wstage[PS_WARPS * 32];  // per-warp top-k staging
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int HCAP = 1 << P.hlog;
   const int C = P.chunk;
@@ -178,6 +180,44 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
           int32_t* tc = hcnt + cj * HCAP;
           const long long j = c0 + cj;
           int taken = 0;
+          // fast path: at most 32 visited nodes -> one key per lane, a warp
+          // bitonic sort (15 compare-exchange steps) instead of k arg-max rounds
+          unsigned long long* st = wstage + warp * 32;
+          int nv = 0;
+          for (int e0 = 0; e0 < HCAP; e0 += 32) {
+            const int e = e0 + lane;
+            const int cnt = tc[e];
+            const unsigned bal = __ballot_sync(0xffffffffu, cnt > 0);
+            if (cnt > 0) {
+              const int pos = nv + __popc(bal & ((1u << lane) - 1u));
+              if (pos < 32)
+                st[pos] = ((unsigned long long)(uint32_t)cnt << 32) | (uint32_t)(0x7FFFFFFF - tk[e]);
+            }
+            nv += __popc(bal);
+          }
+          __syncwarp();
+          if (nv <= 32) {
+            // ascending sort of ~key == descending (count, -id)
+            unsigned long long key = lane < nv ? ~st[lane] : ~0ull;
+#pragma unroll
+            for (int kk = 2; kk <= 32; kk <<= 1) {
+#pragma unroll
+              for (int jj = kk >> 1; jj > 0; jj >>= 1) {
+                const unsigned long long o = __shfl_xor_sync(0xffffffffu, key, jj);
+                const bool asc = (lane & kk) == 0, low = (lane & jj) == 0;
+                key = (low == asc) ? (o < key ? o : key) : (o > key ? o : key);
+              }
+            }
+            taken = min(k, nv);
+            if (lane < taken) {
+              const unsigned long long kv = ~key;
+              const int32_t id = 0x7FFFFFFF - (int32_t)(uint32_t)kv;
+              scratch[j * k + lane] = ((int64_t)(kv >> 32) << 32) | (uint32_t)id;
+              atomicOr(bm + (id >> 5), 1u << (id & 31));
+            }
+          }
+          __syncwarp();
+          if (nv > 32)
           for (; taken < k; ++taken) {
             // best entry of this lane: count descending, id ascending
             unsigned long long best = 0;

@@ -42,7 +42,6 @@ constexpr int SH_THREADS = 512;
 constexpr int SH_WARPS = SH_THREADS / 32;
 constexpr int SH_MAX_CS = 8;                      // portable cluster size
 constexpr int SH_ILP = 8;                         // column positions per lane in flight
-constexpr int SH_V = 4;                           // 16-byte index vectors per lane in flight (count pass)
 constexpr int SH_CLAIM = 4;                       // columns per claim of the count pass
 constexpr int64_t SH_SMEM_CAP = 220 * 1024;      // dynamic shared memory per CTA (bitmap + prefixes)
 
@@ -244,47 +243,27 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       int cnt = 0;
       const long long start = wfill;
       bool staged = true;
-      // 16-byte loads from the 16-byte-aligned element below o: SH_V vectors
-      // (4 positions each) per lane in flight, kept positions staged in
-      // position order (lane-major inside a vector round)
-      const int64_t end = o + d;
-      for (int64_t b0 = d > 0 ? (o & ~int64_t(3)) : end; b0 < end; b0 += 128 * SH_V) {
-        uint4 w[SH_V];
+      for (int64_t i0 = 0; i0 < d; i0 += 32 * SH_ILP) {  // SH_ILP loads, then tests, in flight
+        uint32_t u[SH_ILP];
 #pragma unroll
-        for (int q = 0; q < SH_V; ++q) {
-          const int64_t e0 = b0 + (int64_t)(q * 32 + lane) * 4;
-          w[q] = e0 < end ? ldg_h4(P.indices + e0, pf) : make_uint4(~0u, ~0u, ~0u, ~0u);
+        for (int q = 0; q < SH_ILP; ++q) {
+          const int64_t i = i0 + q * 32 + lane;
+          u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
         }
-        uint32_t km[SH_V];
+        bool m[SH_ILP];
 #pragma unroll
-        for (int q = 0; q < SH_V; ++q) {
-          const int64_t e0 = b0 + (int64_t)(q * 32 + lane) * 4;
-          const uint32_t uu[4] = {w[q].x, w[q].y, w[q].z, w[q].w};
-          uint32_t mm = 0;
+        for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q]);
 #pragma unroll
-          for (int j = 0; j < 4; ++j)
-            if (e0 + j >= o && e0 + j < end && sh_member(cl, bm, bpc32, inv, uu[j])) mm |= 1u << j;
-          km[q] = mm;
-        }
-#pragma unroll
-        for (int q = 0; q < SH_V; ++q) {
-          const int nl = __popc(km[q]);
-          const int inc = warp_inclusive_scan<int>(nl);
-          const int n = __shfl_sync(0xffffffffu, inc, 31);
+        for (int q = 0; q < SH_ILP; ++q) {
+          const uint32_t bal = __ballot_sync(0xffffffffu, m[q]);
+          const int n = __popc(bal);
           cnt += n;
           if (staged && wfill + n > P.wcap) staged = false;  // this column is re-streamed below
           if (staged) {
-            if (nl) {
-              long long idx = wfill + inc - nl;
-              const int64_t e0 = b0 + (int64_t)(q * 32 + lane) * 4;
-              const uint32_t uu[4] = {w[q].x, w[q].y, w[q].z, w[q].w};
-#pragma unroll
-              for (int j = 0; j < 4; ++j)
-                if ((km[q] >> j) & 1u) {
-                  wst_r[idx] = (int32_t)sh_rank(cl, bm, gp, off8, ss, bpc32, inv, uu[j]);
-                  wst_e[idx] = e0 + j;
-                  ++idx;
-                }
+            if (m[q]) {
+              const long long idx = wfill + __popc(bal & ((1u << lane) - 1u));
+              wst_r[idx] = (int32_t)sh_rank(cl, bm, gp, off8, ss, bpc32, inv, u[q]);
+              wst_e[idx] = o + i0 + q * 32 + lane;
             }
             wfill += n;
           }
