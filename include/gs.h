@@ -235,6 +235,54 @@ gs_status gs_sample_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num
                             uint64_t rng_key, void* stream, gs_blocks** out);
 
 /* ------------------------------------------------------------------------ */
+/* Matrix-centric operators (Table 4).            */
+/* A gs_matrix is a materialised sub-matrix of A over GLOBAL node ids:        */
+/* local columns `cols` with a CSC indptr, and per entry its global row id,   */
+/* its edge id (position in the graph's indices) and an fp32 value (the edge  */
+/* weight, 1 if unweighted).  Device-resident, library-owned (allocator hook), */
+/* freed by gs_matrix_destroy.  These are the unfused operators a new         */
+/* algorithm composes; the samplers above fuse them.              */
+/* Calls that size an output (slice_columns, slice_rows, row_ids) synchronise */
+/* the stream once; the others only enqueue.  Node ids outside [0, N) ->      */
+/* GS_ERR_INDEX_OUT_OF_RANGE.                                                 */
+/* ------------------------------------------------------------------------ */
+typedef struct gs_matrix gs_matrix;
+typedef struct gs_matrix_view {
+  int64_t num_nodes, n_cols, nnz;
+  const int32_t* cols;    /* [n_cols]   global id of each local column        */
+  const int64_t* indptr;  /* [n_cols+1] CSC over the local columns            */
+  const int32_t* row;     /* [nnz]      global row id of each entry           */
+  const int64_t* eid;     /* [nnz]      edge id of each entry                 */
+  float* val;             /* [nnz]      entry value (mutable in place)        */
+} gs_matrix_view;
+enum { GS_OP_ADD = 0, GS_OP_SUB = 1, GS_OP_MUL = 2, GS_OP_DIV = 3, GS_OP_POW = 4 };
+/* A[:, cols] (Extract): cols device int32[n_cols] (duplicates allowed);
+ * each column's entries in the graph's CSC order.  *out may be NULL (a new
+ * object) or a previous result (reused). */
+gs_status gs_matrix_slice_columns(const gs_graph* g, const int32_t* cols, int64_t n_cols, void* stream,
+                                  gs_matrix** out);
+/* A[rows, :] (Extract): the entries whose row is in rows (device
+ * int32[n_rows]); same columns; *out must differ from in. */
+gs_status gs_matrix_slice_rows(const gs_matrix* in, const int32_t* rows, int64_t n_rows, void* stream,
+                               gs_matrix** out);
+/* A.sum(axis) (Compute; R1): axis 0 -> out device float[n_cols], the
+ * per-column sums; axis 1 -> out device float[num_nodes], the per-row sums by
+ * global row id (0 for rows without entries).  fp64 accumulation, one fp32
+ * rounding (R19). */
+gs_status gs_matrix_sum(const gs_matrix* m, int axis, float* out, void* stream);
+/* A.<op>(V, axis) in place (Compute): val = val op V[c] (axis 0,
+ * V device float[n_cols]) or val op V[row] (axis 1, V device float[num_nodes]).
+ * op: GS_OP_ADD/SUB/MUL/DIV/POW (IEEE fp32; POW = fp32(pow_fp64)). */
+gs_status gs_matrix_broadcast(gs_matrix* m, int op, const float* V, int axis, void* stream);
+/* A <op> v in place (Compute), e.g. A ** 2 (LADIES, Fig. 2). */
+gs_status gs_matrix_elementwise(gs_matrix* m, int op, float v, void* stream);
+/* A.row() (Finalize; R3): distinct row ids ascending into out (device
+ * int32, capacity >= min(nnz, num_nodes)); *n_out (host) = their number. */
+gs_status gs_matrix_row_ids(const gs_matrix* m, int32_t* out, int64_t* n_out, void* stream);
+gs_status gs_matrix_get_view(const gs_matrix* m, gs_matrix_view* out);
+void      gs_matrix_destroy(gs_matrix* m);
+
+/* ------------------------------------------------------------------------ */
 /* Layer-wise sampling (a1 + a2 + a4 + a6): FastGCN / LADIES.                 */
 /* ------------------------------------------------------------------------ */
 enum {

@@ -34,7 +34,10 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator"
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
            "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_saint_rw", "gs_sample_pinsage",
            "gs_sample_layerwise",
-           "gs_random_walk", "gs_walk_check"]
+           "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
+           "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
+           "gs_matrix_get_view", "gs_matrix_destroy"]
+OP_ADD, OP_SUB, OP_MUL, OP_DIV, OP_POW = 0, 1, 2, 3, 4
 
 
 class GSError(RuntimeError):
@@ -48,6 +51,12 @@ class _BlockView(ctypes.Structure):
                 ("col_map", ctypes.c_void_p), ("row_map", ctypes.c_void_p),
                 ("indptr", ctypes.c_void_p), ("row_local", ctypes.c_void_p),
                 ("eid", ctypes.c_void_p), ("val", ctypes.c_void_p), ("row_prob", ctypes.c_void_p)]
+
+
+class _MatrixView(ctypes.Structure):
+    _fields_ = [("num_nodes", ctypes.c_int64), ("n_cols", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("cols", ctypes.c_void_p), ("indptr", ctypes.c_void_p), ("row", ctypes.c_void_p),
+                ("eid", ctypes.c_void_p), ("val", ctypes.c_void_p)]
 
 
 class _GraphInfo(ctypes.Structure):
@@ -93,7 +102,7 @@ _pending = []
 def _drain():
     while _pending and _alive():
         kind, h = _pending.pop()
-        (_lib.gs_blocks_destroy if kind == "b" else _lib.gs_graph_destroy)(h)
+        {"b": _lib.gs_blocks_destroy, "g": _lib.gs_graph_destroy, "m": _lib.gs_matrix_destroy}[kind](h)
 
 
 def load_library(path: str = LIB_PATH):
@@ -119,6 +128,15 @@ def load_library(path: str = LIB_PATH):
     L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_pinsage.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, ctypes.c_float, u64,
                                     vp, ctypes.POINTER(vp)]
+    L.gs_matrix_slice_columns.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
+    L.gs_matrix_slice_rows.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
+    L.gs_matrix_sum.argtypes = [vp, i32, vp, vp]
+    L.gs_matrix_broadcast.argtypes = [vp, i32, vp, i32, vp]
+    L.gs_matrix_elementwise.argtypes = [vp, i32, ctypes.c_float, vp]
+    L.gs_matrix_row_ids.argtypes = [vp, vp, ctypes.POINTER(i64), vp]
+    L.gs_matrix_get_view.argtypes = [vp, ctypes.POINTER(_MatrixView)]
+    L.gs_matrix_destroy.argtypes = [vp]
+    L.gs_matrix_destroy.restype = None
     L.gs_sample_saint_rw.argtypes = [vp, vp, i64, i64, i64, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_layerwise.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
@@ -365,6 +383,83 @@ def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch
                 raise
     out._seeds = seeds
     return out
+
+
+class Matrix:
+    """A materialised sub-matrix of A over global ids (Table 4) behind
+    the gs_matrix_* C ABI; every operator runs in ops.cu."""
+
+    def __init__(self, handle, keep=None):
+        self._h = handle
+        self._keep = keep
+
+    @staticmethod
+    def slice_columns(g: "Graph", cols: torch.Tensor, stream=None) -> "Matrix":
+        """A[:, cols]."""
+        L = load_library()
+        _drain()
+        cols = cols.to(torch.int32).contiguous()
+        h = ctypes.c_void_p()
+        _check(L.gs_matrix_slice_columns(g.handle, _ptr(cols), cols.numel(), _stream_ptr(stream),
+                                         ctypes.byref(h)), "gs_matrix_slice_columns")
+        return Matrix(h, g)
+
+    def slice_rows(self, rows: torch.Tensor, stream=None) -> "Matrix":
+        """A[rows, :]."""
+        rows = rows.to(torch.int32).contiguous()
+        h = ctypes.c_void_p()
+        _check(_lib.gs_matrix_slice_rows(self._h, _ptr(rows), rows.numel(), _stream_ptr(stream),
+                                         ctypes.byref(h)), "gs_matrix_slice_rows")
+        return Matrix(h, self._keep)
+
+    def view(self) -> dict:
+        v = _MatrixView()
+        _check(_lib.gs_matrix_get_view(self._h, ctypes.byref(v)), "gs_matrix_get_view")
+        return {"num_nodes": v.num_nodes,
+                "cols": _dev_tensor(v.cols, v.n_cols, torch.int32, self),
+                "indptr": _dev_tensor(v.indptr, v.n_cols + 1, torch.int64, self),
+                "row": _dev_tensor(v.row, v.nnz, torch.int32, self),
+                "eid": _dev_tensor(v.eid, v.nnz, torch.int64, self),
+                "val": _dev_tensor(v.val, v.nnz, torch.float32, self)}
+
+    def sum(self, axis: int, stream=None) -> torch.Tensor:
+        """A.sum(axis): axis 0 per column, axis 1 dense per global row id."""
+        v = self.view()
+        n = v["cols"].numel() if axis == 0 else v["num_nodes"]
+        out = torch.empty(n, dtype=torch.float32, device="cuda")
+        _check(_lib.gs_matrix_sum(self._h, int(axis), _ptr(out), _stream_ptr(stream)), "gs_matrix_sum")
+        return out
+
+    def broadcast_(self, op: int, V: torch.Tensor, axis: int, stream=None) -> "Matrix":
+        """A.<op>(V, axis), in place."""
+        V = V.to(torch.float32).contiguous()
+        _check(_lib.gs_matrix_broadcast(self._h, int(op), _ptr(V), int(axis), _stream_ptr(stream)),
+               "gs_matrix_broadcast")
+        self._V = V
+        return self
+
+    def elementwise_(self, op: int, x: float, stream=None) -> "Matrix":
+        """A <op> x, in place."""
+        _check(_lib.gs_matrix_elementwise(self._h, int(op), float(x), _stream_ptr(stream)),
+               "gs_matrix_elementwise")
+        return self
+
+    def row_ids(self, stream=None) -> torch.Tensor:
+        """A.row(): distinct row ids ascending."""
+        v = self.view()
+        out = torch.empty(max(1, min(v["row"].numel(), v["num_nodes"])), dtype=torch.int32, device="cuda")
+        n = ctypes.c_int64()
+        _check(_lib.gs_matrix_row_ids(self._h, _ptr(out), ctypes.byref(n), _stream_ptr(stream)),
+               "gs_matrix_row_ids")
+        return out[:n.value]
+
+    def __del__(self):
+        try:
+            if getattr(self, "_h", None) and self._h.value and _alive():
+                _pending.append(("m", self._h))
+                self._h = None
+        except TypeError:  # interpreter shutdown: module globals already cleared
+            pass
 
 
 def sample_pinsage(g: Graph, seeds: torch.Tensor, topk, num_walks: int, walk_length: int,
