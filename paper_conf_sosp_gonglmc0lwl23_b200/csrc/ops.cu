@@ -248,9 +248,20 @@ __global__ void bcast_row_kernel(const int32_t* __restrict__ row, float* val, in
     val[i] = apply_op(op, val[i], __ldg(V + __ldcs(row + i)));
 }
 
+// 16-byte vectors (val is 256-byte aligned by the allocator), scalar tail
 __global__ void map_kernel(float* val, int64_t nnz, int op, float x) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
-    val[i] = apply_op(op, val[i], x);
+  float4* v4 = reinterpret_cast<float4*>(val);
+  const int64_t n4 = nnz >> 2;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+    float4 a = __ldcs(v4 + i);
+    a.x = apply_op(op, a.x, x);
+    a.y = apply_op(op, a.y, x);
+    a.z = apply_op(op, a.z, x);
+    a.w = apply_op(op, a.w, x);
+    __stcs(v4 + i, a);
+  }
+  const int64_t t = (n4 << 2) + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t < nnz) val[t] = apply_op(op, val[t], x);
 }
 
 // ---- row() ----
@@ -439,7 +450,7 @@ gs_status gs_matrix_broadcast(gs_matrix* m, int op, const float* V, int axis, vo
 gs_status gs_matrix_elementwise(gs_matrix* m, int op, float x, void* stream_) {
   if (!m || op < GS_OP_ADD || op > GS_OP_POW) return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_elementwise: bad argument");
   if (m->nnz == 0) return GS_OK;
-  map_kernel<<<grid_for(m->nnz, 256), 256, 0, (cudaStream_t)stream_>>>((float*)m->b_val.ptr, m->nnz, op, x);
+  map_kernel<<<grid_for((m->nnz + 3) / 4, 256), 256, 0, (cudaStream_t)stream_>>>((float*)m->b_val.ptr, m->nnz, op, x);
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
