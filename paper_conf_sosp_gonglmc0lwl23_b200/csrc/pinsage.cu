@@ -36,7 +36,7 @@ constexpr uint32_t TAG_PINSAGE = 7;
 constexpr int PS_THREADS = 512;
 constexpr int PS_WARPS = PS_THREADS / 32;
 constexpr int PS_SMEM = 48 * 1024;   // hash tables of one chunk (4 CTAs per SM fit)
-constexpr int PS_GROUP = 4;          // bitmap words per prefix entry
+constexpr int PS_GROUP = 4;          // bitmap words per prefix entry (one uint4; the relabel relies on it)
 constexpr int PS_ILP = 2;            // walks per thread in lockstep
 
 struct PSParams {
@@ -291,18 +291,27 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
       // ---- relabel: row_local = rank of the id, val = count ----
       int32_t* rowl = P.rowl[l] + ebase;
       float* val = P.val[l] + ebase;
-      for (long long j = warp; j < nF; j += PS_WARPS) {
-        const long long p0 = ip[j], n = ip[j + 1] - p0;
-        if (lane < n) {
-          const int64_t s = scratch[j * k + lane];
-          const int32_t id = (int32_t)(uint32_t)s;
-          const long long g = id >> 7;  // PS_GROUP words x 32 bits
-          int rank = __ldcg(gp + g);
-          const int wi = id >> 5;
-          for (int q = (int)(g * PS_GROUP); q < wi; ++q) rank += __popc(__ldcg(bm + q));
-          rank += __popc(__ldcg(bm + wi) & ((1u << (id & 31)) - 1u));
-          rowl[p0 + lane] = rank;
-          val[p0 + lane] = (float)(uint32_t)(s >> 32);
+      // flat over the (column, rank) slots so every lane works; the rank of
+      // an id = its group prefix + popc of the group's words below it (one
+      // 16-byte load of the group, issued beside the prefix load)
+      for (long long t = tid; t < nF * k; t += PS_THREADS) {
+        const long long j = t / k, r = t - j * k;
+        const long long p0 = ip[j];
+        if (r < ip[j + 1] - p0) {
+          const int64_t sv = scratch[t];
+          const int32_t id = (int32_t)(uint32_t)sv;
+          const long long g = id >> 7;  // PS_GROUP (4) words x 32 bits
+          const int base = __ldcg(gp + g);
+          const uint4 w4 = __ldcg(reinterpret_cast<const uint4*>(bm) + g);
+          const int q = (id >> 5) & 3;
+          const uint32_t below = (1u << (id & 31)) - 1u;
+          int rank = base;
+          rank += q > 0 ? __popc(w4.x) : __popc(w4.x & below);
+          if (q >= 1) rank += q > 1 ? __popc(w4.y) : __popc(w4.y & below);
+          if (q >= 2) rank += q > 2 ? __popc(w4.z) : __popc(w4.z & below);
+          if (q >= 3) rank += __popc(w4.w & below);
+          rowl[p0 + r] = rank;
+          val[p0 + r] = (float)(uint32_t)(sv >> 32);
         }
       }
       __syncthreads();

@@ -64,3 +64,22 @@ def test_sources_have_no_oracle_dependency():
                 txt = open(os.path.join(dirpath, f)).read()
                 for b in banned:
                     assert b not in txt, f"{f} references the oracle ({b})"
+
+
+def test_host_validation_new_entry_points(lib):
+    """GraphSAINT-RW, PinSAGE-style and the Table-4 operators reject bad
+    arguments on the host (no CUDA call)."""
+    out = ctypes.c_void_p()
+    assert lib.gs_sample_saint_rw(None, None, 0, 1, 0, 2, ctypes.c_uint64(0), None,
+                                  ctypes.byref(out)) == 1
+    k = (ctypes.c_int * 2)(5, 5)
+    assert lib.gs_sample_pinsage(None, None, 0, 1, 0, k, 2, 10, 3, ctypes.c_float(0.5),
+                                 ctypes.c_uint64(0), None, ctypes.byref(out)) == 1
+    assert lib.gs_matrix_slice_columns(None, None, 0, None, ctypes.byref(out)) == 1
+    assert lib.gs_matrix_slice_rows(None, None, 0, None, ctypes.byref(out)) == 1
+    assert lib.gs_matrix_sum(None, 0, None, None) == 1
+    assert lib.gs_matrix_broadcast(None, 0, None, 0, None) == 1
+    assert lib.gs_matrix_elementwise(None, 9, ctypes.c_float(1.0), None) == 1
+    n = ctypes.c_int64()
+    assert lib.gs_matrix_row_ids(None, None, ctypes.byref(n), None) == 1
+    assert b"null" in lib.gs_last_error()

@@ -107,3 +107,10 @@ def test_pinsage_pd_epoch(gs, oracle_lib):
             v = out.view(b, l)
             compare_block({k: (None if x is None else x.cpu().numpy()) for k, x in v.items()},
                           ref[l], f"pinsage PD batch {b} layer {l}")
+
+
+def test_pinsage_empty(gs, tiny):
+    g, G, O = tiny
+    out = gs.sample_pinsage(G, torch.zeros(0, dtype=torch.int32, device="cuda"), [3, 3], 4, 2, 0.5,
+                            batch_size=10)
+    assert out.to_host() == []

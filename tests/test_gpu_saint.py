@@ -106,3 +106,9 @@ def test_saint_pd_full_epoch(gs, oracle_lib):
         v = out.view(b, 0)
         compare_block({k: (None if x is None else x.cpu().numpy()) for k, x in v.items()}, ref,
                       f"saint PD batch {b}")
+
+
+def test_saint_empty(gs, tiny):
+    g, G, O = tiny
+    out = gs.sample_saint_rw(G, torch.zeros(0, dtype=torch.int32, device="cuda"), 3, batch_size=10)
+    assert out.to_host() == []
