@@ -273,3 +273,13 @@ def degree_stats(indptr) -> dict:
         "median": float(np.median(d)), "p90": float(np.percentile(d, 90)),
         "p99": float(np.percentile(d, 99)), "max": int(d.max()) if d.size else 0,
     }
+
+
+def make_grid_matrix(stream: int, rows: int, cols: int, levels: int = 4, device="cpu") -> torch.Tensor:
+    """Seeded synthetic dense matrix (PASS features X and projections W1, W2),
+    bf16 with values on the grid {-levels..levels} / levels: every product of two
+    entries is a multiple of 1/levels^2 and every sum the path forms stays exactly
+    representable (R29), so results do not depend on summation order."""
+    idx = torch.arange(rows * cols, device=device, dtype=torch.int64)
+    q = (hash_u32(stream, idx) % (2 * levels + 1)) - levels
+    return (q.to(torch.float32) / levels).to(torch.bfloat16).reshape(rows, cols)
