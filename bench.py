@@ -62,6 +62,11 @@ WORKLOADS = {
     "saint_pd": dict(kind="saint", graph="PD", walk_length=2, batch=3000, seeds=None,
                      desc="GraphSAINT-RW 3000 roots x walk length 2 + induce per subgraph, every "
                           "node a root once per epoch (817 subgraphs), PD-shaped"),
+    "pass_full_pd": dict(kind="pass_full", graph="PDw", fanouts=[10, 10], batch=1024,
+                         seeds=196_615, F=128, H=32, W3=[0.2, -0.4, 0.9],
+                         desc="PASS full bias (A1, A2 SDDMM of 128-d features projected to 32-d, "
+                              "A3, softmax(W3) mix, relu) for every edge + weighted A-Res [10,10], "
+                              "batch 1024, full epoch, PD-shaped weighted"),
     "pinsage_pd": dict(kind="pinsage", graph="PD", topk=[10, 10], num_walks=10, walk_length=3,
                        restart=0.5, batch=1024, seeds=196_615,
                        desc="PinSAGE-style top-k [10,10] of 10 restart walks (<= 3 steps, restart "
@@ -360,6 +365,14 @@ def run_gpu(args, wl, world, rank, device):
     else:
         bs = wl["batch"]
         nunits = (inputs.numel() + bs - 1) // bs
+    if kind == "pass_full":
+        import synth
+        N = g["indptr"].numel() - 1
+        PX = synth.make_grid_matrix(21, N, wl["F"], device=device)
+        PW1 = synth.make_grid_matrix(22, wl["F"], wl["H"], device=device)
+        PW2 = synth.make_grid_matrix(23, wl["F"], wl["H"], device=device)
+        att = torch.empty(g["indices"].numel(), dtype=torch.float32, device=device)
+        Ga = gs.Graph(g["indptr"], g["indices"], g["weights"])
         wbase = gdist.weak_batch_base(rank, nunits)
         L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer")
                                                        or wl.get("topk"))
@@ -375,6 +388,13 @@ def run_gpu(args, wl, world, rank, device):
             gs.sample_shadow(G, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
                              bias_mode=wl["bias"], rng_key=key, stream=stream, out=out,
                              retry=False)
+        elif kind == "pass_full":
+            # Fig. 3(c): the learned bias of every edge (W1..W3 change per
+            # training step, so it is recomputed every epoch), then line 10
+            gs.pass_attention(G, PX, PW1, PW2, wl["W3"], stream=stream, out=att)
+            Ga.set_weights(att, stream=stream)
+            gs.sample_neighbors(Ga, x, wl["fanouts"], batch_size=bs, batch_index_base=wbase,
+                                bias_mode=1, rng_key=key, stream=stream, out=out)
         elif kind == "pinsage":
             gs.sample_pinsage(G, x, wl["topk"], wl["num_walks"], wl["walk_length"], wl["restart"],
                               batch_size=bs, batch_index_base=wbase, rng_key=key, stream=stream,
@@ -420,6 +440,18 @@ def run_gpu(args, wl, world, rank, device):
             return (edges * (32 + 4) + walkers * (32 + 4) + 32 * straddle, edges,
                     edges + walkers + straddle)
         out.sync()
+        if kind == "pass_full":
+            # sampling as weighted node-wise (att streamed by the A-Res select) +
+            # the bias: per edge 4 (index) + 4 (w) + 4 (att written) + 8H (the
+            # projected row of u, 2H fp32, a random gather); per node 8H (its own
+            # row) + 16 (indptr pair) + 4 (colsum); the GEMM reads X (2F per
+            # node) and writes the projections (8H per node)
+            tot, e, rnd = _blocks_byte_model(out, g, "nodewise", False, L, weighted_select=True)
+            N = g["indptr"].numel() - 1
+            nnz = g["indices"].numel()
+            H = wl["H"]
+            tot += nnz * (12 + 8 * H) + N * (8 * H + 20) + N * (2 * wl["F"] + 8 * H)
+            return tot, e, rnd + N
         if kind == "pinsage":
             # per frontier column: 4 (id) + its walks' steps, each one random
             # indptr-pair sector + one random index sector (32 + 32); the steps
@@ -550,6 +582,7 @@ def run_gpu(args, wl, world, rank, device):
 
 KERNEL_OF = {"nodewise": "gsb::nodewise_wave_kernel", "shadow": "gsb::shadow_induce_kernel",
              "saint": "gsb::shadow_induce_kernel", "pinsage": "gsb::pinsage_kernel",
+             "pass_full": "gsb::pass_att_kernel + gsb::nodewise_wave_kernel<1>",
              "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
 
 
@@ -587,7 +620,7 @@ def main():
     r = run_gpu(args, wl, world, rank, device)
     if rank == 0:
         cpu = None
-        if not args.no_cpu_baseline and world == 1:
+        if not args.no_cpu_baseline and world == 1 and wl["kind"] != "pass_full":
             cpu, _, _ = oracle_rate(r["graph"], r["inputs"], wl)
         kind = wl["kind"]
         line = {
@@ -617,7 +650,7 @@ def main():
                                      "(profiles/r01_random_access_probe.md)"}},
             "e2e": {"value": r["e2e_value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d"],
                     "d2h_bytes_per_step": r["d2h"]},
-            "gpu_launches": args.steps * (2 if kind in ("shadow", "saint") else 1),
+            "gpu_launches": args.steps * {"shadow": 2, "saint": 2, "pass_full": 3}.get(kind, 1),
             "clocks": r["clocks"],
         }
         if kind == "nodewise":

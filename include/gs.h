@@ -91,6 +91,11 @@ typedef struct gs_graph_info {
   const float* weights;    /* device or NULL */
 } gs_graph_info;
 gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out);
+/* Replaces the edge weights (device float[num_edges]) and recomputes the a0
+ * column sums; copied unless flags has GS_GRAPH_BORROW (then used in place and
+ * kept alive by the caller).  Structure, validation and derived index arrays
+ * are unchanged.  Used to sample over a computed bias (PASS att, R29). */
+gs_status gs_graph_set_weights(gs_graph* g, const float* weights, uint32_t flags, void* stream);
 void gs_graph_destroy(gs_graph* g);
 
 /* ------------------------------------------------------------------------ */
@@ -281,6 +286,22 @@ gs_status gs_matrix_elementwise(gs_matrix* m, int op, float v, void* stream);
 gs_status gs_matrix_row_ids(const gs_matrix* m, int32_t* out, int64_t* n_out, void* stream);
 gs_status gs_matrix_get_view(const gs_matrix* m, gs_matrix_view* out);
 void      gs_matrix_destroy(gs_matrix* m);
+
+/* PASS learned bias in full (Fig. 3(c) lines 3-9; DESIGN R29; SURVEY
+ * 8(f) f2).  att[e] for every edge e = (u -> v) of g (weight w_e, 1 if unweighted):
+ *   A1 = w_e <X_u W1, X_v W1>, A2 = w_e <X_u W2, X_v W2>, A3 = fp32(w_e / colsum_v),
+ *   att = fp32(relu((s0 A1 + s1 A2) + s2 A3)), s = softmax(W3) (fp64).
+ *   X   device bf16 [num_nodes][F] row-major (node features)
+ *   W1, W2 device bf16 [F][H] row-major, H in {8, 16, 32, 64}
+ *   W3  host float[3] (mixing logits)
+ *   att device float[num_edges] (caller-owned), CSC order
+ * The projections X [W1 | W2] are one dense bf16 GEMM on the tensor cores
+ * (cuBLAS, fp32 accumulate); the SDDMM + mix is a hand-written kernel.  Exact
+ * (order-independent) for the grid-valued inputs of R29.  Line 10
+ * (individual_sample(k, att)) = gs_graph_set_weights(att) + gs_sample_neighbors
+ * with GS_W_EDGE.  Stream-ordered; workspace through the allocator hook. */
+gs_status gs_pass_attention(const gs_graph* g, const void* X, int F, const void* W1, const void* W2,
+                            int H, const float* W3, void* stream, float* att);
 
 /* ------------------------------------------------------------------------ */
 /* Layer-wise sampling (a1 + a2 + a4 + a6): FastGCN / LADIES.                 */

@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libgsb200.so")
-SOURCES = ["capi.cu", "nodewise_wave.cu", "shadow.cu", "layerwise.cu", "layerwise_bm.cu", "walk.cu", "pack.cu", "pinsage.cu", "ops.cu"]
+SOURCES = ["capi.cu", "nodewise_wave.cu", "shadow.cu", "layerwise.cu", "layerwise_bm.cu", "walk.cu", "pack.cu", "pinsage.cu", "ops.cu", "pass_att.cu"]
 HEADERS = ["common.cuh", "gs_internal.h", "nodewise_common.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-fmad=false",
@@ -44,7 +44,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if force or _stale(LIB, objs):
         tmp = LIB + ".tmp"
         subprocess.check_call([NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a",
-                               "-o", tmp] + objs)
+                               "-o", tmp] + objs + ["-lcublas", "-Xlinker", "-rpath=/usr/local/cuda/lib64"])
         os.replace(tmp, LIB)
     return LIB
 

@@ -268,6 +268,28 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
   return GS_OK;
 }
 
+gs_status gs_graph_set_weights(gs_graph* g, const float* weights, uint32_t flags, void* stream_) {
+  if (!g || (!weights && g->num_edges > 0))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_graph_set_weights: null pointer");
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (flags & GS_GRAPH_BORROW) {
+    g->weights = const_cast<float*>(weights);
+  } else {
+    if (!g->b_weights.ensure(g->al, (size_t)std::max<int64_t>(g->num_edges, 1) * 4, stream))
+      return fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_set_weights: device allocation failed");
+    g->weights = (float*)g->b_weights.ptr;
+    if (g->num_edges)
+      GS_CUDA_TRY(cudaMemcpyAsync(g->weights, weights, g->num_edges * 4, cudaMemcpyDeviceToDevice, stream));
+  }
+  if (!g->b_colsum.ensure(g->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
+    return fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_set_weights: device allocation failed");
+  g->colsum = (float*)g->b_colsum.ptr;
+  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((g->num_nodes + 7) / 8, (int64_t)num_sms() * 16));
+  if (g->num_nodes > 0) colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, g->num_nodes, g->colsum);
+  GS_CUDA_TRY(cudaGetLastError());
+  return GS_OK;
+}
+
 gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out) {
   if (!g || !out) return fail(GS_ERR_INVALID_ARGUMENT, "gs_graph_get_info: null pointer");
   out->num_nodes = g->num_nodes;

@@ -1,0 +1,157 @@
+// pass_att.cu -- PASS's learned sampling bias in full (Fig. 3(c) lines 3-9,
+// P:185-226; R29).  For every edge e = (u -> v) with weight w_e:
+//   A1 = w_e <X_u W1, X_v W1>,  A2 = w_e <X_u W2, X_v W2>,  A3 = fp32(w_e / colsum_v),
+//   att = relu((s0 A1 + s1 A2) + s2 A3),  s = softmax(W3).
+// Every term depends on the edge alone, so att is computed once per set of
+// projection weights for the whole graph (the paper's pre-processing rule (2),
+// P:300) and line 10's individual_sample(k, att) is the weighted A-Res sampler
+// over att (gs_graph_set_weights + gs_sample_neighbors(GS_W_EDGE)).
+//
+//   1. projections P = X [W1 | W2] : [N, F] x [F, 2H] bf16 -> fp32, one plain
+//      dense GEMM on the tensor cores (cuBLAS, bf16 inputs, fp32 accumulate);
+//      the grid-valued inputs of R29 make every partial sum exact.
+//   2. SDDMM + mix: a warp per column v keeps P_v (2H floats) in shared memory;
+//      each lane takes one in-edge, gathers P_u as 16-byte vectors (one random
+//      2H*4-byte row per edge), forms both dot products in fp64 (exact, any
+//      order), A3 from the a0 column sum, mixes in fp64 and writes fp32 att.
+#include <cublas_v2.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <mutex>
+
+#include "common.cuh"
+#include "gs_internal.h"
+
+namespace gsb {
+
+constexpr int PA_THREADS = 256;
+constexpr int PA_WARPS = PA_THREADS / 32;
+constexpr int PA_MAX_H = 64;
+
+template <int H2>  // 2H floats per projected row
+__global__ void __launch_bounds__(PA_THREADS) pass_att_kernel(const int64_t* __restrict__ indptr,
+                                                              const int32_t* __restrict__ indices,
+                                                              const float* __restrict__ w,
+                                                              const float* __restrict__ colsum,
+                                                              const float* __restrict__ P, int64_t N,
+                                                              double s0, double s1, double s2,
+                                                              float* __restrict__ att) {
+  __shared__ __align__(16) float pv[PA_WARPS][H2];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  constexpr int H = H2 / 2;
+  for (int64_t v = warp; v < N; v += nwarps) {
+    const int64_t o = __ldg(indptr + v), d = __ldg(indptr + v + 1) - o;
+    if (d == 0) continue;
+    __syncwarp();
+    for (int i = lane; i < H2; i += 32) pv[wl][i] = __ldg(P + v * H2 + i);
+    __syncwarp();
+    const float cs = w ? __ldg(colsum + v) : (float)d;
+    for (int64_t i = lane; i < d; i += 32) {
+      const int64_t e = o + i;
+      const int32_t u = __ldg(indices + e);
+      const float we = w ? __ldg(w + e) : 1.0f;
+      const float4* pu = reinterpret_cast<const float4*>(P + (int64_t)u * H2);
+      double d1 = 0.0, d2 = 0.0;
+#pragma unroll
+      for (int q = 0; q < H / 4; ++q) {
+        const float4 a = __ldg(pu + q);
+        d1 += (double)a.x * pv[wl][4 * q] + (double)a.y * pv[wl][4 * q + 1] +
+              (double)a.z * pv[wl][4 * q + 2] + (double)a.w * pv[wl][4 * q + 3];
+      }
+#pragma unroll
+      for (int q = H / 4; q < H2 / 4; ++q) {
+        const float4 a = __ldg(pu + q);
+        d2 += (double)a.x * pv[wl][4 * q] + (double)a.y * pv[wl][4 * q + 1] +
+              (double)a.z * pv[wl][4 * q + 2] + (double)a.w * pv[wl][4 * q + 3];
+      }
+      const double a1 = (double)we * d1, a2 = (double)we * d2;
+      const double a3 = (double)__fdiv_rn(we, cs);
+      const double mix = (s0 * a1 + s1 * a2) + s2 * a3;
+      att[e] = mix > 0.0 ? (float)mix : 0.0f;  // relu (NaN -> 0)
+    }
+  }
+}
+
+static cublasHandle_t pa_handle() {
+  static cublasHandle_t h = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    if (cublasCreate(&h) != CUBLAS_STATUS_SUCCESS) h = nullptr;
+  });
+  return h;
+}
+
+static std::mutex pa_mutex;  // the shared handle's stream binding
+
+}  // namespace gsb
+
+using namespace gsb;
+
+extern "C" gs_status gs_pass_attention(const gs_graph* g, const void* X, int F, const void* W1,
+                                       const void* W2, int H, const float* W3, void* stream_,
+                                       float* att) {
+  if (!g || !X || !W1 || !W2 || !W3 || (!att && g && g->num_edges > 0))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_pass_attention: null pointer");
+  if (F <= 0 || (H != 8 && H != 16 && H != 32 && H != PA_MAX_H))
+    return fail(GS_ERR_NOT_SUPPORTED, "gs_pass_attention: F > 0 and H in {8, 16, 32, 64} required");
+  cudaStream_t s = (cudaStream_t)stream_;
+  const int64_t N = g->num_nodes, H2 = 2 * (int64_t)H;
+  // softmax(W3) in fp64, libm exp, sum order (e0 + e1) + e2 (R29)
+  const double m = std::max((double)W3[0], std::max((double)W3[1], (double)W3[2]));
+  const double e0 = exp((double)W3[0] - m), e1 = exp((double)W3[1] - m), e2 = exp((double)W3[2] - m);
+  const double tot = (e0 + e1) + e2;
+  const double s0 = e0 / tot, s1 = e1 / tot, s2 = e2 / tot;
+  if (N == 0 || g->num_edges == 0) return GS_OK;
+  const Allocator al = g->al;
+  DevBuf wc, P;
+  if (!wc.ensure(al, (size_t)F * H2 * 2, s) || !P.ensure(al, (size_t)N * H2 * 4 + 16, s))
+    return fail(GS_ERR_OUT_OF_MEMORY, "gs_pass_attention: device allocation failed");
+  gs_status st = GS_OK;
+  // [W1 | W2] as one row-major [F, 2H] bf16 operand
+  cudaError_t ce = cudaMemcpy2DAsync(wc.ptr, H2 * 2, W1, (size_t)H * 2, (size_t)H * 2, F,
+                                     cudaMemcpyDeviceToDevice, s);
+  if (ce == cudaSuccess)
+    ce = cudaMemcpy2DAsync((char*)wc.ptr + H * 2, H2 * 2, W2, (size_t)H * 2, (size_t)H * 2, F,
+                           cudaMemcpyDeviceToDevice, s);
+  if (ce != cudaSuccess) st = cuda_fail(ce, "gs_pass_attention: weight copy");
+  if (st == GS_OK) {
+    // row-major P[N, 2H] = X[N, F] Wc[F, 2H]  <=>  column-major P^T = Wc^T X^T
+    cublasHandle_t h = pa_handle();
+    if (!h) {
+      st = fail(GS_ERR_CUDA, "gs_pass_attention: cublasCreate failed");
+    } else {
+      std::lock_guard<std::mutex> lk(pa_mutex);
+      const float one = 1.0f, zero = 0.0f;
+      cublasStatus_t cs = cublasSetStream(h, s);
+      if (cs == CUBLAS_STATUS_SUCCESS)
+        cs = cublasGemmEx(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)H2, (int)N, F, &one, wc.ptr, CUDA_R_16BF,
+                          (int)H2, X, CUDA_R_16BF, F, &zero, P.ptr, CUDA_R_32F, (int)H2,
+                          CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT);
+      if (cs != CUBLAS_STATUS_SUCCESS) st = fail(GS_ERR_CUDA, "gs_pass_attention: cublasGemmEx failed (%d)", (int)cs);
+    }
+  }
+  if (st == GS_OK) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((N + PA_WARPS - 1) / PA_WARPS, (int64_t)sms * 8));
+    const float* Pp = (const float*)P.ptr;
+    switch (H) {
+      case 8: pass_att_kernel<16><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
+      case 16: pass_att_kernel<32><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
+      case 32: pass_att_kernel<64><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
+      default: pass_att_kernel<128><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
+    }
+    ce = cudaGetLastError();
+    if (ce != cudaSuccess) st = cuda_fail(ce, "pass_att_kernel launch");
+  }
+  wc.reset(al, s);
+  P.reset(al, s);
+  return st;
+}

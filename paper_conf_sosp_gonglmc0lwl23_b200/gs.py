@@ -36,7 +36,7 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator"
            "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
            "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
-           "gs_matrix_get_view", "gs_matrix_destroy"]
+           "gs_matrix_get_view", "gs_matrix_destroy", "gs_pass_attention", "gs_graph_set_weights"]
 OP_ADD, OP_SUB, OP_MUL, OP_DIV, OP_POW = 0, 1, 2, 3, 4
 
 
@@ -128,6 +128,8 @@ def load_library(path: str = LIB_PATH):
     L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_pinsage.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, ctypes.c_float, u64,
                                     vp, ctypes.POINTER(vp)]
+    L.gs_pass_attention.argtypes = [vp, vp, i32, vp, vp, i32, vp, vp, vp]
+    L.gs_graph_set_weights.argtypes = [vp, vp, ctypes.c_uint32, vp]
     L.gs_matrix_slice_columns.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_slice_rows.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_sum.argtypes = [vp, i32, vp, vp]
@@ -242,6 +244,14 @@ class Graph:
     @property
     def handle(self):
         return self._h
+
+    def set_weights(self, weights: torch.Tensor, borrow: bool = True, stream=None) -> "Graph":
+        """Replaces the edge weights (e.g. PASS att) and recomputes the a0 column sums."""
+        weights = weights.to(torch.float32).contiguous()
+        _check(load_library().gs_graph_set_weights(self._h, _ptr(weights), GRAPH_BORROW if borrow else 0,
+                                                   _stream_ptr(stream)), "gs_graph_set_weights")
+        self._w = weights
+        return self
 
     def __del__(self):
         try:
@@ -382,6 +392,23 @@ def sample_shadow(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch
             if e.status != 7 or attempt == 2:
                 raise
     out._seeds = seeds
+    return out
+
+
+def pass_attention(g: "Graph", X: torch.Tensor, W1: torch.Tensor, W2: torch.Tensor, W3,
+                   stream=None, out: torch.Tensor = None) -> torch.Tensor:
+    """PASS learned bias att[e] for every edge (Fig. 3(c) lines 3-9; DESIGN R29)
+    through gs_pass_attention.  X [N, F], W1/W2 [F, H] bf16 on the device."""
+    L = load_library()
+    X = X.to(torch.bfloat16).contiguous()
+    W1 = W1.to(torch.bfloat16).contiguous()
+    W2 = W2.to(torch.bfloat16).contiguous()
+    nnz = g.num_edges
+    if out is None:
+        out = torch.empty(nnz, dtype=torch.float32, device=X.device)
+    w3 = (ctypes.c_float * 3)(*[float(x) for x in W3])
+    _check(L.gs_pass_attention(g.handle, _ptr(X), X.shape[1], _ptr(W1), _ptr(W2), W1.shape[1], w3,
+                               _stream_ptr(stream), _ptr(out)), "gs_pass_attention")
     return out
 
 

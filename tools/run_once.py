@@ -25,6 +25,17 @@ if wl["kind"] in ("nodewise", "shadow"):
         else:
             gs.sample_shadow(G, seeds, wl["fanouts"], batch_size=wl["batch"], bias_mode=wl["bias"],
                              rng_key=i, out=out)
+elif wl["kind"] == "pass_full":
+    N = g["indptr"].numel() - 1
+    X = synth.make_grid_matrix(21, N, wl["F"], device="cuda")
+    W1 = synth.make_grid_matrix(22, wl["F"], wl["H"], device="cuda")
+    W2 = synth.make_grid_matrix(23, wl["F"], wl["H"], device="cuda")
+    Ga = gs.Graph(g["indptr"], g["indices"], g["weights"])
+    seeds = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
+    for i in range(reps):
+        att = gs.pass_attention(G, X, W1, W2, wl["W3"])
+        Ga.set_weights(att)
+        gs.sample_neighbors(Ga, seeds, wl["fanouts"], batch_size=wl["batch"], bias_mode=1, rng_key=i, out=out)
 elif wl["kind"] == "pinsage":
     seeds = synth.make_seeds(wl["graph"], wl["seeds"], device="cuda")
     for i in range(reps):
