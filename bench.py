@@ -365,6 +365,9 @@ def run_gpu(args, wl, world, rank, device):
     else:
         bs = wl["batch"]
         nunits = (inputs.numel() + bs - 1) // bs
+        wbase = gdist.weak_batch_base(rank, nunits)
+        L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer")
+                                                       or wl.get("topk"))
     if kind == "pass_full":
         import synth
         N = g["indptr"].numel() - 1
@@ -373,9 +376,6 @@ def run_gpu(args, wl, world, rank, device):
         PW2 = synth.make_grid_matrix(23, wl["F"], wl["H"], device=device)
         att = torch.empty(g["indices"].numel(), dtype=torch.float32, device=device)
         Ga = gs.Graph(g["indptr"], g["indices"], g["weights"])
-        wbase = gdist.weak_batch_base(rank, nunits)
-        L = 1 if kind in ("shadow", "saint") else len(wl.get("fanouts") or wl.get("n_per_layer")
-                                                       or wl.get("topk"))
 
     def step(i, x=None):
         x = inputs if x is None else x
