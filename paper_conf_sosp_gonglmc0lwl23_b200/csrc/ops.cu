@@ -408,7 +408,8 @@ gs_status gs_matrix_slice_rows(const gs_matrix* in, const int32_t* rows, int64_t
 }
 
 gs_status gs_matrix_sum(const gs_matrix* m, int axis, float* out, void* stream_) {
-  if (!m || !out || (axis != 0 && axis != 1)) return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_sum: bad argument");
+  if (!m || (axis != 0 && axis != 1) || (!out && (axis == 0 ? m->n_cols : m->num_nodes) > 0))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_sum: bad argument");
   cudaStream_t s = (cudaStream_t)stream_;
   if (axis == 0) {
     if (m->n_cols > 0) {

@@ -58,17 +58,16 @@ __global__ void __launch_bounds__(PA_THREADS) pass_att_kernel(const int64_t* __r
       const float we = w ? __ldg(w + e) : 1.0f;
       const float4* pu = reinterpret_cast<const float4*>(P + (int64_t)u * H2);
       double d1 = 0.0, d2 = 0.0;
+      const float4* pv4 = reinterpret_cast<const float4*>(pv[wl]);
 #pragma unroll
       for (int q = 0; q < H / 4; ++q) {
-        const float4 a = __ldg(pu + q);
-        d1 += (double)a.x * pv[wl][4 * q] + (double)a.y * pv[wl][4 * q + 1] +
-              (double)a.z * pv[wl][4 * q + 2] + (double)a.w * pv[wl][4 * q + 3];
+        const float4 a = __ldg(pu + q), b = pv4[q];
+        d1 += (double)a.x * b.x + (double)a.y * b.y + (double)a.z * b.z + (double)a.w * b.w;
       }
 #pragma unroll
       for (int q = H / 4; q < H2 / 4; ++q) {
-        const float4 a = __ldg(pu + q);
-        d2 += (double)a.x * pv[wl][4 * q] + (double)a.y * pv[wl][4 * q + 1] +
-              (double)a.z * pv[wl][4 * q + 2] + (double)a.w * pv[wl][4 * q + 3];
+        const float4 a = __ldg(pu + q), b = pv4[q];
+        d2 += (double)a.x * b.x + (double)a.y * b.y + (double)a.z * b.z + (double)a.w * b.w;
       }
       const double a1 = (double)we * d1, a2 = (double)we * d2;
       const double a3 = (double)__fdiv_rn(we, cs);
