@@ -11,9 +11,9 @@
 //      dense GEMM on the tensor cores (cuBLAS, bf16 inputs, fp32 accumulate);
 //      the grid-valued inputs of R29 make every partial sum exact.
 //   2. SDDMM + mix: a warp per column v keeps P_v (2H floats) in shared memory;
-//      each lane takes one in-edge, gathers P_u as 16-byte vectors (one random
-//      2H*4-byte row per edge), forms both dot products in fp64 (exact, any
-//      order), A3 from the a0 column sum, mixes in fp64 and writes fp32 att.
+//      8 lanes per in-edge gather P_u as 16-byte vectors (one random 2H*4-byte
+//      row per edge), form both dot products in fp64 (exact, any order), A3
+//      from the a0 column sum, mix in fp64 and write fp32 att.
 #include <cublas_v2.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -31,6 +31,7 @@ namespace gsb {
 constexpr int PA_THREADS = 256;
 constexpr int PA_WARPS = PA_THREADS / 32;
 constexpr int PA_MAX_H = 64;
+constexpr int PA_EILP = 4;  // edge steps (4 edges each) per warp in flight
 
 template <int H2>  // 2H floats per projected row
 __global__ void __launch_bounds__(PA_THREADS) pass_att_kernel(const int64_t* __restrict__ indptr,
@@ -45,6 +46,7 @@ __global__ void __launch_bounds__(PA_THREADS) pass_att_kernel(const int64_t* __r
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   constexpr int H = H2 / 2;
+  constexpr int QL = (H2 / 4 + 7) / 8;  // 16-byte vectors per lane per edge
   for (int64_t v = warp; v < N; v += nwarps) {
     const int64_t o = __ldg(indptr + v), d = __ldg(indptr + v + 1) - o;
     if (d == 0) continue;
@@ -52,27 +54,58 @@ __global__ void __launch_bounds__(PA_THREADS) pass_att_kernel(const int64_t* __r
     for (int i = lane; i < H2; i += 32) pv[wl][i] = __ldg(P + v * H2 + i);
     __syncwarp();
     const float cs = w ? __ldg(colsum + v) : (float)d;
-    for (int64_t i = lane; i < d; i += 32) {
-      const int64_t e = o + i;
-      const int32_t u = __ldg(indices + e);
-      const float we = w ? __ldg(w + e) : 1.0f;
-      const float4* pu = reinterpret_cast<const float4*>(P + (int64_t)u * H2);
-      double d1 = 0.0, d2 = 0.0;
-      const float4* pv4 = reinterpret_cast<const float4*>(pv[wl]);
+    // 8 lanes per edge, 4 edges per warp step: a load instruction covers 4
+    // projected rows as whole 128-byte lines (lane-per-edge gathers touch 32
+    // lines per instruction); the 8 partial sums of each dot are combined by
+    // xor-shuffles (exact in fp64, so the combination order is immaterial)
+    const int slot = lane >> 3, sub = lane & 7;
+    const float4* pv4 = reinterpret_cast<const float4*>(pv[wl]);
+    for (int64_t i0 = 0; i0 < d; i0 += 4 * PA_EILP) {  // PA_EILP edge steps in flight
+      int64_t e[PA_EILP];
+      int32_t u[PA_EILP];
 #pragma unroll
-      for (int q = 0; q < H / 4; ++q) {
-        const float4 a = __ldg(pu + q), b = pv4[q];
-        d1 += (double)a.x * b.x + (double)a.y * b.y + (double)a.z * b.z + (double)a.w * b.w;
+      for (int r = 0; r < PA_EILP; ++r) {
+        const int64_t i = i0 + r * 4 + slot;
+        e[r] = i < d ? o + i : -1;
+        u[r] = e[r] >= 0 ? __ldg(indices + e[r]) : 0;
+      }
+      float4 a[PA_EILP][QL];
+#pragma unroll
+      for (int r = 0; r < PA_EILP; ++r) {
+        const float4* pu = reinterpret_cast<const float4*>(P + (int64_t)u[r] * H2);
+#pragma unroll
+        for (int j = 0; j < QL; ++j) {
+          const int q = sub + 8 * j;
+          a[r][j] = (e[r] >= 0 && q < H2 / 4) ? __ldg(pu + q) : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
       }
 #pragma unroll
-      for (int q = H / 4; q < H2 / 4; ++q) {
-        const float4 a = __ldg(pu + q), b = pv4[q];
-        d2 += (double)a.x * b.x + (double)a.y * b.y + (double)a.z * b.z + (double)a.w * b.w;
+      for (int r = 0; r < PA_EILP; ++r) {
+        double d1 = 0.0, d2 = 0.0;
+#pragma unroll
+        for (int j = 0; j < QL; ++j) {
+          const int q = sub + 8 * j;
+          if (q < H2 / 4) {
+            const float4 b = pv4[q];
+            const double t = (double)a[r][j].x * b.x + (double)a[r][j].y * b.y +
+                             (double)a[r][j].z * b.z + (double)a[r][j].w * b.w;
+            if (q < H / 4) d1 += t;
+            else d2 += t;
+          }
+        }
+#pragma unroll
+        for (int off = 4; off > 0; off >>= 1) {
+          d1 += __shfl_xor_sync(0xffffffffu, d1, off);
+          d2 += __shfl_xor_sync(0xffffffffu, d2, off);
+        }
+        if (e[r] >= 0 && sub == 0) {
+          const float we = w ? __ldg(w + e[r]) : 1.0f;
+          const double a1 = (double)we * d1, a2 = (double)we * d2;
+          const double a3 = (double)__fdiv_rn(we, cs);
+          const double mix = (s0 * a1 + s1 * a2) + s2 * a3;
+          att[e[r]] = mix > 0.0 ? (float)mix : 0.0f;  // relu (NaN -> 0)
+        }
       }
-      const double a1 = (double)we * d1, a2 = (double)we * d2;
-      const double a3 = (double)__fdiv_rn(we, cs);
-      const double mix = (s0 * a1 + s1 * a2) + s2 * a3;
-      att[e] = mix > 0.0 ? (float)mix : 0.0f;  // relu (NaN -> 0)
     }
   }
 }
