@@ -47,7 +47,7 @@ struct WalkParams {
 // ~log log n steps instead of log n; after WALK_INTERP probes the remaining
 // interval is bisected.  The probe order changes only the bytes read, never
 // the answer.
-constexpr int WALK_INTERP = 3;
+constexpr int WALK_INTERP = 8;
 __device__ __forceinline__ bool in_sorted(const int32_t* __restrict__ a, int64_t n, int32_t x) {
   if (n <= 0) return false;
   int64_t lo = 0, hi = n - 1;
