@@ -47,6 +47,11 @@ WORKLOADS = {
                          desc="GraphSAGE [25,10] uniform, batch 1024, full epoch (196,615 seeds, "
                               "193 batches), Ogbn-Products-shaped R-MAT graph (2,449,029 nodes, "
                               "61,859,140 undirected edges)"),
+    "graphsage_pd_uva": dict(kind="nodewise", graph="PD", fanouts=[25, 10], batch=1024,
+                             seeds=196_615, replace=False, bias=0, host_mapped=True,
+                             desc="GraphSAGE [25,10] as graphsage_pd with the CSC index array in "
+                                  "pinned host memory read over the host link (UVA, P:415; "
+                                  "SURVEY 8(f) f4)"),
     "graphsage_tiny": dict(kind="nodewise", graph="tiny", fanouts=[5, 5], batch=512, seeds=512,
                            replace=False, bias=0,
                            desc="GraphSAGE [5,5] uniform, 512 seeds, 10k-node/100k-edge R-MAT"),
@@ -351,7 +356,7 @@ def run_gpu(args, wl, world, rank, device):
     t0 = time.time()
     g = make_graph_dist(wl["graph"], world, rank, device)
     gen_s = time.time() - t0
-    G = gs.Graph(g["indptr"], g["indices"], g["weights"])
+    G = gs.Graph(g["indptr"], g["indices"], g["weights"], host_mapped=wl.get("host_mapped", False))
     inputs = workload_inputs(wl, g, device)
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=device)  # > 126 MB L2

@@ -68,7 +68,12 @@ typedef struct gs_graph gs_graph;
 
 enum {
   GS_GRAPH_HOST_PTRS = 1, /* indptr/indices/weights are host pointers (copied to HBM)      */
-  GS_GRAPH_BORROW = 2     /* device pointers are used in place; caller keeps them alive    */
+  GS_GRAPH_BORROW = 2,    /* device pointers are used in place; caller keeps them alive    */
+  GS_GRAPH_HOST_MAPPED = 4 /* with HOST_PTRS: indices / weights stay in host memory, pinned
+                             and mapped (cudaHostRegister), read by every kernel over the
+                             host link (UVA; graphs beyond 180 GB of HBM, SURVEY
+                             8(f) f4); indptr is copied to HBM; the caller keeps the host
+                             arrays alive until gs_graph_destroy                          */
 };                        /* default (0): device pointers, copied into library-owned HBM  */
 
 /* Validates the CSC on the device (indptr[0] == 0, monotone, indptr[N] ==
@@ -89,6 +94,7 @@ typedef struct gs_graph_info {
   const int64_t* indptr;   /* device */
   const int32_t* indices;  /* device */
   const float* weights;    /* device or NULL */
+  int host_mapped;         /* indices / weights are mapped host memory (GS_GRAPH_HOST_MAPPED) */
 } gs_graph_info;
 gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out);
 /* Replaces the edge weights (device float[num_edges]) and recomputes the a0

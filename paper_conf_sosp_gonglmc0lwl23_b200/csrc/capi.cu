@@ -211,7 +211,37 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
     gs_graph_destroy(g);
     return st;
   };
-  if (flags & GS_GRAPH_BORROW) {
+  if (flags & GS_GRAPH_HOST_MAPPED) {
+    // beyond-HBM graphs (P:415 UVA): indptr copied to HBM, the
+    // index / weight arrays stay in pinned host memory and every kernel reads
+    // them through their mapped device aliases over the host link
+    if (!(flags & GS_GRAPH_HOST_PTRS))
+      return cleanup(fail(GS_ERR_INVALID_ARGUMENT, "gs_graph_create: HOST_MAPPED needs host pointers"));
+    if (!g->b_indptr.ensure(g->al, (num_nodes + 1) * 8, stream))
+      return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_create: device allocation failed"));
+    g->indptr = (int64_t*)g->b_indptr.ptr;
+    cudaError_t e = cudaMemcpyAsync(g->indptr, indptr, (num_nodes + 1) * 8, cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cleanup(cuda_fail(e, "gs_graph_create copy"));
+    const void* arrs[2] = {indices, weights};
+    for (int k = 0; k < 2; ++k) {
+      if (!arrs[k] || num_edges == 0) continue;
+      void* hp = const_cast<void*>(arrs[k]);
+      e = cudaHostRegister(hp, (size_t)num_edges * 4, cudaHostRegisterMapped | cudaHostRegisterReadOnly);
+      if (e == cudaErrorHostMemoryAlreadyRegistered) {
+        cudaGetLastError();  // already pinned by the caller: use its mapping, do not unregister
+      } else if (e != cudaSuccess) {
+        return cleanup(cuda_fail(e, "gs_graph_create: cudaHostRegister"));
+      } else {
+        g->host_reg[g->n_reg++] = hp;
+      }
+      void* dp = nullptr;
+      e = cudaHostGetDevicePointer(&dp, hp, 0);
+      if (e != cudaSuccess) return cleanup(cuda_fail(e, "gs_graph_create: cudaHostGetDevicePointer"));
+      if (k == 0) g->indices = (int32_t*)dp;
+      else g->weights = (float*)dp;
+    }
+    g->host_mapped = true;
+  } else if (flags & GS_GRAPH_BORROW) {
     g->indptr = const_cast<int64_t*>(indptr);
     g->indices = const_cast<int32_t*>(indices);
     g->weights = const_cast<float*>(weights);
@@ -300,6 +330,7 @@ gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out) {
   out->indptr = g->indptr;
   out->indices = g->indices;
   out->weights = g->weights;
+  out->host_mapped = g->host_mapped ? 1 : 0;
   return GS_OK;
 }
 
@@ -313,6 +344,7 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_deg.reset(g->al, s);
   g->b_walk.reset(g->al, s);
   g->b_err.reset(g->al, s);
+  for (int k = 0; k < g->n_reg; ++k) cudaHostUnregister(g->host_reg[k]);
   delete g;
 }
 

@@ -64,6 +64,9 @@ struct gs_graph {
   const int4* walk_rec = nullptr;
   bool walk_index_failed = false;
   int* d_err = nullptr;  // walk error word
+  bool host_mapped = false;  // indices (+ weights) read from pinned host memory (UVA)
+  void* host_reg[2] = {nullptr, nullptr};  // ranges this graph registered (unregistered at destroy)
+  int n_reg = 0;
 };
 
 struct gs_blocks {

@@ -166,11 +166,13 @@ __global__ void walk_index_kernel(const int64_t* __restrict__ indptr, const int3
 
 // Builds the walk index once per graph (16 bytes per CSC entry) unless
 // disabled (GS_WALK_PLAIN_CSC / GS_WALK_INDEX=0), the graph has in-degrees
-// >= 2^31, or the allocation fails -- then the walk reads the plain CSC.
+// >= 2^31, the graph lives in host memory (GS_GRAPH_HOST_MAPPED: the index
+// would put 4x the index array back into HBM), or the allocation fails --
+// then the walk reads the plain CSC.
 static const int4* walk_index(const gs_graph* g, cudaStream_t stream, bool plain) {
   gs_graph* gm = const_cast<gs_graph*>(g);
   const char* e = getenv("GS_WALK_INDEX");
-  if (plain || (e && e[0] == '0')) return nullptr;
+  if (plain || (e && e[0] == '0') || g->host_mapped) return nullptr;
   if (gm->walk_rec) return gm->walk_rec;
   if (gm->walk_index_failed || g->num_edges == 0 || g->max_in_degree >= (int64_t(1) << 31)) return nullptr;
   if (!gm->b_walk.ensure(gm->al, (size_t)g->num_edges * 16, stream)) {

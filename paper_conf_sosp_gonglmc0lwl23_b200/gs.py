@@ -24,7 +24,7 @@ STATUS = {0: "GS_OK", 1: "GS_ERR_INVALID_ARGUMENT", 2: "GS_ERR_OUT_OF_MEMORY", 3
           7: "GS_ERR_CAPACITY", 8: "GS_ERR_INVALID_GRAPH"}
 UNIFORM, EDGE, PASS_COLNORM = 0, 1, 2
 LADIES, DEGREE, COUNT = 0, 1, 2
-GRAPH_HOST_PTRS, GRAPH_BORROW = 1, 2
+GRAPH_HOST_PTRS, GRAPH_BORROW, GRAPH_HOST_MAPPED = 1, 2, 4
 WALK_FORCE_NODE2VEC = 1
 META_FIELDS = 8
 
@@ -63,7 +63,8 @@ class _GraphInfo(ctypes.Structure):
     _fields_ = [("num_nodes", ctypes.c_int64), ("num_edges", ctypes.c_int64),
                 ("weighted", ctypes.c_int), ("sorted", ctypes.c_int),
                 ("max_in_degree", ctypes.c_int64), ("indptr", ctypes.c_void_p),
-                ("indices", ctypes.c_void_p), ("weights", ctypes.c_void_p)]
+                ("indices", ctypes.c_void_p), ("weights", ctypes.c_void_p),
+                ("host_mapped", ctypes.c_int)]
 
 
 class _LayerBuffers(ctypes.Structure):
@@ -215,7 +216,7 @@ class Graph:
     """gs_graph: validated CSC in HBM (a0)."""
 
     def __init__(self, indptr: torch.Tensor, indices: torch.Tensor, weights=None, borrow=False,
-                 stream=None):
+                 stream=None, host_mapped=False):
         L = load_library()
         _drain()
         indptr = indptr.to(torch.int64).contiguous()
@@ -223,7 +224,12 @@ class Graph:
         if weights is not None:
             weights = weights.to(torch.float32).contiguous()
         flags = 0
-        if indptr.device.type == "cpu":
+        if host_mapped:  # CPU tensors kept in host memory, read over the host link (UVA)
+            indptr, indices = indptr.cpu(), indices.cpu()
+            weights = None if weights is None else weights.cpu()
+            flags |= GRAPH_HOST_PTRS | GRAPH_HOST_MAPPED
+            self._keep = (indptr, indices, weights)
+        elif indptr.device.type == "cpu":
             flags |= GRAPH_HOST_PTRS
         elif borrow:
             flags |= GRAPH_BORROW
@@ -240,6 +246,7 @@ class Graph:
         self.weighted = bool(info.weighted)
         self.sorted = bool(info.sorted)
         self.max_in_degree = info.max_in_degree
+        self.host_mapped = bool(info.host_mapped)
 
     @property
     def handle(self):
