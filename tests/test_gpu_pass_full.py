@@ -74,3 +74,27 @@ def test_pass_full_sampling_medium(gs, oracle_lib):
     ref = oracle_lib.sample_neighbors(O, seeds.numpy(), [10, 10], batch_size=1024, bias_mode=1,
                                       rng_key=61)
     compare_all(out, ref, "PASS full [10,10]")
+
+
+def test_pass_attention_pdw_full_size(gs):
+    """The bench configuration (PDw, 128-d features, H = 32): att of 300 random
+    columns and the 20 highest-degree columns recomputed by the oracle."""
+    g = synth.make_graph("PDw", device="cuda")
+    G = gs.Graph(g["indptr"], g["indices"], g["weights"])
+    N = g["indptr"].numel() - 1
+    X = synth.make_grid_matrix(21, N, 128, device="cuda")
+    W1 = synth.make_grid_matrix(22, 128, 32, device="cuda")
+    W2 = synth.make_grid_matrix(23, 128, 32, device="cuda")
+    W3 = [0.2, -0.4, 0.9]
+    att = gs.pass_attention(G, X, W1, W2, W3)
+    ip = g["indptr"].cpu().numpy()
+    deg = np.diff(ip)
+    cols = sorted(set(np.random.default_rng(3).integers(0, N, 300).tolist()) |
+                  set(np.argsort(deg)[-20:].tolist()))
+    ix = g["indices"].cpu().numpy()
+    w = g["weights"].cpu().numpy()
+    ref = pass_att.pass_attention_columns(ip, ix, w, X.float().cpu().numpy(),
+                                          W1.float().cpu().numpy(), W2.float().cpu().numpy(), W3, cols)
+    a = att.cpu().numpy()
+    for v in cols:
+        assert np.array_equal(a[ip[v]:ip[v + 1]], ref[v]), f"column {v}"
