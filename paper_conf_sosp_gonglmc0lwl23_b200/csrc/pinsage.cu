@@ -6,9 +6,8 @@
 //   W  walks: the frontier is cut into chunks of C columns whose visit-count
 //      hash tables (HCAP >= 2 * num_walks * walk_length entries each, linear
 //      probing, shared memory) fit the CTA's shared memory; every thread runs
-//      the flat (column, walk) pairs of the chunk -- one Philox call and one
-//      random 16-byte walk-index record per step (the neighbour and its own
-//      column range; indptr pair + index gather without the index) -- and counts
+//      the flat (column, walk) pairs of the chunk -- one Philox call, the
+//      current node's indptr pair and one index gather per step -- and counts
 //      each visit of x != v with a shared-memory atomicAdd;
 //   S  select: a warp per column takes the k most visited entries (count
 //      descending, id ascending) -- a warp bitonic sort of the (<= 32)
@@ -67,7 +66,6 @@ struct PSParams {
   int64_t nwords, ngroups;
   int* err;
   unsigned int* claim;
-  const int4* rec;                   // walk index (walk.cu) or NULL: one record per step
 };
 
 __device__ __forceinline__ uint32_t ps_hash(uint32_t x) {
@@ -129,7 +127,6 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
         for (int i = tid; i < npairs; i += PS_ILP * PS_THREADS) {
           int32_t wv[PS_ILP], wx[PS_ILP];
           int wcol[PS_ILP], ww[PS_ILP];
-          int64_t woff[PS_ILP], wd[PS_ILP];  // column range of the current node
           bool alive[PS_ILP];
 #pragma unroll
           for (int a = 0; a < PS_ILP; ++a) {
@@ -140,36 +137,24 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
             wv[a] = alive[a] ? __ldcg(F + c0 + wcol[a]) : 0;
             if (wv[a] < 0 || (int64_t)wv[a] >= P.N) alive[a] = false;
             wx[a] = wv[a];
-            woff[a] = alive[a] ? __ldg(P.indptr + wv[a]) : 0;  // shared by the column's walks (L1/L2)
-            wd[a] = alive[a] ? __ldg(P.indptr + wv[a] + 1) - woff[a] : 0;
           }
           for (int t = 1; t <= T; ++t) {
+            U4 r[PS_ILP];
+            int64_t off[PS_ILP], d[PS_ILP];
+#pragma unroll
+            for (int a = 0; a < PS_ILP; ++a) {
+              r[a] = philox((uint32_t)wv[a], (uint32_t)(ww[a] * T + t - 1), ctr2(l, TAG_PINSAGE), gb, P.key);
+              if ((float)(r[a].z >> 8) * 0x1p-24f < P.restart) alive[a] = false;  // restart at v (R27)
+              off[a] = alive[a] ? __ldg(P.indptr + wx[a]) : 0;
+              d[a] = alive[a] ? __ldg(P.indptr + wx[a] + 1) : 0;
+            }
             bool any = false;
 #pragma unroll
             for (int a = 0; a < PS_ILP; ++a) {
-              const U4 r = philox((uint32_t)wv[a], (uint32_t)(ww[a] * T + t - 1), ctr2(l, TAG_PINSAGE), gb, P.key);
-              if ((float)(r.z >> 8) * 0x1p-24f < P.restart) alive[a] = false;  // restart at v (R27)
-              if (wd[a] == 0) alive[a] = false;                                  // dead end (R13)
-              if (alive[a]) {
-                const int64_t pos = woff[a] + (int64_t)draw_below((uint64_t)wd[a], r.x, r.y);
-                if (P.rec) {  // walk index: the neighbour and its own column range in one record
-                  const int4 R = __ldg(P.rec + pos);
-                  wx[a] = R.x;
-                  woff[a] = (int64_t)(((uint64_t)(uint32_t)R.z << 32) | (uint32_t)R.y);
-                  wd[a] = R.w;
-                } else {
-                  wx[a] = __ldg(P.indices + pos);
-                }
-              }
+              d[a] -= off[a];
+              if (d[a] == 0) alive[a] = false;            // dead end (R13)
+              if (alive[a]) wx[a] = __ldg(P.indices + off[a] + (int64_t)draw_below((uint64_t)d[a], r[a].x, r[a].y));
               any |= alive[a];
-            }
-            if (!P.rec) {
-#pragma unroll
-              for (int a = 0; a < PS_ILP; ++a)
-                if (alive[a]) {
-                  woff[a] = __ldg(P.indptr + wx[a]);
-                  wd[a] = __ldg(P.indptr + wx[a] + 1) - woff[a];
-                }
             }
             if (!any) break;
 #pragma unroll
@@ -359,8 +344,6 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
   }
 }
 
-const int4* walk_index_of(const gs_graph* g, cudaStream_t stream);
-
 gs_status run_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                       int64_t batch_size, int64_t batch_base, const int32_t* topk, int L,
                       int num_walks, int walk_length, float restart, uint64_t key,
@@ -386,7 +369,6 @@ gs_status run_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds
   P.walk_length = walk_length;
   P.restart = restart;
   P.key = key;
-  P.rec = walk_index_of(g, stream);
   int hlog = 5;
   while ((1 << hlog) < 2 * num_walks * walk_length) ++hlog;
   P.hlog = hlog;

@@ -192,9 +192,6 @@ static const int4* walk_index(const gs_graph* g, cudaStream_t stream, bool plain
   return gm->walk_rec;
 }
 
-// The walk index for other kernels (PinSAGE-style restart walks), or NULL.
-const int4* walk_index_of(const gs_graph* g, cudaStream_t stream) { return walk_index(g, stream, false); }
-
 gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walkers,
                       int64_t walker_base, int length, float p, float q, uint64_t key,
                       bool node2vec, bool plain, cudaStream_t stream, int32_t* traces,

@@ -114,16 +114,3 @@ def test_pinsage_empty(gs, tiny):
     out = gs.sample_pinsage(G, torch.zeros(0, dtype=torch.int32, device="cuda"), [3, 3], 4, 2, 0.5,
                             batch_size=10)
     assert out.to_host() == []
-
-
-def test_pinsage_plain_csc(gs, oracle_lib, monkeypatch):
-    """Without the walk index (GS_WALK_INDEX=0) the walks read the plain CSC:
-    same samples."""
-    monkeypatch.setenv("GS_WALK_INDEX", "0")
-    g = synth.make_graph("tiny", device="cuda")
-    G = gs.Graph(g["indptr"], g["indices"], g["weights"])
-    seeds = synth.make_seeds("tiny", 800)
-    out = gs.sample_pinsage(G, seeds.cuda(), [5, 3], 10, 3, 0.5, batch_size=300, rng_key=0xB0B).to_host()
-    ref = oracle_lib.pinsage(oracle_lib.Graph(*host_graph(g)), seeds.numpy(), [5, 3], 10, 3, 0.5,
-                             batch_size=300, rng_key=0xB0B)
-    compare_all(out, ref, "pinsage plain CSC")
