@@ -5,8 +5,8 @@
 // materialise these intermediates (Extract-Select / Edge-MapReduce fusion,
 // P:289-294); this layer is the unfused reference path of the same algebra.
 //
-//   A[:, cols]      degree gather + CUB-free multi-block scan + warp-per-column
-//                   segmented copy of the column slices (indices, edge ids, weights)
+//   A[:, cols]      degree gather + CUB-free multi-block scan + a flat copy of
+//                   each 32-column group's slices (indices, edge ids, weights)
 //   A[rows, :]      N-bit row bitmap, warp ballot count + scan + compaction
 //   A.sum(axis)     axis 0: warp shuffle fp64 reduction per column; axis 1:
 //                   fp64 atomics into a dense per-node accumulator (R1, R19)
@@ -109,6 +109,11 @@ __global__ void col_degree_kernel(const int64_t* __restrict__ indptr, int64_t N,
   }
 }
 
+// A warp takes 32 columns at a time: one round trip fetches their ids, indptr
+// pairs and output offsets (a lane each); the group's entries are then copied
+// as one flat range, 4 per lane in flight, each lane finding its column by a
+// 5-step shuffle search over the inclusive degree prefix (no per-column
+// dependent-load chain, every lane busy whatever the degrees).
 __global__ void __launch_bounds__(OPS_THREADS) col_copy_kernel(const int64_t* __restrict__ indptr,
                                                               const int32_t* __restrict__ indices,
                                                               const float* __restrict__ w, int64_t N,
@@ -118,14 +123,48 @@ __global__ void __launch_bounds__(OPS_THREADS) col_copy_kernel(const int64_t* __
   const int lane = threadIdx.x & 31;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t j = warp; j < n; j += nwarps) {
-    const int32_t v = cols[j];
-    if (v < 0 || (int64_t)v >= N) continue;
-    const int64_t o = __ldg(indptr + v), d = __ldg(indptr + v + 1) - o, p = ip[j];
-    for (int64_t i = lane; i < d; i += 32) {
-      row[p + i] = __ldcs(indices + o + i);
-      eid[p + i] = o + i;
-      val[p + i] = w ? __ldcs(w + o + i) : 1.0f;
+  for (int64_t g0 = warp * 32; g0 < n; g0 += nwarps * 32) {
+    const int64_t j = g0 + lane;
+    const int32_t v = j < n ? __ldg(cols + j) : -1;
+    const bool valid = v >= 0 && (int64_t)v < N;
+    const int64_t o = valid ? __ldg(indptr + v) : 0;
+    const int64_t d = valid ? __ldg(indptr + v + 1) - o : 0;
+    const int64_t p = j < n ? __ldg(ip + j) : 0;
+    int64_t S = d;  // inclusive prefix of the group's degrees
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const int64_t y = __shfl_up_sync(0xffffffffu, S, off);
+      if (lane >= off) S += y;
+    }
+    const int64_t D = __shfl_sync(0xffffffffu, S, 31);
+    for (int64_t f0 = 0; f0 < D; f0 += 32 * 4) {
+      int64_t src[4], dst[4];
+      int32_t rv[4];
+      float wv[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int64_t f = f0 + k * 32 + lane;
+        int l = 0;  // smallest l with S_l > f
+#pragma unroll
+        for (int step = 16; step >= 1; step >>= 1) {
+          const int64_t sc = __shfl_sync(0xffffffffu, S, l + step - 1);
+          if (sc <= f) l += step;
+        }
+        const int64_t Sl = __shfl_sync(0xffffffffu, S, l & 31), dl = __shfl_sync(0xffffffffu, d, l & 31);
+        const int64_t ol = __shfl_sync(0xffffffffu, o, l & 31), pl = __shfl_sync(0xffffffffu, p, l & 31);
+        const int64_t r = f - (Sl - dl);
+        src[k] = f < D ? ol + r : -1;
+        dst[k] = pl + r;
+        rv[k] = src[k] >= 0 ? __ldcs(indices + src[k]) : 0;
+        wv[k] = (src[k] >= 0 && w) ? __ldcs(w + src[k]) : 1.0f;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (src[k] >= 0) {
+          row[dst[k]] = rv[k];
+          eid[dst[k]] = src[k];
+          val[dst[k]] = wv[k];
+        }
     }
   }
 }
@@ -356,7 +395,7 @@ gs_status gs_matrix_slice_columns(const gs_graph* g, const int32_t* cols, int64_
   if ((st = alloc_entries(m, n_cols, nnz, s))) return st;
   if (n_cols > 0) GS_CUDA_TRY(cudaMemcpyAsync(m->b_cols.ptr, cols, n_cols * 4, cudaMemcpyDeviceToDevice, s));
   if (n_cols > 0) {
-    col_copy_kernel<<<grid_for(n_cols * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
+    col_copy_kernel<<<grid_for(n_cols, OPS_THREADS), OPS_THREADS, 0, s>>>(
         g->indptr, g->indices, g->weights, g->num_nodes, cols, n_cols, ip, (int32_t*)m->b_row.ptr,
         (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr);
     GS_CUDA_TRY(cudaGetLastError());
