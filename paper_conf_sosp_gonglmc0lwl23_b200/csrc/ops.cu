@@ -233,54 +233,18 @@ __global__ void __launch_bounds__(OPS_THREADS) row_copy_kernel(const int64_t* __
 }
 
 // ---- sums ----
-// 32-column groups as in col_copy_kernel: one round trip for the group's
-// offsets, the group's entries read as one flat range (4 per lane in flight),
-// each added in fp64 to its column's shared-memory accumulator (exact for the
-// usual sums, R19), one fp32 rounding per column.
 __global__ void __launch_bounds__(OPS_THREADS) col_sum_kernel(const int64_t* __restrict__ ip,
                                                              const float* __restrict__ val, int64_t n,
                                                              float* __restrict__ out) {
-  __shared__ double acc[OPS_THREADS];
   const int lane = threadIdx.x & 31;
-  double* wacc = acc + (threadIdx.x & ~31);
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t g0 = warp * 32; g0 < n; g0 += nwarps * 32) {
-    const int64_t j = g0 + lane;
-    const int64_t lo = j < n ? __ldg(ip + j) : 0, hi = j < n ? __ldg(ip + j + 1) : 0;
-    const int64_t d = hi - lo;
-    const int64_t base = __shfl_sync(0xffffffffu, lo, 0);
-    int64_t S = d;
+  for (int64_t j = warp; j < n; j += nwarps) {
+    double s = 0.0;
+    for (int64_t i = ip[j] + lane; i < ip[j + 1]; i += 32) s += (double)__ldcs(val + i);
 #pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const int64_t y = __shfl_up_sync(0xffffffffu, S, off);
-      if (lane >= off) S += y;
-    }
-    const int64_t D = __shfl_sync(0xffffffffu, S, 31);
-    wacc[lane] = 0.0;
-    __syncwarp();
-    for (int64_t f0 = 0; f0 < D; f0 += 32 * 4) {
-      float x[4];
-      int col[4];
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const int64_t f = f0 + k * 32 + lane;
-        int l = 0;
-#pragma unroll
-        for (int step = 16; step >= 1; step >>= 1) {
-          const int64_t sc = __shfl_sync(0xffffffffu, S, l + step - 1);
-          if (sc <= f) l += step;
-        }
-        col[k] = f < D ? l : -1;
-        x[k] = f < D ? __ldcs(val + base + f) : 0.0f;  // the group's entries are contiguous
-      }
-#pragma unroll
-      for (int k = 0; k < 4; ++k)
-        if (col[k] >= 0) atomicAdd(wacc + col[k], (double)x[k]);
-    }
-    __syncwarp();
-    if (j < n) out[j] = (float)wacc[lane];
-    __syncwarp();
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) out[j] = (float)s;
   }
 }
 
@@ -488,7 +452,7 @@ gs_status gs_matrix_sum(const gs_matrix* m, int axis, float* out, void* stream_)
   cudaStream_t s = (cudaStream_t)stream_;
   if (axis == 0) {
     if (m->n_cols > 0) {
-      col_sum_kernel<<<grid_for(m->n_cols, OPS_THREADS), OPS_THREADS, 0, s>>>(
+      col_sum_kernel<<<grid_for(m->n_cols * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
           (const int64_t*)m->b_indptr.ptr, (const float*)m->b_val.ptr, m->n_cols, out);
       GS_CUDA_TRY(cudaGetLastError());
     }
