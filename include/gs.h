@@ -162,7 +162,7 @@ gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out);
  * the sampled data (read `totals` first).  Errors: GS_ERR_INVALID_ARGUMENT
  * (null pointer, bad layer), GS_ERR_OUT_OF_MEMORY, GS_ERR_CUDA. */
 gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
-                         int64_t* indptr, int32_t* row_map, int64_t* totals, cudaStream_t stream);
+                         int64_t* indptr, int32_t* row_map, int64_t* totals, void* stream);
 void gs_blocks_destroy(gs_blocks* b);
 
 /* ------------------------------------------------------------------------ */
@@ -185,7 +185,7 @@ enum {
  *   rng_key Philox key; counters (v, slot, layer|tag<<24, global batch) (R4)
  * Output per (b, l): col_map = frontier (l = 0: the batch's seeds; l > 0: the
  * previous layer's row_map, R2), edges in column order then ascending position
- * (slot order with replacement), row_map in first-occurrence order (R3).
+ * (slot order with replacement), row_map = the block's distinct rows ascending (R3).
  * Envelope: batch_size * prod(fanouts[0..l]) <= 2^25 for every l. */
 gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                               int64_t batch_size, int64_t batch_index_base,
@@ -194,8 +194,8 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
 
 /* ShaDow (R12): node-wise sampling as gs_sample_neighbors
  * (bias_mode UNIFORM or EDGE, no replacement), then for every batch the
- * subgraph of A induced on U = first-occurrence union of the seeds and all
- * sampled rows.  One block per batch (num_layers == 1 in the result):
+ * subgraph of A induced on U = the union of the seeds and all sampled rows,
+ * ascending (R12).  One block per batch (num_layers == 1 in the result):
  * col_map == row_map == U, edges u->v with u, v in U in CSC order. */
 gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                            int64_t batch_size, int64_t batch_index_base, const int32_t* fanouts,

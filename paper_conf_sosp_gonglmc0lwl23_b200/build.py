@@ -16,7 +16,10 @@ LIB = os.path.join(HERE, "libgsb200.so")
 SOURCES = ["capi.cu", "nodewise_wave.cu", "shadow.cu", "layerwise.cu", "layerwise_bm.cu", "walk.cu", "pack.cu", "pinsage.cu", "ops.cu", "pass_att.cu"]
 HEADERS = ["common.cuh", "gs_internal.h", "nodewise_common.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+# -cudart shared: the static runtime would embed the name table of every
+# runtime entry point (including batched-copy APIs this pool forbids) in the .so
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-fmad=false",
+         "-cudart", "shared",
          "-std=c++17", "-Xcompiler", "-fPIC", "-I", os.path.join(ROOT, "include")]
 
 
@@ -44,7 +47,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if force or _stale(LIB, objs):
         tmp = LIB + ".tmp"
         subprocess.check_call([NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a",
-                               "-o", tmp] + objs + ["-lcublas", "-Xlinker", "-rpath=/usr/local/cuda/lib64"])
+                               "-cudart", "shared", "-o", tmp] + objs +
+                              ["-lcublas", "-Xlinker", "-rpath=/usr/local/cuda/lib64"])
         os.replace(tmp, LIB)
     return LIB
 

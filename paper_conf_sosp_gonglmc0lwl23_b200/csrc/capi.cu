@@ -520,7 +520,9 @@ gs_status gs_blocks_sync(gs_blocks* b) {
   GS_CUDA_TRY(cudaMemcpy(err, b->b_err.ptr, 16, cudaMemcpyDeviceToHost));
   GS_CUDA_TRY(cudaMemcpy(ctr, b->b_ctr.ptr, std::min<size_t>(sizeof(ctr), b->b_ctr.bytes),
                          cudaMemcpyDeviceToHost));
-  b->synced = true;
+  // views only of a result whose every block is complete (out-of-range seeds
+  // leave valid, empty columns; an overflowed or inconsistent block does not)
+  b->synced = (err[0] & (ERR_CAPACITY | ERR_INTERNAL)) == 0;
   if (err[0] & ERR_INTERNAL) return fail(GS_ERR_CUDA, "internal consistency check failed in a sampling kernel");
   if (err[0] & ERR_SEED_RANGE) return fail(GS_ERR_INDEX_OUT_OF_RANGE, "a seed id is outside [0, N)");
   if (err[0] & ERR_CAPACITY) {

@@ -480,8 +480,9 @@ __global__ void __launch_bounds__(LW_THREADS) layerwise_kernel(LWParams P) {
       if (threadIdx.x == 0) {
         P.indptr_out[l][ibase + T] = E;
         long long* m = (long long*)(P.meta + (b * P.L + l) * 8);
-        m[0] = T; m[1] = nsel; m[2] = E; m[3] = colbase; m[4] = rbase; m[5] = ibase;
-        m[6] = ebase; m[7] = 0;
+        // an overflowed block wrote no edges: record it empty (GS_ERR_CAPACITY is raised)
+        m[0] = T; m[1] = nsel; m[2] = fits ? E : 0; m[3] = colbase; m[4] = rbase; m[5] = ibase;
+        m[6] = fits ? ebase : 0; m[7] = 0;
       }
       __syncthreads();
       F = P.row_map[l] + rbase;

@@ -677,8 +677,9 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       if (threadIdx.x == 0) {
         P.indptr_out[l][ibase + T] = E;
         long long* mt = (long long*)(P.meta + (b * P.L + l) * 8);
-        mt[0] = T; mt[1] = nsel; mt[2] = E; mt[3] = colbase; mt[4] = rbase; mt[5] = ibase;
-        mt[6] = ebase; mt[7] = 0;
+        // an overflowed block wrote no edges: record it empty (GS_ERR_CAPACITY is raised)
+        mt[0] = T; mt[1] = nsel; mt[2] = fits ? E : 0; mt[3] = colbase; mt[4] = rbase; mt[5] = ibase;
+        mt[6] = fits ? ebase : 0; mt[7] = 0;
       }
       __syncthreads();
       F = P.row_map[l] + rbase;

@@ -59,12 +59,16 @@ struct PackParams {
   int64_t* eid;
   int64_t* indptr;
   int32_t* row_map;
+  int64_t edge_cap, indptr_cap, row_cap;  // the layer buffers' capacities (copies are clamped)
 };
 
 __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
   for (int64_t b = blockIdx.x; b < P.nb; b += gridDim.x) {
     const int64_t* m = P.meta + (b * P.L + P.layer) * GS_META_FIELDS;
-    const int64_t T = m[0], R = m[1], E = m[2];
+    // clamped to the layer buffers: a block recorded past them is never read
+    const int64_t E = min(m[2], max(P.edge_cap - m[6], (int64_t)0));
+    const int64_t T = min(m[0], max(P.indptr_cap - m[5] - 1, (int64_t)-1));
+    const int64_t R = min(m[1], max(P.row_cap - m[4], (int64_t)0));
     const int64_t* o = P.off + b * 3;
     const int64_t eo = o[0], io = o[1], ro = o[2];
     for (int64_t i = threadIdx.x; i < E; i += PK_THREADS) {
@@ -82,7 +86,8 @@ using namespace gsb;
 
 extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
                                     int64_t* indptr, int32_t* row_map, int64_t* totals,
-                                    cudaStream_t stream) {
+                                    void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
   if (!b || !row_local || !eid || !indptr || !row_map || !totals)
     return fail(GS_ERR_INVALID_ARGUMENT, "gs_blocks_pack: null argument");
   if (layer < 0 || layer >= b->num_layers) return fail(GS_ERR_INVALID_ARGUMENT, "gs_blocks_pack: bad layer");
@@ -110,6 +115,9 @@ extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_
   P.eid = eid;
   P.indptr = indptr;
   P.row_map = row_map;
+  P.edge_cap = lb.edge_capacity;
+  P.indptr_cap = lb.indptr_capacity;
+  P.row_cap = lb.row_capacity;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);

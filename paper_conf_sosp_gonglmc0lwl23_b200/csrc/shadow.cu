@@ -311,6 +311,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
       long long* m = (long long*)(P.meta + b * 8);
       m[0] = nU; m[1] = nU; m[2] = E; m[3] = b * P.stride; m[4] = b * P.stride;
       m[5] = b * P.stride + b; m[6] = fits ? eoff : 0; m[7] = 0;
+      if (!fits) m[2] = 0;  // nothing was written: an overflowed block is empty (GS_ERR_CAPACITY)
       if (!fits) atomicOr(P.err, ERR_CAPACITY);
     }
     // ---- write kept edges in CSC order: a copy of the staged edges (the
@@ -476,6 +477,11 @@ static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bp
     const int64_t o_s = o_e + nw * P.wcap * 8;
     if (!blk->b_ws.ensure(al, (size_t)(o_s + std::max<int64_t>(nodes, 1) * 8), stream))
       return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (induce staging)");
+    // the staging overwrites whatever layout another sampler left in b_ws
+    // (node-wise / PinSAGE / layer-wise keep zeroed bitmaps there between
+    // calls): invalidate it so their next launch on this object re-clears it
+    blk->ws_kind_prev = 0;
+    blk->ws_stride_prev = -1;
     P.stage_row = (int32_t*)blk->b_ws.ptr;
     P.stage_eid = (int64_t*)((char*)blk->b_ws.ptr + o_e);
     P.ustart = (int64_t*)((char*)blk->b_ws.ptr + o_s);
