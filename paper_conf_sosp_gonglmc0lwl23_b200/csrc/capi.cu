@@ -88,6 +88,22 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
                             int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                             int replace, int bias, uint64_t key, cudaStream_t stream,
                             gs_blocks* blk);
+gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                           const int64_t* bptr_host, int64_t batch_size, int64_t nbatch,
+                           int64_t batch_base, const int32_t* fanouts, int L, int replace, int bias,
+                           uint64_t key, cudaStream_t stream, gs_blocks* blk);
+// node-wise engine: the hop-synchronous kernels (default) or the round-1
+// single-launch wave kernel (GS_NODEWISE=wave; kept for comparison)
+gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                       int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
+                       int replace, int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  const char* e = getenv("GS_NODEWISE");
+  if (e && e[0] == 'w')
+    return run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, replace, bias, key,
+                             stream, blk);
+  return run_nodewise_hop(g, seeds, num_seeds, nullptr, batch_size, (num_seeds + batch_size - 1) / batch_size,
+                          batch_base, fanouts, L, replace, bias, key, stream, blk);
+}
 gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
@@ -137,17 +153,31 @@ __global__ void validate_csc_kernel(const int64_t* __restrict__ indptr,
 // a0 pre-processing of weighted graphs: colsum[v] = fp32(sum_fp64 of
 // the column's weights) -- the PASS A3 denominator (R11) and the scale of the
 // A-Res candidate threshold (nodewise_wave.cu).
+// Also poscnt[v] = #{w > 0} in the column: the number of eligible edges, so
+// the weighted node-wise sampler knows each column's sample count min(k,
+// poscnt) (R6) before it samples.
 __global__ void colsum_kernel(const int64_t* __restrict__ indptr, const float* __restrict__ w,
-                              int64_t N, float* __restrict__ colsum) {
+                              int64_t N, float* __restrict__ colsum, int32_t* __restrict__ poscnt) {
   const int lane = threadIdx.x & 31;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t v = warp; v < N; v += nwarps) {
     const int64_t a = indptr[v], b = indptr[v + 1];
     double sum = 0.0;
-    for (int64_t i = a + lane; i < b; i += 32) sum += (double)w[i];
-    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-    if (lane == 0) colsum[v] = (float)sum;
+    int pos = 0;
+    for (int64_t i = a + lane; i < b; i += 32) {
+      const float x = w[i];
+      sum += (double)x;
+      pos += x > 0.0f ? 1 : 0;
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+      sum += __shfl_xor_sync(0xffffffffu, sum, o);
+      pos += __shfl_xor_sync(0xffffffffu, pos, o);
+    }
+    if (lane == 0) {
+      colsum[v] = (float)sum;
+      poscnt[v] = pos;
+    }
   }
 }
 
@@ -286,10 +316,13 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
   g->sorted = (vflags & 4) ? 0 : 1;
   g->max_in_degree = (int64_t)mdeg;
   if (g->weights) {
-    if (!g->b_colsum.ensure(g->al, std::max<int64_t>(num_nodes, 1) * 4, stream))
+    if (!g->b_colsum.ensure(g->al, std::max<int64_t>(num_nodes, 1) * 4, stream) ||
+        !g->b_poscnt.ensure(g->al, std::max<int64_t>(num_nodes, 1) * 4, stream))
       return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_create: device allocation failed"));
     g->colsum = (float*)g->b_colsum.ptr;
-    colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, num_nodes, g->colsum);
+    g->poscnt = (int32_t*)g->b_poscnt.ptr;
+    colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, num_nodes, g->colsum,
+                                                         g->poscnt);
     e = cudaGetLastError();
     if (e != cudaSuccess) return cleanup(cuda_fail(e, "colsum_kernel launch"));
   }
@@ -311,11 +344,14 @@ gs_status gs_graph_set_weights(gs_graph* g, const float* weights, uint32_t flags
     if (g->num_edges)
       GS_CUDA_TRY(cudaMemcpyAsync(g->weights, weights, g->num_edges * 4, cudaMemcpyDeviceToDevice, stream));
   }
-  if (!g->b_colsum.ensure(g->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
+  if (!g->b_colsum.ensure(g->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream) ||
+      !g->b_poscnt.ensure(g->al, (size_t)std::max<int64_t>(g->num_nodes, 1) * 4, stream))
     return fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_set_weights: device allocation failed");
   g->colsum = (float*)g->b_colsum.ptr;
+  g->poscnt = (int32_t*)g->b_poscnt.ptr;
   const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((g->num_nodes + 7) / 8, (int64_t)num_sms() * 16));
-  if (g->num_nodes > 0) colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, g->num_nodes, g->colsum);
+  if (g->num_nodes > 0)
+    colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, g->num_nodes, g->colsum, g->poscnt);
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -341,6 +377,7 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_indices.reset(g->al, s);
   g->b_weights.reset(g->al, s);
   g->b_colsum.reset(g->al, s);
+  g->b_poscnt.reset(g->al, s);
   g->b_deg.reset(g->al, s);
   g->b_walk.reset(g->al, s);
   g->b_err.reset(g->al, s);
@@ -395,8 +432,8 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
   }
   cudaStream_t stream = (cudaStream_t)stream_;
   if ((st = prepare_blocks(out, stream))) return st;
-  return run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
-                           num_layers, replace, bias_mode, rng_key, stream, *out);
+  return run_nodewise(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
+                      num_layers, replace, bias_mode, rng_key, stream, *out);
 }
 
 gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
@@ -582,6 +619,12 @@ gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out) 
 void gs_blocks_destroy(gs_blocks* b) {
   if (!b) return;
   if (b->aux) gs_blocks_destroy(b->aux);
+  if (b->side) {
+    cudaStreamSynchronize(b->side);
+    cudaStreamDestroy(b->side);
+  }
+  if (b->ev_fork) cudaEventDestroy(b->ev_fork);
+  if (b->ev_join) cudaEventDestroy(b->ev_join);
   cudaStream_t s = b->stream;
   for (int l = 0; l < MAX_LAYERS; ++l) {
     b->b_col[l].reset(b->al, s);

@@ -54,11 +54,12 @@ struct gs_graph {
   int32_t* indices = nullptr;
   float* weights = nullptr;
   float* colsum = nullptr;   // weighted graphs: fp32(sum_fp64 w) per column (a0 pre-processing)
+  int32_t* poscnt = nullptr; // weighted graphs: #{w > 0} per column (a0; the A-Res sample count)
   bool owns = false;
   int sorted = 0;
   int64_t max_in_degree = 0;
   gsb::Allocator al;
-  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_err, b_deg;
+  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_poscnt, b_err, b_deg;
   int32_t* deg = nullptr;    // FastGCN a0 pre-processing: in-degree per node (built on first use)
   gsb::DevBuf b_walk;        // walk index (walk.cu): 16 B per CSC entry, built on the first walk
   const int4* walk_rec = nullptr;
@@ -93,4 +94,6 @@ struct gs_blocks {
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;
   gs_blocks* aux = nullptr;    // ShaDow: the internal node-wise result
+  cudaStream_t side = nullptr; // node-wise: second stream (groups of batches alternate), forked/joined by events
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };

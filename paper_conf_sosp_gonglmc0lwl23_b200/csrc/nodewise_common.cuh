@@ -103,6 +103,24 @@ __device__ __forceinline__ bool ares_maybe_below(uint32_t r, float t) {
   return -__logf(u) * 0.999f <= t;
 }
 
+// A-Res threshold search state: tau is widened / narrowed geometrically, or
+// bisected once both a too-small and a too-large value are known.
+struct TauSearch {
+  float tau, lo, hi;
+  __device__ bool next(int verdict, float tau0) {  // false: give up
+    if (verdict == -3) { tau = -1.0f; return true; }
+    if (verdict == -1) lo = tau;                     // too few below tau
+    else hi = tau < 0.0f ? tau0 * 4.0f : tau;        // too many candidates
+    if (lo > 0.0f && hi > 0.0f) {
+      if (hi <= lo * 1.0001f) return false;
+      tau = sqrtf(lo * hi);
+    } else {
+      tau = lo > 0.0f ? lo * 4.0f : hi * 0.25f;
+    }
+    return true;
+  }
+};
+
 struct AresState {   // per filtering group (warp or CTA), in shared memory
   int m;             // candidates appended (may exceed the capacity)
   int elig;          // eligible (w > 0) edges seen

@@ -264,24 +264,6 @@ __device__ __forceinline__ void nv_cols(const NVParams& P, WarpChunk& C, const N
   d_out = d;
 }
 
-// A-Res threshold search state: tau is widened / narrowed geometrically, or
-// bisected once both a too-small and a too-large value are known.
-struct TauSearch {
-  float tau, lo, hi;
-  __device__ bool next(int verdict, float tau0) {  // false: give up
-    if (verdict == -3) { tau = -1.0f; return true; }
-    if (verdict == -1) lo = tau;                     // too few below tau
-    else hi = tau < 0.0f ? tau0 * 4.0f : tau;        // too many candidates
-    if (lo > 0.0f && hi > 0.0f) {
-      if (hi <= lo * 1.0001f) return false;
-      tau = sqrtf(lo * hi);
-    } else {
-      tau = lo > 0.0f ? lo * 4.0f : hi * 0.25f;
-    }
-    return true;
-  }
-};
-
 __device__ __forceinline__ float nv_tau0(const NVParams& P, int k, int32_t v, int64_t d) {
   const float W = P.core.weights ? __ldg(P.core.colsum + v) : (float)d;
   return W > 0.0f ? 2.0f * (float)k / W : -1.0f;

@@ -29,7 +29,7 @@ namespace cg = cooperative_groups;
 
 namespace gsb {
 
-gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                             int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                             int replace, int bias, uint64_t key, cudaStream_t stream,
                             gs_blocks* blk);
@@ -504,7 +504,7 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
     blk->aux->al = blk->al;
   }
   blk->aux->stream = stream;
-  st = run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias, key,
+  st = run_nodewise(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias, key,
                          stream, blk->aux);
   if (st) return st;
   const gs_blocks* nw = blk->aux;
