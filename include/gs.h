@@ -192,6 +192,30 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
                               const int32_t* fanouts, int num_layers, int replace, int bias_mode,
                               uint64_t rng_key, void* stream, gs_blocks** out);
 
+/* Ragged mini-batches (super-batch with per-batch ID spaces):
+ * as gs_sample_neighbors, but batch b holds seeds [batch_ptr[b],
+ * batch_ptr[b+1]) for any non-decreasing HOST int64[num_batches + 1] with
+ * batch_ptr[0] == 0 and batch_ptr[num_batches] == num_seeds (empty batches
+ * allowed; copied, the caller may free it on return).  Batch b's blocks live
+ * in the fixed regions starting at batch_ptr[b].
+ * Envelope: max batch size * prod(fanouts) <= 2^25.  Errors as
+ * gs_sample_neighbors, plus GS_ERR_INVALID_ARGUMENT for a malformed batch_ptr. */
+gs_status gs_sample_neighbors_ragged(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                                     const int64_t* batch_ptr, int64_t num_batches, int64_t batch_index_base,
+                                     const int32_t* fanouts, int num_layers, int replace, int bias_mode,
+                                     uint64_t rng_key, void* stream, gs_blocks** out);
+
+/* Induce ("induce a subgraph using all the sampled nodes", P:113;
+ * R12) over an existing node-wise result `sampled` (from gs_sample_neighbors
+ * or gs_sample_neighbors_ragged, same stream order): for every batch, U = its
+ * seeds and the rows of every layer, ascending; one block per batch
+ * (num_layers == 1 in *out): col_map == row_map == U, the edges u->v of A with
+ * u, v in U in CSC order.  *out (NULL or a previous result, != sampled) is
+ * library-owned.  Edge overflow -> GS_ERR_CAPACITY at gs_blocks_sync (the
+ * object has grown: call again).  Envelope: N within the cluster shared-
+ * memory bitmap (GS_ERR_NOT_SUPPORTED otherwise). */
+gs_status gs_induce_subgraph(const gs_graph* g, const gs_blocks* sampled, void* stream, gs_blocks** out);
+
 /* ShaDow (R12): node-wise sampling as gs_sample_neighbors
  * (bias_mode UNIFORM or EDGE, no replacement), then for every batch the
  * subgraph of A induced on U = the union of the seeds and all sampled rows,

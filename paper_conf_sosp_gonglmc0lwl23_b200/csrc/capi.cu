@@ -104,6 +104,7 @@ gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seed
   return run_nodewise_hop(g, seeds, num_seeds, nullptr, batch_size, (num_seeds + batch_size - 1) / batch_size,
                           batch_base, fanouts, L, replace, bias, key, stream, blk);
 }
+gs_status run_induce(const gs_graph* g, const gs_blocks* nw, cudaStream_t stream, gs_blocks* blk);
 gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk);
@@ -434,6 +435,47 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
   if ((st = prepare_blocks(out, stream))) return st;
   return run_nodewise(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
                       num_layers, replace, bias_mode, rng_key, stream, *out);
+}
+
+gs_status gs_sample_neighbors_ragged(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
+                                     const int64_t* batch_ptr, int64_t num_batches, int64_t batch_index_base,
+                                     const int32_t* fanouts, int num_layers, int replace, int bias_mode,
+                                     uint64_t rng_key, void* stream_, gs_blocks** out) {
+  if (!batch_ptr || num_batches < 0) return fail(GS_ERR_INVALID_ARGUMENT, "batch_ptr: null or negative num_batches");
+  int64_t maxbs = 1;
+  if (batch_ptr[0] != 0 || batch_ptr[num_batches] != num_seeds)
+    return fail(GS_ERR_INVALID_ARGUMENT, "batch_ptr must start at 0 and end at num_seeds");
+  for (int64_t b = 0; b < num_batches; ++b) {
+    if (batch_ptr[b + 1] < batch_ptr[b]) return fail(GS_ERR_INVALID_ARGUMENT, "batch_ptr must be non-decreasing");
+    maxbs = std::max<int64_t>(maxbs, batch_ptr[b + 1] - batch_ptr[b]);
+  }
+  gs_status st = check_batches(g, seeds, num_seeds, maxbs, batch_index_base, fanouts, num_layers, out);
+  if (st) return st;
+  if (bias_mode < 0 || bias_mode > 2) return fail(GS_ERR_INVALID_ARGUMENT, "unknown bias_mode %d", bias_mode);
+  if (replace && bias_mode != GS_W_UNIFORM)
+    return fail(GS_ERR_NOT_SUPPORTED, "weighted sampling with replacement is not implemented");
+  int64_t prod = maxbs;
+  for (int l = 0; l < num_layers; ++l) {
+    if (fanouts[l] > MAX_FANOUT) return fail(GS_ERR_NOT_SUPPORTED, "fanout must be <= %d", MAX_FANOUT);
+    prod *= fanouts[l];
+    if (prod > MAX_SLOTS_PER_BATCH)
+      return fail(GS_ERR_NOT_SUPPORTED, "max batch size * prod(fanouts) must be <= 2^25");
+  }
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if ((st = prepare_blocks(out, stream))) return st;
+  return run_nodewise_hop(g, seeds, num_seeds, batch_ptr, 0, num_batches, batch_index_base, fanouts, num_layers,
+                          replace, bias_mode, rng_key, stream, *out);
+}
+
+gs_status gs_induce_subgraph(const gs_graph* g, const gs_blocks* sampled, void* stream_, gs_blocks** out) {
+  if (!g || !sampled || !out) return fail(GS_ERR_INVALID_ARGUMENT, "gs_induce_subgraph: null argument");
+  if (*out == sampled) return fail(GS_ERR_INVALID_ARGUMENT, "gs_induce_subgraph: out must differ from sampled");
+  if (sampled->kind != gs_blocks::NODEWISE)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_induce_subgraph: sampled must come from gs_sample_neighbors");
+  cudaStream_t stream = (cudaStream_t)stream_;
+  gs_status st = prepare_blocks(out, stream);
+  if (st) return st;
+  return run_induce(g, sampled, stream, *out);
 }
 
 gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,

@@ -94,6 +94,8 @@ struct gs_blocks {
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
   bool synced = false;
   gs_blocks* aux = nullptr;    // ShaDow: the internal node-wise result
+  int64_t num_seeds = 0, batch_size = 0;  // node-wise: the seeds and (fixed) batch size sampled
+  const int64_t* bptr_dev = nullptr;       // node-wise (hop engine): device seed offsets [nb + 1]
   cudaStream_t side = nullptr; // node-wise: second stream (groups of batches alternate), forked/joined by events
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };

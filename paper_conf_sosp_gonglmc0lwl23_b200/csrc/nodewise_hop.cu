@@ -836,6 +836,9 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   unsigned long long* stat = (unsigned long long*)((char*)blk->b_sched.ptr + std::max<int64_t>(G * L, 1) * 16);
   int64_t* bptr_dev = (int64_t*)((char*)blk->b_sched.ptr + ctr_bytes);
   P.bptr = bptr_dev;
+  blk->bptr_dev = bptr_dev;
+  blk->num_seeds = num_seeds;
+  blk->batch_size = bptr_host ? 0 : batch_size;
 
   P.col0 = (int32_t*)blk->b_col[0].ptr;
   for (int l = 0; l < L; ++l) {

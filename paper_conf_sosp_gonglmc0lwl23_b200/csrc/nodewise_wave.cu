@@ -843,6 +843,9 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   P.G = (int)((nbatch + P.WB - 1) / P.WB);
   P.S = nbatch > 0 ? P.G + 3 * L : 0;  // the last step clears the last group's bitmaps
   blk->kind = gs_blocks::NODEWISE;
+  blk->bptr_dev = nullptr;
+  blk->num_seeds = num_seeds;
+  blk->batch_size = batch_size;
   blk->num_batches = nbatch;
   blk->num_layers = L;
   blk->stream = stream;

@@ -57,7 +57,9 @@ struct SHParams {
   const int64_t* nmeta;             // node-wise meta [b][L][8]
   const int32_t* traces;            // GraphSAINT-RW: walk traces [root][L1] (U source instead of seeds + rows)
   int64_t L1;                       // walk_length + 1
-  int64_t stride;                   // U capacity per batch
+  int64_t stride;                   // U capacity per batch (fixed batches)
+  const int64_t* bptr;              // [nb + 1] seed offsets (ragged batches) or NULL: b * batch_size
+  int64_t mult;                     // U capacity per seed (region of batch b at bstart * mult)
   int32_t* U;                       // [b * stride] U ascending (col_map == row_map)
   int64_t* indptr_out;              // [b * stride + b] CSC over U
   int32_t* row_local;
@@ -114,6 +116,15 @@ __device__ __forceinline__ long long sh_rank(const cg::cluster_group& cl, uint32
   return ss.base[owner] + p[x >> 8] + o[x >> 5] + __popc(w[x >> 5] & ((1u << (x & 31)) - 1u));
 }
 
+// batch b's first seed, seed count and U region (fixed or ragged batches)
+__device__ __forceinline__ int64_t sh_bstart(const SHParams& P, int64_t b) {
+  return P.bptr ? __ldg(P.bptr + b) : b * P.batch_size;
+}
+__device__ __forceinline__ long long sh_T0(const SHParams& P, int64_t b) {
+  return P.bptr ? (long long)(__ldg(P.bptr + b + 1) - __ldg(P.bptr + b))
+                : min(P.batch_size, P.num_seeds - b * P.batch_size);
+}
+
 __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ SHShared ss;
@@ -136,8 +147,9 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     // ---- mark U ----
     for (int i = tid; i < nwords; i += SH_THREADS) bm[i] = 0u;
     cl.sync();
-    const int64_t bstart = b * P.batch_size;
-    const long long T0 = min(P.batch_size, P.num_seeds - bstart);
+    const int64_t bstart = sh_bstart(P, b);
+    const long long T0 = sh_T0(P, b);
+    const int64_t ub = bstart * P.mult;  // the batch's U region
     long long nitems = T0;
     long long cnt_l[MAX_LAYERS];
     if (P.traces) {
@@ -203,7 +215,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     }
     __syncthreads();
     const long long nU = ss.nU;
-    int32_t* U = P.U + b * P.stride;
+    int32_t* U = P.U + ub;
     for (int g = tid; g < ngroups; g += SH_THREADS) {
       long long r = ss.base[rank] + gp[g];
       for (int i = 0; i < 8; ++i) {
@@ -221,8 +233,8 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     // kept edge (row rank, eid) in this warp's private region so that the
     // emit below is a copy, not a second stream of the columns ----
     const long long c_lo = nU * rank / CS, c_hi = nU * (rank + 1) / CS;
-    int32_t* ucnt = P.ucnt + b * P.stride;
-    int64_t* ustart = P.ustart + b * P.stride;
+    int32_t* ucnt = P.ucnt + ub;
+    int64_t* ustart = P.ustart + ub;
     const int64_t wreg = ((int64_t)blockIdx.x * SH_WARPS + warp) * P.wcap;
     int32_t* wst_r = P.stage_row + wreg;
     int64_t* wst_e = P.stage_eid + wreg;
@@ -304,13 +316,13 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
     const long long E = ss.E, ebase = ss.ebase;
     const long long eoff = *cl.map_shared_rank(&ss.eoff, 0);
     const bool fits = eoff + E <= P.edge_cap;
-    int64_t* ip = P.indptr_out + b * P.stride + b;
+    int64_t* ip = P.indptr_out + ub + b;
     for (long long c = c_lo + tid; c < c_hi; c += SH_THREADS) ip[c] = ebase + __ldcg(ucnt + c);
     if (rank == 0 && tid == 0) {
       ip[nU] = E;
       long long* m = (long long*)(P.meta + b * 8);
-      m[0] = nU; m[1] = nU; m[2] = E; m[3] = b * P.stride; m[4] = b * P.stride;
-      m[5] = b * P.stride + b; m[6] = fits ? eoff : 0; m[7] = 0;
+      m[0] = nU; m[1] = nU; m[2] = E; m[3] = ub; m[4] = ub;
+      m[5] = ub + b; m[6] = fits ? eoff : 0; m[7] = 0;
       if (!fits) m[2] = 0;  // nothing was written: an overflowed block is empty (GS_ERR_CAPACITY)
       if (!fits) atomicOr(P.err, ERR_CAPACITY);
     }
@@ -396,10 +408,10 @@ static gs_status induce_envelope(int64_t N, int* CS_out, int64_t* bpc_out) {
 // rows, or walk traces); stride = U capacity per batch; err_src = the device
 // error word of the producing kernel, folded into the result's.
 static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bpc, int64_t nbatch,
-                               int64_t stride, const int* err_src, cudaStream_t stream,
+                               int64_t mult, const int* err_src, cudaStream_t stream,
                                gs_blocks* blk) {
   const Allocator& al = blk->al;
-  const int64_t nodes = nbatch * stride;
+  const int64_t nodes = P.bptr ? P.num_seeds * mult : nbatch * P.batch_size * mult;
   blk->kind = gs_blocks::SHADOW;
   blk->num_batches = nbatch;
   blk->num_layers = 1;
@@ -429,7 +441,8 @@ static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bp
   P.indices = g->indices;
   P.N = g->num_nodes;
   P.num_batches = nbatch;
-  P.stride = stride;
+  P.mult = mult;
+  P.stride = P.batch_size * mult;
   P.U = lb.row_map;
   P.indptr_out = lb.indptr;
   P.row_local = lb.row_local;
@@ -490,6 +503,8 @@ static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bp
   return GS_OK;
 }
 
+gs_status run_induce(const gs_graph* g, const gs_blocks* nw, cudaStream_t stream, gs_blocks* blk);
+
 gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                      int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                      int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
@@ -507,26 +522,34 @@ gs_status run_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
   st = run_nodewise(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, 0, bias, key,
                          stream, blk->aux);
   if (st) return st;
-  const gs_blocks* nw = blk->aux;
-  // 2. induce on U = seeds + every hop's rows
-  const int64_t nbatch = (num_seeds + batch_size - 1) / batch_size;
-  int64_t sumK = 0, prod = 1;
-  for (int l = 0; l < L; ++l) {
-    prod *= fanouts[l];
-    sumK += prod;
-  }
+  return run_induce(g, blk->aux, stream, blk);
+}
+
+// Induce (a7; R12) over a node-wise result: per batch U = its
+// seeds + every hop's rows, ascending; the subgraph of A induced on U.
+gs_status run_induce(const gs_graph* g, const gs_blocks* nw, cudaStream_t stream, gs_blocks* blk) {
+  int CS = 1;
+  int64_t bpc = 0;
+  gs_status st = induce_envelope(g->num_nodes, &CS, &bpc);
+  if (st) return st;
+  if (nw->kind != gs_blocks::NODEWISE || (nw->num_seeds <= 0 && nw->num_batches > 0))
+    return fail(GS_ERR_INVALID_ARGUMENT, "induce: the sampled blocks must be a node-wise result");
+  const int L = nw->num_layers;
+  const int64_t num_seeds = nw->num_seeds;
+  int64_t sumK = 0;
   SHParams P = {};
-  P.seeds = seeds;
+  P.seeds = nw->layers[0].col_map;
   P.num_seeds = num_seeds;
-  P.batch_size = batch_size;
+  P.batch_size = nw->batch_size;
+  P.bptr = nw->bptr_dev;
   P.L = L;
   for (int l = 0; l < L; ++l) {
     P.rows[l] = nw->layers[l].row_map;
-    P.K[l] = l == 0 ? fanouts[0] : P.K[l - 1] * fanouts[l];
+    P.K[l] = num_seeds > 0 ? nw->layers[l].row_capacity / num_seeds : 0;
+    sumK += P.K[l];
   }
   P.nmeta = (const int64_t*)nw->b_meta.ptr;
-  return launch_induce(g, P, CS, bpc, nbatch, batch_size * (1 + sumK), (const int*)nw->b_err.ptr,
-                       stream, blk);
+  return launch_induce(g, P, CS, bpc, nw->num_batches, 1 + sumK, (const int*)nw->b_err.ptr, stream, blk);
 }
 
 // GraphSAINT-RW (Table 2; R26): a DeepWalk walk from every root
@@ -556,7 +579,7 @@ gs_status run_saint_rw(const gs_graph* g, const int32_t* roots, int64_t num_root
   P.batch_size = batch_size;
   P.traces = (const int32_t*)blk->b_trace.ptr;
   P.L1 = L1;
-  return launch_induce(g, P, CS, bpc, nbatch, batch_size * L1, werr, stream, blk);
+  return launch_induce(g, P, CS, bpc, nbatch, L1, werr, stream, blk);
 }
 
 }  // namespace gsb

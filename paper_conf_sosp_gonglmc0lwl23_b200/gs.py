@@ -32,7 +32,8 @@ META_FIELDS = 8
 EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
-           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_shadow", "gs_sample_saint_rw", "gs_sample_pinsage",
+           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_neighbors_ragged",
+           "gs_induce_subgraph", "gs_sample_shadow", "gs_sample_saint_rw", "gs_sample_pinsage",
            "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
            "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
@@ -126,6 +127,9 @@ def load_library(path: str = LIB_PATH):
     L.gs_graph_destroy.restype = None
     L.gs_sample_neighbors.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, u64, vp,
                                       ctypes.POINTER(vp)]
+    L.gs_sample_neighbors_ragged.argtypes = [vp, vp, i64, vp, i64, i64, vp, i32, i32, i32, u64, vp,
+                                             ctypes.POINTER(vp)]
+    L.gs_induce_subgraph.argtypes = [vp, vp, vp, ctypes.POINTER(vp)]
     L.gs_sample_shadow.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, u64, vp, ctypes.POINTER(vp)]
     L.gs_sample_pinsage.argtypes = [vp, vp, i64, i64, i64, vp, i32, i32, i32, ctypes.c_float, u64,
                                     vp, ctypes.POINTER(vp)]
@@ -360,20 +364,52 @@ def _host_i32(xs):
 
 
 def sample_neighbors(g: Graph, seeds: torch.Tensor, fanouts, batch_size=None, batch_index_base=0,
-                     replace=False, bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None):
-    """GraphSAGE / KGCN / weighted A-Res / PASS-style node-wise sampling (gs_sample_neighbors)."""
+                     replace=False, bias_mode=UNIFORM, rng_key=0, stream=None, out: Blocks = None,
+                     batch_ptr=None):
+    """GraphSAGE / KGCN / weighted A-Res / PASS-style node-wise sampling
+    (gs_sample_neighbors; gs_sample_neighbors_ragged when batch_ptr -- a host
+    sequence of num_batches + 1 seed offsets -- is given)."""
     L = load_library()
     _drain()
     seeds = seeds.to(torch.int32).contiguous()
-    bs = int(batch_size or max(1, seeds.numel()))
     out = out or Blocks()
     f = _host_i32(fanouts)
-    _check(L.gs_sample_neighbors(g.handle, _ptr(seeds), seeds.numel(), bs, int(batch_index_base),
-                                 f, len(fanouts), int(replace), int(bias_mode),
-                                 ctypes.c_uint64(rng_key), _stream_ptr(stream),
-                                 ctypes.byref(out._h)), "gs_sample_neighbors")
+    if batch_ptr is not None:
+        bp = (ctypes.c_int64 * len(batch_ptr))(*[int(x) for x in batch_ptr])
+        _check(L.gs_sample_neighbors_ragged(g.handle, _ptr(seeds), seeds.numel(), bp, len(batch_ptr) - 1,
+                                            int(batch_index_base), f, len(fanouts), int(replace),
+                                            int(bias_mode), ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                                            ctypes.byref(out._h)), "gs_sample_neighbors_ragged")
+    else:
+        bs = int(batch_size or max(1, seeds.numel()))
+        _check(L.gs_sample_neighbors(g.handle, _ptr(seeds), seeds.numel(), bs, int(batch_index_base),
+                                     f, len(fanouts), int(replace), int(bias_mode),
+                                     ctypes.c_uint64(rng_key), _stream_ptr(stream),
+                                     ctypes.byref(out._h)), "gs_sample_neighbors")
     out.synced = False
     out._seeds = seeds
+    return out
+
+
+def induce_subgraph(g: Graph, sampled: Blocks, stream=None, out: Blocks = None, retry=True):
+    """gs_induce_subgraph: per batch of a node-wise result, the subgraph of A
+    induced on its seeds + sampled rows (ascending)."""
+    L = load_library()
+    _drain()
+    out = out or Blocks()
+    for attempt in range(3):
+        _check(L.gs_induce_subgraph(g.handle, sampled._h, _stream_ptr(stream), ctypes.byref(out._h)),
+               "gs_induce_subgraph")
+        out.synced = False
+        if not retry:
+            break
+        try:
+            out.sync()
+            break
+        except GSError as e:
+            if e.status != 7 or attempt == 2:
+                raise
+    out._sampled = sampled
     return out
 
 
