@@ -50,6 +50,9 @@ const char* gs_last_error(void);
 const char* gs_status_string(gs_status s);
 /* Library version: major*10000 + minor*100 + patch. */
 int gs_version(void);
+/* Kernels this library has enqueued from the calling thread so far (a
+ * cumulative counter: the difference around a call = its kernel launches). */
+int64_t gs_kernel_launches(void);
 
 /* Device-memory hook.  Every device buffer the library owns (graph copies,
  * blocks, workspaces) is obtained through alloc(bytes, stream, ctx) and
@@ -164,6 +167,14 @@ gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out);
 gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
                          int64_t* indptr, int32_t* row_map, int64_t* totals, void* stream);
 void gs_blocks_destroy(gs_blocks* b);
+/* Profiling (diagnostic, off by default): while on, the node-wise sampler
+ * records a CUDA event after each of its kernels, runs them on one stream and
+ * synchronises at the end of the call; gs_blocks_profile(b, i, &name, &ms)
+ * then returns the i-th (kernel, milliseconds) pair of that call
+ * (GS_ERR_INVALID_ARGUMENT past the last).  name stays valid until the next
+ * call on b. */
+gs_status gs_set_profiling(int on);
+gs_status gs_blocks_profile(const gs_blocks* b, int i, const char** name, double* ms);
 
 /* ------------------------------------------------------------------------ */
 /* Node-wise sampling (a1 + a3 + a6; + a2 for PASS-style).                    */

@@ -19,6 +19,8 @@ namespace gsb {
 // errors
 // ---------------------------------------------------------------------------
 static thread_local char g_err[512] = "";
+thread_local int64_t g_launches = 0;
+bool g_profiling = false;
 
 void set_error(const char* fmt, ...) {
   va_list ap;
@@ -212,7 +214,22 @@ const char* gs_status_string(gs_status s) {
   return "GS_ERR_UNKNOWN";
 }
 
-int gs_version(void) { return 100; }
+int gs_version(void) { return 200; }
+
+int64_t gs_kernel_launches(void) { return g_launches; }
+
+gs_status gs_set_profiling(int on) {
+  g_profiling = on != 0;
+  return GS_OK;
+}
+
+gs_status gs_blocks_profile(const gs_blocks* b, int i, const char** name, double* ms) {
+  if (!b || !name || !ms) return fail(GS_ERR_INVALID_ARGUMENT, "gs_blocks_profile: null argument");
+  if (i < 0 || i >= (int)b->prof.size()) return fail(GS_ERR_INVALID_ARGUMENT, "gs_blocks_profile: no entry %d", i);
+  *name = b->prof[i].first.c_str();
+  *ms = b->prof[i].second;
+  return GS_OK;
+}
 
 gs_status gs_set_allocator(gs_alloc_fn alloc, gs_free_fn free_fn, void* ctx) {
   if ((alloc == nullptr) != (free_fn == nullptr))
@@ -302,7 +319,7 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
   const int sms = num_sms();
   int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((num_nodes + 7) / 8, (int64_t)sms * 16));
   validate_csc_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->indices, num_nodes,
-                                                             num_edges, d_flags, d_maxdeg);
+                                                             num_edges, d_flags, d_maxdeg); count_launch();
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cleanup(cuda_fail(e, "validate_csc_kernel launch"));
   int h[16] = {0};
@@ -323,7 +340,7 @@ gs_status gs_graph_create(const int64_t* indptr, const int32_t* indices, const f
     g->colsum = (float*)g->b_colsum.ptr;
     g->poscnt = (int32_t*)g->b_poscnt.ptr;
     colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, num_nodes, g->colsum,
-                                                         g->poscnt);
+                                                         g->poscnt); count_launch();
     e = cudaGetLastError();
     if (e != cudaSuccess) return cleanup(cuda_fail(e, "colsum_kernel launch"));
   }
@@ -351,8 +368,10 @@ gs_status gs_graph_set_weights(gs_graph* g, const float* weights, uint32_t flags
   g->colsum = (float*)g->b_colsum.ptr;
   g->poscnt = (int32_t*)g->b_poscnt.ptr;
   const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((g->num_nodes + 7) / 8, (int64_t)num_sms() * 16));
-  if (g->num_nodes > 0)
+  if (g->num_nodes > 0) {
     colsum_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->weights, g->num_nodes, g->colsum, g->poscnt);
+    count_launch();
+  }
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

@@ -14,6 +14,11 @@ constexpr int MAX_LAYERS = 8;
 constexpr int MAX_FANOUT = 32;
 constexpr int64_t MAX_SLOTS_PER_BATCH = (1ll << 25);  // table value field (R3 positions)
 
+// ---- kernel launches enqueued by this thread (gs_kernel_launches) ----
+extern thread_local int64_t g_launches;
+extern bool g_profiling;  // gs_set_profiling
+inline void count_launch(int n = 1) { g_launches += n; }
+
 // ---- error reporting (thread-local message) ----
 void set_error(const char* fmt, ...);
 gs_status fail(gs_status st, const char* fmt, ...);
@@ -98,4 +103,5 @@ struct gs_blocks {
   const int64_t* bptr_dev = nullptr;       // node-wise (hop engine): device seed offsets [nb + 1]
   cudaStream_t side = nullptr; // node-wise: second stream (groups of batches alternate), forked/joined by events
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  std::vector<std::pair<std::string, double>> prof;  // per-kernel ms of the last call (profiling on)
 };

@@ -657,7 +657,7 @@ gs_status run_layerwise_old(const gs_graph* g, const int32_t* seeds, int64_t num
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
-  layerwise_kernel<<<nctas, LW_THREADS, dyn, stream>>>(P);
+  layerwise_kernel<<<nctas, LW_THREADS, dyn, stream>>>(P); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

@@ -705,8 +705,10 @@ gs_status layerwise_degree_array(const gs_graph* g, cudaStream_t stream) {
     return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (degree array)");
   gm->deg = (int32_t*)gm->b_deg.ptr;
   const int64_t blocks = std::min<int64_t>((g->num_nodes + 255) / 256, 148 * 16);
-  if (g->num_nodes > 0)
+  if (g->num_nodes > 0) {
     degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
+    count_launch();
+  }
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -852,7 +854,7 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
-  layerwise_bm_kernel<<<nctas, LB_THREADS, smem, stream>>>(P);
+  layerwise_bm_kernel<<<nctas, LB_THREADS, smem, stream>>>(P); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

@@ -699,7 +699,7 @@ static gs_status launch_select(const HopParams& P, int l, int64_t b0, int nbg, u
     if (getenv("GS_VERBOSE"))
       fprintf(stderr, "hop_select<%d,%d>: smem %zu B, %d CTAs/SM\n", (int)W, KCAP, smem, per_sm);
   }
-  kfn<<<grid, HS_THREADS, smem, stream>>>(P, l, b0, nbg, claim);
+  kfn<<<grid, HS_THREADS, smem, stream>>>(P, l, b0, nbg, claim); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -812,7 +812,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   // group's HBM-bound select (each stream has its own bitmap slots)
   int NS = G > 1 ? 2 : 1;
   if (const char* e = getenv("GS_HOP_STREAMS")) NS = std::max(1, std::min(2, atoi(e)));
-  if (getenv("GS_HOP_TIMING")) NS = 1;
+  if (g_profiling || getenv("GS_HOP_TIMING")) NS = 1;
   // workspace: bitmaps + summaries (kept clear between calls), column staging
   const int64_t o_bm = 0;
   const int64_t o_summ = a256h(o_bm + NS * WB * P.nwp * 8);
@@ -868,13 +868,15 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     GS_CUDA_TRY(cudaMemcpyAsync(bptr_dev, bptr_host, (nbatch + 1) * 8, cudaMemcpyHostToDevice, stream));
   } else {
     bptr_fill_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((nbatch + 256) / 256, 1024)), 256, 0,
-                       stream>>>(bptr_dev, nbatch, batch_size, num_seeds);
+                       stream>>>(bptr_dev, nbatch, batch_size, num_seeds); count_launch();
     GS_CUDA_TRY(cudaGetLastError());
   }
   if (nbatch == 0) return GS_OK;
 
-  // GS_HOP_TIMING: per-kernel event timing (debug aid; synchronises)
-  const bool timing = getenv("GS_HOP_TIMING") != nullptr;
+  // profiling (gs_set_profiling / GS_HOP_TIMING): per-kernel event timing,
+  // one stream, synchronises at the end of the call; kept in the result
+  const bool timing = g_profiling || getenv("GS_HOP_TIMING") != nullptr;
+  blk->prof.clear();
   std::vector<cudaEvent_t> ev;
   std::vector<std::string> evname;
   auto mark = [&](const char* name, int l) {
@@ -912,7 +914,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       const Scan srow{c4 + 1, st};
       st += WB * ntile[l];
       {
-        hop_nprep_kernel<<<(unsigned)(nbg * nseg_max[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, snp);
+        hop_nprep_kernel<<<(unsigned)(nbg * nseg_max[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, snp); count_launch();
         GS_CUDA_TRY(cudaGetLastError());
         mark("nprep", l);
       }
@@ -928,16 +930,16 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       }
       if (rc) return rc;
       mark("select", l);
-      hop_rows_kernel<<<(unsigned)(nbg * ntile[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, ntile[l], srow);
+      hop_rows_kernel<<<(unsigned)(nbg * ntile[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, ntile[l], srow); count_launch();
       GS_CUDA_TRY(cudaGetLastError());
       mark("rows", l);
       const int64_t tiles = (maxbs * P.K[l] + RL_TILE - 1) / RL_TILE;
       hop_relabel_kernel<<<dim3((unsigned)std::max<int64_t>(tiles, 1), (unsigned)nbg), HB_THREADS, 0, stream>>>(
-          P, l, b0);
+          P, l, b0); count_launch();
       mark("relabel", l);
       const unsigned ct = P.use_sum[l] ? (unsigned)std::max<int64_t>(1, std::min<int64_t>(tiles, 64))
                                        : (unsigned)((P.nw + CLEAR_TILE - 1) / CLEAR_TILE);
-      hop_clear_kernel<<<dim3(ct, (unsigned)nbg), HB_THREADS, 0, stream>>>(P, l, b0);
+      hop_clear_kernel<<<dim3(ct, (unsigned)nbg), HB_THREADS, 0, stream>>>(P, l, b0); count_launch();
       GS_CUDA_TRY(cudaGetLastError());
       mark("clear", l);
     }
@@ -959,9 +961,12 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     }
     float tot = 0.f;
     cudaEventElapsedTime(&tot, ev.front(), ev.back());
-    fprintf(stderr, "nodewise_hop timing (ms): total %.3f", tot);
-    for (auto& a : acc) fprintf(stderr, " %s %.3f", a.first.c_str(), a.second);
-    fprintf(stderr, "\n");
+    for (auto& a : acc) blk->prof.push_back({"hop_" + a.first, (double)a.second});
+    if (getenv("GS_HOP_TIMING")) {
+      fprintf(stderr, "nodewise_hop timing (ms): total %.3f", tot);
+      for (auto& a : acc) fprintf(stderr, " %s %.3f", a.first.c_str(), a.second);
+      fprintf(stderr, "\n");
+    }
     for (auto e : ev) cudaEventDestroy(e);
   }
   return GS_OK;

@@ -965,7 +965,7 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   }
   void* args[] = {&P};
   GS_CUDA_TRY(cudaLaunchCooperativeKernel(kfn, dim3(grid),
-                                          dim3(NV_THREADS), args, smem, stream));
+                                          dim3(NV_THREADS), args, smem, stream)); count_launch();
   if (trace_path) {  // tracing aid: per-super-step timestamps
     std::vector<unsigned long long> h((size_t)P.S * 4);
     GS_CUDA_TRY(cudaStreamSynchronize(stream));

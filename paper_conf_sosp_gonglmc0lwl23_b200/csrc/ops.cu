@@ -80,16 +80,16 @@ static gs_status scan_inclusive(int64_t* a, int64_t n, const Allocator& al, cuda
   if (n <= 0) return GS_OK;
   const int64_t tiles = (n + SCAN_TILE - 1) / SCAN_TILE;
   if (tiles == 1) {
-    scan_tile_kernel<<<1, SCAN_THREADS, 0, s>>>(a, n, nullptr);
+    scan_tile_kernel<<<1, SCAN_THREADS, 0, s>>>(a, n, nullptr); count_launch();
     GS_CUDA_TRY(cudaGetLastError());
     return GS_OK;
   }
   DevBuf t;
   if (!t.ensure(al, (size_t)tiles * 8, s)) return fail(GS_ERR_OUT_OF_MEMORY, "scan workspace");
-  scan_tile_kernel<<<(unsigned)tiles, SCAN_THREADS, 0, s>>>(a, n, (int64_t*)t.ptr);
+  scan_tile_kernel<<<(unsigned)tiles, SCAN_THREADS, 0, s>>>(a, n, (int64_t*)t.ptr); count_launch();
   gs_status st = scan_inclusive((int64_t*)t.ptr, tiles, al, s);
   if (st == GS_OK) {
-    scan_add_kernel<<<grid_for(n, 256), 256, 0, s>>>(a, n, (const int64_t*)t.ptr);
+    scan_add_kernel<<<grid_for(n, 256), 256, 0, s>>>(a, n, (const int64_t*)t.ptr); count_launch();
     if (cudaGetLastError() != cudaSuccess) st = fail(GS_ERR_CUDA, "scan_add_kernel launch");
   }
   t.reset(al, s);
@@ -381,7 +381,7 @@ gs_status gs_matrix_slice_columns(const gs_graph* g, const int32_t* cols, int64_
   GS_CUDA_TRY(cudaMemsetAsync(m->b_indptr.ptr, 0, 8, s));
   int64_t* ip = (int64_t*)m->b_indptr.ptr;
   if (n_cols > 0) {
-    col_degree_kernel<<<grid_for(n_cols, 256), 256, 0, s>>>(g->indptr, g->num_nodes, cols, n_cols, ip, (int*)err.ptr);
+    col_degree_kernel<<<grid_for(n_cols, 256), 256, 0, s>>>(g->indptr, g->num_nodes, cols, n_cols, ip, (int*)err.ptr); count_launch();
     GS_CUDA_TRY(cudaGetLastError());
     if ((st = scan_inclusive(ip + 1, n_cols, m->al, s))) return st;
   }
@@ -397,7 +397,7 @@ gs_status gs_matrix_slice_columns(const gs_graph* g, const int32_t* cols, int64_
   if (n_cols > 0) {
     col_copy_kernel<<<grid_for(n_cols, OPS_THREADS), OPS_THREADS, 0, s>>>(
         g->indptr, g->indices, g->weights, g->num_nodes, cols, n_cols, ip, (int32_t*)m->b_row.ptr,
-        (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr);
+        (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr); count_launch();
     GS_CUDA_TRY(cudaGetLastError());
   }
   return GS_OK;
@@ -420,11 +420,13 @@ gs_status gs_matrix_slice_rows(const gs_matrix* in, const int32_t* rows, int64_t
   GS_CUDA_TRY(cudaMemsetAsync(err.ptr, 0, 4, s));
   GS_CUDA_TRY(cudaMemsetAsync(m->b_indptr.ptr, 0, 8, s));
   int64_t* ip = (int64_t*)m->b_indptr.ptr;
-  if (n_rows > 0)
+  if (n_rows > 0) {
     mark_rows_kernel<<<grid_for(n_rows, 256), 256, 0, s>>>(rows, n_rows, in->num_nodes, (uint32_t*)bm.ptr, (int*)err.ptr);
+    count_launch();
+  }
   if (n > 0) {
     row_count_kernel<<<grid_for(n * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
-        (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr, n, (const uint32_t*)bm.ptr, ip);
+        (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr, n, (const uint32_t*)bm.ptr, ip); count_launch();
     GS_CUDA_TRY(cudaGetLastError());
     if ((st = scan_inclusive(ip + 1, n, m->al, s))) return st;
   }
@@ -438,7 +440,7 @@ gs_status gs_matrix_slice_rows(const gs_matrix* in, const int32_t* rows, int64_t
     row_copy_kernel<<<grid_for(n * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
         (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr, (const int64_t*)in->b_eid.ptr,
         (const float*)in->b_val.ptr, n, (const uint32_t*)bm.ptr, ip, (int32_t*)m->b_row.ptr,
-        (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr);
+        (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr); count_launch();
     if (cudaGetLastError() != cudaSuccess) st = fail(GS_ERR_CUDA, "row_copy_kernel launch");
   }
   bm.reset(m->al, s);
@@ -453,7 +455,7 @@ gs_status gs_matrix_sum(const gs_matrix* m, int axis, float* out, void* stream_)
   if (axis == 0) {
     if (m->n_cols > 0) {
       col_sum_kernel<<<grid_for(m->n_cols * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
-          (const int64_t*)m->b_indptr.ptr, (const float*)m->b_val.ptr, m->n_cols, out);
+          (const int64_t*)m->b_indptr.ptr, (const float*)m->b_val.ptr, m->n_cols, out); count_launch();
       GS_CUDA_TRY(cudaGetLastError());
     }
     return GS_OK;
@@ -462,10 +464,15 @@ gs_status gs_matrix_sum(const gs_matrix* m, int axis, float* out, void* stream_)
   const int64_t N = m->num_nodes;
   if (!acc.ensure(m->al, (size_t)std::max<int64_t>(N, 1) * 8, s)) return fail(GS_ERR_OUT_OF_MEMORY, "row-sum accumulator");
   GS_CUDA_TRY(cudaMemsetAsync(acc.ptr, 0, (size_t)std::max<int64_t>(N, 1) * 8, s));
-  if (m->nnz > 0)
+  if (m->nnz > 0) {
     row_sum_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((const int32_t*)m->b_row.ptr, (const float*)m->b_val.ptr,
                                                         m->nnz, (double*)acc.ptr);
-  if (N > 0) to_float_kernel<<<grid_for(N, 256), 256, 0, s>>>((const double*)acc.ptr, N, out);
+    count_launch();
+  }
+  if (N > 0) {
+    to_float_kernel<<<grid_for(N, 256), 256, 0, s>>>((const double*)acc.ptr, N, out);
+    count_launch();
+  }
   cudaError_t e = cudaGetLastError();
   acc.reset(m->al, s);
   if (e != cudaSuccess) return cuda_fail(e, "gs_matrix_sum(axis=1)");
@@ -477,12 +484,14 @@ gs_status gs_matrix_broadcast(gs_matrix* m, int op, const float* V, int axis, vo
     return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_broadcast: bad argument");
   cudaStream_t s = (cudaStream_t)stream_;
   if (m->nnz == 0) return GS_OK;
-  if (axis == 0)
+  if (axis == 0) {
     bcast_col_kernel<<<grid_for(m->n_cols * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
         (const int64_t*)m->b_indptr.ptr, (float*)m->b_val.ptr, m->n_cols, op, V);
+    count_launch();
+  }
   else
     bcast_row_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((const int32_t*)m->b_row.ptr, (float*)m->b_val.ptr,
-                                                          m->nnz, op, V);
+                                                          m->nnz, op, V); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -490,7 +499,7 @@ gs_status gs_matrix_broadcast(gs_matrix* m, int op, const float* V, int axis, vo
 gs_status gs_matrix_elementwise(gs_matrix* m, int op, float x, void* stream_) {
   if (!m || op < GS_OP_ADD || op > GS_OP_POW) return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_elementwise: bad argument");
   if (m->nnz == 0) return GS_OK;
-  map_kernel<<<grid_for((m->nnz + 3) / 4, 256), 256, 0, (cudaStream_t)stream_>>>((float*)m->b_val.ptr, m->nnz, op, x);
+  map_kernel<<<grid_for((m->nnz + 3) / 4, 256), 256, 0, (cudaStream_t)stream_>>>((float*)m->b_val.ptr, m->nnz, op, x); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -506,12 +515,14 @@ gs_status gs_matrix_row_ids(const gs_matrix* m, int32_t* out, int64_t* n_out, vo
     return fail(GS_ERR_OUT_OF_MEMORY, "row() workspace");
   gs_status st = GS_OK;
   GS_CUDA_TRY(cudaMemsetAsync(bm.ptr, 0, (size_t)nw * 4, s));
-  if (m->nnz > 0)
+  if (m->nnz > 0) {
     mark_all_rows_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((const int32_t*)m->b_row.ptr, m->nnz, (uint32_t*)bm.ptr);
-  word_count_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (int64_t*)cnt.ptr);
+    count_launch();
+  }
+  word_count_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (int64_t*)cnt.ptr); count_launch();
   st = scan_inclusive((int64_t*)cnt.ptr, nw, m->al, s);
   if (st == GS_OK) {
-    emit_rows_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (const int64_t*)cnt.ptr, out);
+    emit_rows_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (const int64_t*)cnt.ptr, out); count_launch();
     if (cudaGetLastError() != cudaSuccess) st = fail(GS_ERR_CUDA, "emit_rows_kernel launch");
     else if (cudaMemcpyAsync(n_out, (int64_t*)cnt.ptr + nw - 1, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
              cudaStreamSynchronize(s) != cudaSuccess)

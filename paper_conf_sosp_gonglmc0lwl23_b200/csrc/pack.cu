@@ -98,7 +98,7 @@ extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_
   const gs_layer_buffers& lb = b->layers[layer];
   int64_t* off = (int64_t*)mb->b_pack.ptr;
   pack_scan_kernel<<<1, PK_THREADS, 0, stream>>>((const int64_t*)b->b_meta.ptr, nb, b->num_layers, layer,
-                                                 off, totals);
+                                                 off, totals); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   if (nb == 0) return GS_OK;
   PackParams P;
@@ -122,7 +122,7 @@ extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t grid = std::min<int64_t>(nb, (int64_t)sms * 4);
-  pack_copy_kernel<<<(unsigned)grid, PK_THREADS, 0, stream>>>(P);
+  pack_copy_kernel<<<(unsigned)grid, PK_THREADS, 0, stream>>>(P); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

@@ -175,10 +175,10 @@ extern "C" gs_status gs_pass_attention(const gs_graph* g, const void* X, int F, 
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((N + PA_WARPS - 1) / PA_WARPS, (int64_t)sms * 8));
     const float* Pp = (const float*)P.ptr;
     switch (H) {
-      case 8: pass_att_kernel<16><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
-      case 16: pass_att_kernel<32><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
-      case 32: pass_att_kernel<64><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
-      default: pass_att_kernel<128><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); break;
+      case 8: pass_att_kernel<16><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); count_launch(); break;
+      case 16: pass_att_kernel<32><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); count_launch(); break;
+      case 32: pass_att_kernel<64><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); count_launch(); break;
+      default: pass_att_kernel<128><<<grid, PA_THREADS, 0, s>>>(g->indptr, g->indices, g->weights, g->colsum, Pp, N, s0, s1, s2, att); count_launch(); break;
     }
     ce = cudaGetLastError();
     if (ce != cudaSuccess) st = cuda_fail(ce, "pass_att_kernel launch");

@@ -441,7 +441,7 @@ gs_status run_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num_seeds
   blk->ws_stride_prev = layout;
   P.bitmap = (uint32_t*)blk->b_ws.ptr;
   P.gprefix = (int32_t*)((char*)blk->b_ws.ptr + grid * P.nwords * 4);
-  pinsage_kernel<<<(unsigned)grid, PS_THREADS, smem, stream>>>(P);
+  pinsage_kernel<<<(unsigned)grid, PS_THREADS, smem, stream>>>(P); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

@@ -500,6 +500,7 @@ static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bp
     P.ustart = (int64_t*)((char*)blk->b_ws.ptr + o_s);
   }
   GS_CUDA_TRY(cudaLaunchKernelEx(&cfg, shadow_induce_kernel, P));
+  count_launch();
   return GS_OK;
 }
 

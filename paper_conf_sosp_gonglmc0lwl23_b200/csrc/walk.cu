@@ -183,7 +183,7 @@ static const int4* walk_index(const gs_graph* g, cudaStream_t stream, bool plain
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  walk_index_kernel<<<sms * 16, 256, 0, stream>>>(g->indptr, g->indices, g->num_edges, (int4*)gm->b_walk.ptr);
+  walk_index_kernel<<<sms * 16, 256, 0, stream>>>(g->indptr, g->indices, g->num_edges, (int4*)gm->b_walk.ptr); count_launch();
   if (cudaGetLastError() != cudaSuccess) {
     gm->walk_index_failed = true;
     return nullptr;
@@ -220,7 +220,7 @@ gs_status launch_walk(const gs_graph* g, const int32_t* starts, int64_t num_walk
   int64_t blocks = (num_walkers + threads - 1) / threads;
   const int64_t max_blocks = (int64_t)sms * 8 * 64;
   if (blocks > max_blocks) blocks = max_blocks;
-  walk_kernel<<<(unsigned)blocks, threads, 0, stream>>>(P);
+  walk_kernel<<<(unsigned)blocks, threads, 0, stream>>>(P); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }

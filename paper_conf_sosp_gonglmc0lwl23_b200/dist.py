@@ -27,9 +27,25 @@ def seed_slice(num_seeds: int, batch_size: int, lo_batch: int, hi_batch: int) ->
     return min(num_seeds, lo_batch * batch_size), min(num_seeds, hi_batch * batch_size)
 
 
+def shard_epoch(num_inputs: int, batch_size: int | None, world: int, rank: int) -> tuple[int, int, int]:
+    """Strong-scaling split of ONE epoch: returns (s0, s1, base):
+    this rank's slice [s0, s1) of the epoch's inputs and the global index of its
+    first unit, which keys the RNG so that the union over ranks equals a
+    single-process run.  batch_size > 0: the units are mini-batches (contiguous
+    batch ranges, base = first global batch index); batch_size None: the units
+    are walkers (contiguous walker ranges, base = first global walker index)."""
+    if batch_size:
+        nb = (num_inputs + batch_size - 1) // batch_size
+        lo, hi = shard_range(nb, world, rank)
+        s0, s1 = seed_slice(num_inputs, batch_size, lo, hi)
+        return s0, s1, lo
+    lo, hi = shard_range(num_inputs, world, rank)
+    return lo, hi, lo
+
+
 def weak_batch_base(rank: int, num_batches: int) -> int:
-    """Weak scaling: rank r samples a whole epoch with global batch ids
-    r * num_batches + b (a different epoch per rank)."""
+    """Weak scaling (bench.py --scaling weak only): rank r samples a whole
+    epoch with global batch ids r * num_batches + b (a different epoch per rank)."""
     return rank * num_batches
 
 

@@ -29,7 +29,8 @@ WALK_FORCE_NODE2VEC = 1
 META_FIELDS = 8
 
 # Every symbol include/gs.h declares (checked by tests/test_capi_symbols.py).
-EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_set_allocator",
+EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_kernel_launches", "gs_set_profiling", "gs_blocks_profile",
+           "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
            "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_neighbors_ragged",
@@ -119,6 +120,11 @@ def load_library(path: str = LIB_PATH):
     vp, i64, i32, u64, u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_uint64, ctypes.c_uint32
     L.gs_last_error.restype = ctypes.c_char_p
     L.gs_status_string.restype = ctypes.c_char_p
+    L.gs_kernel_launches.restype = ctypes.c_int64
+    L.gs_kernel_launches.argtypes = []
+    L.gs_set_profiling.argtypes = [ctypes.c_int]
+    L.gs_blocks_profile.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.POINTER(ctypes.c_char_p),
+                                    ctypes.POINTER(ctypes.c_double)]
     L.gs_status_string.argtypes = [i32]
     L.gs_set_allocator.argtypes = [_ALLOC_FN, _FREE_FN, vp]
     L.gs_graph_create.argtypes = [vp, vp, vp, i64, i64, u32, vp, ctypes.POINTER(vp)]
@@ -323,8 +329,13 @@ class Blocks:
         """gs_blocks_pack: layer `layer` of every batch packed densely on the
         device (batch order).  Returns device tensors (capacity-sized; the used
         prefix lengths are in `totals` = device int64 [edges, indptr entries, rows])."""
+        cap = self.layer_capacity(layer)
+        if out is not None:  # the C call writes up to the layer's capacity: check the caller's buffers
+            for k, n in (("row_local", cap["edges"]), ("eid", cap["edges"]), ("indptr", cap["indptr"]),
+                         ("row_map", cap["rows"])):
+                if out[k].numel() < n:
+                    raise GSError(1, f"pack: out['{k}'] holds {out[k].numel()} < layer capacity {n}")
         if out is None:
-            cap = self.layer_capacity(layer)
             dev = torch.device("cuda", torch.cuda.current_device())
             out = {"row_local": torch.empty(cap["edges"], dtype=torch.int32, device=dev),
                    "eid": torch.empty(cap["edges"], dtype=torch.int64, device=dev),
@@ -620,3 +631,25 @@ def random_walk(g: Graph, starts: torch.Tensor, length: int, p=1.0, q=1.0, walke
 
 def walk_check(g: Graph, stream=None):
     _check(load_library().gs_walk_check(g.handle, _stream_ptr(stream)), "gs_walk_check")
+
+
+def kernel_launches() -> int:
+    """Cumulative number of kernels the library enqueued from this thread
+    (gs_kernel_launches); the difference around a call = its launches."""
+    return int(load_library().gs_kernel_launches())
+
+
+def set_profiling(on: bool) -> None:
+    """gs_set_profiling: per-kernel event timing of the node-wise sampler."""
+    _check(load_library().gs_set_profiling(int(bool(on))), "gs_set_profiling")
+
+
+def blocks_profile(b: "Blocks") -> list:
+    """[(kernel, ms)] of the call that produced b (profiling on), gs_blocks_profile."""
+    L = load_library()
+    res, i = [], 0
+    name, ms = ctypes.c_char_p(), ctypes.c_double()
+    while b._h and L.gs_blocks_profile(b._h, i, ctypes.byref(name), ctypes.byref(ms)) == 0:
+        res.append((name.value.decode(), ms.value))
+        i += 1
+    return res
