@@ -7,9 +7,12 @@
 // P:300) and line 10's individual_sample(k, att) is the weighted A-Res sampler
 // over att (gs_graph_set_weights + gs_sample_neighbors(GS_W_EDGE)).
 //
-//   1. projections P = X [W1 | W2] : [N, F] x [F, 2H] bf16 -> fp32, one plain
-//      dense GEMM on the tensor cores (cuBLAS, bf16 inputs, fp32 accumulate);
-//      the grid-valued inputs of R29 make every partial sum exact.
+//   1. projections P = X [W1 | W2] : [N, F] x [F, 2H] bf16 -> fp32, one dense
+//      GEMM on the 5th-generation tensor cores: the hand-written TMA +
+//      tcgen05.mma + TMEM kernel of proj_gemm.cuh (F % 16 == 0; cuBLAS for
+//      other F, or with GS_PASS_GEMM=cublas); fp32 accumulation, so general
+//      inputs agree with the fp64 oracle within the magnitude-scaled bound of
+//      DESIGN.md R29 and the grid-valued inputs bit for bit.
 //   2. SDDMM + mix: a warp per column v keeps P_v (2H floats) in shared memory;
 //      8 lanes per in-edge gather P_u as 16-byte vectors (one random 2H*4-byte
 //      row per edge), form both dot products in fp64 (exact, any order), A3
@@ -25,6 +28,9 @@
 
 #include "common.cuh"
 #include "gs_internal.h"
+#include "proj_gemm.cuh"
+#include <cudaTypedefs.h>
+#include <cstdlib>
 
 namespace gsb {
 
@@ -121,6 +127,74 @@ static cublasHandle_t pa_handle() {
 
 static std::mutex pa_mutex;  // the shared handle's stream binding
 
+// WT[n][f] = [W1 | W2][f][n]: the B operand K-major (f contiguous)
+__global__ void pg_pack_wt_kernel(const __nv_bfloat16* __restrict__ W1, const __nv_bfloat16* __restrict__ W2,
+                                  int F, int H, __nv_bfloat16* __restrict__ WT) {
+  const int n2 = 2 * H;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n2 * F; i += gridDim.x * blockDim.x) {
+    const int n = i / F, f = i - n * F;
+    WT[i] = n < H ? W1[(size_t)f * H + n] : W2[(size_t)f * H + (n - H)];
+  }
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 pg_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+  });
+  return fn;
+}
+
+// P[N][2H] = X[N][F] [W1 | W2] on the tensor cores (proj_gemm.cuh).
+static gs_status pg_project(const void* X, int64_t N, int F, const void* W1, const void* W2, int H, float* P,
+                            const Allocator& al, cudaStream_t s) {
+  const int N2 = 2 * H;
+  PFN_cuTensorMapEncodeTiled_v12000 enc = pg_encode();
+  if (!enc) return fail(GS_ERR_CUDA, "gs_pass_attention: cuTensorMapEncodeTiled unavailable");
+  DevBuf wt;
+  if (!wt.ensure(al, (size_t)N2 * F * 2, s)) return fail(GS_ERR_OUT_OF_MEMORY, "gs_pass_attention: WT");
+  pg_pack_wt_kernel<<<(N2 * F + 255) / 256, 256, 0, s>>>((const __nv_bfloat16*)W1, (const __nv_bfloat16*)W2, F, H,
+                                                         (__nv_bfloat16*)wt.ptr);
+  count_launch();
+  CUtensorMap map;
+  const cuuint64_t gdim[2] = {(cuuint64_t)F, (cuuint64_t)N};
+  const cuuint64_t gstride[1] = {(cuuint64_t)F * 2};
+  const cuuint32_t box[2] = {8, (cuuint32_t)PG_BM};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(X), gdim, gstride, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    wt.reset(al, s);
+    return fail(GS_ERR_CUDA, "gs_pass_attention: cuTensorMapEncodeTiled failed (%d)", (int)r);
+  }
+  const size_t a_bytes = (size_t)PG_BM * F * 2, b_bytes = (size_t)N2 * F * 2;
+  const size_t cap = 200 * 1024;
+  int stages = (int)std::min<size_t>(6, (cap - b_bytes) / a_bytes);
+  stages = std::max(stages, 2);
+  const size_t smem = stages * a_bytes + b_bytes + (size_t)(2 * stages + 4) * 8 + 16;
+  gs_status st = GS_OK;
+  cudaError_t e = cudaFuncSetAttribute(proj_gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t tiles = (N + PG_BM - 1) / PG_BM;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(tiles, sms));
+    proj_gemm_kernel<<<grid, PG_THREADS, smem, s>>>(map, (const __nv_bfloat16*)wt.ptr, P, N, F, N2, stages);
+    count_launch();
+    e = cudaGetLastError();
+  }
+  if (e != cudaSuccess) st = cuda_fail(e, "proj_gemm_kernel launch");
+  wt.reset(al, s);
+  return st;
+}
+
 }  // namespace gsb
 
 using namespace gsb;
@@ -152,7 +226,10 @@ extern "C" gs_status gs_pass_attention(const gs_graph* g, const void* X, int F, 
     ce = cudaMemcpy2DAsync((char*)wc.ptr + H * 2, H2 * 2, W2, (size_t)H * 2, (size_t)H * 2, F,
                            cudaMemcpyDeviceToDevice, s);
   if (ce != cudaSuccess) st = cuda_fail(ce, "gs_pass_attention: weight copy");
-  if (st == GS_OK) {
+  const char* ge = getenv("GS_PASS_GEMM");
+  const bool tc = F % 16 == 0 && F <= 256 && !(ge && ge[0] == 'c');
+  if (st == GS_OK && tc) st = pg_project(X, N, F, W1, W2, H, (float*)P.ptr, al, s);
+  if (st == GS_OK && !tc) {
     // row-major P[N, 2H] = X[N, F] Wc[F, 2H]  <=>  column-major P^T = Wc^T X^T
     cublasHandle_t h = pa_handle();
     if (!h) {

@@ -4,5 +4,5 @@ Holds none of the sampling method's arithmetic: only R-MAT graph generation,
 edge-weight data, seed permutations and grid-valued dense matrices (PASS
 features / projections) (DESIGN.md "Input recipe").
 """
-from .graphs import (CONFIGS, GraphSpec, degree_stats, make_graph, make_grid_matrix,  # noqa: F401
+from .graphs import (CONFIGS, GraphSpec, degree_stats, make_graph, make_grid_matrix, make_feature_matrix,  # noqa: F401
                      make_seeds, small_graph)

@@ -283,3 +283,15 @@ def make_grid_matrix(stream: int, rows: int, cols: int, levels: int = 4, device=
     idx = torch.arange(rows * cols, device=device, dtype=torch.int64)
     q = (hash_u32(stream, idx) % (2 * levels + 1)) - levels
     return (q.to(torch.float32) / levels).to(torch.bfloat16).reshape(rows, cols)
+
+
+def make_feature_matrix(stream: int, rows: int, cols: int, device="cpu") -> torch.Tensor:
+    """Seeded synthetic dense matrix with GENERAL bf16 values (no grid): roughly
+    standard normal (sum of 4 uniforms, centred and scaled), rounded to bf16.
+    The PASS projections of such inputs depend on the summation order in fp32,
+    so GPU and oracle agree within the magnitude-scaled bound of DESIGN.md R29."""
+    idx = torch.arange(rows * cols, device=device, dtype=torch.int64)
+    acc = torch.zeros(rows * cols, device=device, dtype=torch.float32)
+    for j in range(4):
+        acc += (hash_u32(stream * 4 + j, idx).to(torch.float32) + 0.5) * (1.0 / 4294967296.0)
+    return ((acc - 2.0) * 1.7320508).to(torch.bfloat16).reshape(rows, cols)
