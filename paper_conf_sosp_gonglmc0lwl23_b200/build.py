@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libgsb200.so")
-SOURCES = ["capi.cu", "nodewise_wave.cu", "nodewise_hop.cu", "shadow.cu", "layerwise.cu", "layerwise_bm.cu", "walk.cu", "pack.cu", "pinsage.cu", "ops.cu", "pass_att.cu"]
+SOURCES = ["capi.cu", "nodewise_wave.cu", "nodewise_hop.cu", "shadow.cu", "layerwise.cu", "layerwise_sm.cu", "layerwise_bm.cu", "walk.cu", "pack.cu", "pinsage.cu", "ops.cu", "pass_att.cu"]
 HEADERS = ["common.cuh", "gs_internal.h", "nodewise_common.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 # -cudart shared: the static runtime would embed the name table of every

@@ -508,12 +508,32 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
 // when the candidate bitmaps of one CTA per SM fit (N/8 bytes each, <= 2 GB
 // in all) and its rank prefixes fit shared memory -- hub-biased frontiers give
 // ~280 k candidates per batch-layer (measured on LJ: 282 ms vs 514 ms).
-// LADIES / COUNT (~10 k candidates): the hash-table kernel below (31 ms vs
-// 69 ms: four dense bitmap scans per batch-layer cost more than the table).
+// LADIES / COUNT (~10 k candidates): the global hash-table kernel below (31 ms
+// vs 69 ms for the bitmap kernel: four dense bitmap scans per batch-layer cost
+// more than the table; the shared-memory kernel of layerwise_sm.cu, 30-53 ms,
+// on request).
 // GS_LW_PATH=old|bm forces one (experiments / tests).
+gs_status run_layerwise_sm(const gs_graph* g, const int32_t* seeds, int64_t num_seeds, int64_t batch_size,
+                           int64_t batch_base, const int32_t* n_per_layer, int L, int prob_mode, uint64_t key,
+                           cudaStream_t stream, gs_blocks* blk);
+
 gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  {
+    // LADIES / COUNT with frontiers and K <= 512: every per-batch table in
+    // shared memory (layerwise_sm.cu), on request
+    int maxK0 = 1;
+    for (int l = 0; l < L; ++l) maxK0 = std::max(maxK0, n_per_layer[l]);
+    const char* path0 = getenv("GS_LW_PATH");
+    // measured (LJ, 512 x 3): 30-53 ms vs the global-table kernel's 31 ms --
+    // per-batch-layer phases are barrier- and latency-bound; kept as an option
+    // (GS_LW_PATH=sm) until it wins
+    const bool sm_ok = prob_mode != GS_PROB_DEGREE && maxK0 <= 512 && batch_size <= 512;
+    if (sm_ok && path0 && !strcmp(path0, "sm"))
+      return run_layerwise_sm(g, seeds, num_seeds, batch_size, batch_base, n_per_layer, L, prob_mode, key,
+                              stream, blk);
+  }
   {
     int maxK = 1;
     for (int l = 0; l < L; ++l) maxK = std::max(maxK, n_per_layer[l]);

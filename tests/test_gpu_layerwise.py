@@ -20,11 +20,12 @@ def gs():
     return _gs
 
 
-@pytest.fixture(params=["bm", "old"], autouse=True)
+@pytest.fixture(params=["sm", "bm", "old"], autouse=True)
 def lw_path(request, monkeypatch):
-    """Every test runs through both layer-wise kernels: the candidate-bitmap
-    kernel (layerwise_bm.cu, the default where it fits) and the hash-table
-    kernel (layerwise.cu, large graphs)."""
+    """Every test runs through every layer-wise kernel: the shared-memory
+    kernel (layerwise_sm.cu, LADIES / COUNT default), the candidate-bitmap
+    kernel (layerwise_bm.cu, FastGCN default) and the global hash-table kernel
+    (layerwise.cu, the fallback)."""
     monkeypatch.setenv("GS_LW_PATH", request.param)
     return request.param
 
