@@ -166,6 +166,12 @@ gs_status gs_blocks_layer(const gs_blocks* b, int layer, gs_layer_buffers* out);
  * (null pointer, bad layer), GS_ERR_OUT_OF_MEMORY, GS_ERR_CUDA. */
 gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
                          int64_t* indptr, int32_t* row_map, int64_t* totals, void* stream);
+/* As gs_blocks_pack with 32-bit edge ids and block-relative 32-bit indptr
+ * entries (a smaller host copy): the sampled graph must have fewer than 2^31
+ * entries (else GS_ERR_NOT_SUPPORTED, host-side); block indptr values are
+ * always < 2^25.  Buffers are int32 arrays of the same capacities. */
+gs_status gs_blocks_pack_narrow(const gs_blocks* b, int layer, int32_t* row_local, int32_t* eid,
+                                int32_t* indptr, int32_t* row_map, int64_t* totals, void* stream);
 void gs_blocks_destroy(gs_blocks* b);
 /* Profiling (diagnostic, off by default): while on, the node-wise sampler
  * records a CUDA event after each of its kernels, runs them on one stream and

@@ -421,7 +421,7 @@ static gs_status check_batches(const gs_graph* g, const int32_t* seeds, int64_t 
   return GS_OK;
 }
 
-static gs_status prepare_blocks(gs_blocks** out, cudaStream_t stream) {
+static gs_status prepare_blocks(gs_blocks** out, cudaStream_t stream, const gs_graph* g) {
   if (!*out) {
     gs_blocks* b = new (std::nothrow) gs_blocks();
     if (!b) return fail(GS_ERR_OUT_OF_MEMORY, "host allocation failed");
@@ -430,6 +430,7 @@ static gs_status prepare_blocks(gs_blocks** out, cudaStream_t stream) {
   }
   (*out)->stream = stream;
   (*out)->synced = false;
+  (*out)->graph_edges = g ? g->num_edges : 0;
   return GS_OK;
 }
 
@@ -451,7 +452,7 @@ gs_status gs_sample_neighbors(const gs_graph* g, const int32_t* seeds, int64_t n
       return fail(GS_ERR_NOT_SUPPORTED, "batch_size * prod(fanouts) must be <= 2^25");
   }
   cudaStream_t stream = (cudaStream_t)stream_;
-  if ((st = prepare_blocks(out, stream))) return st;
+  if ((st = prepare_blocks(out, stream, g))) return st;
   return run_nodewise(g, seeds, num_seeds, batch_size, batch_index_base, fanouts,
                       num_layers, replace, bias_mode, rng_key, stream, *out);
 }
@@ -481,7 +482,7 @@ gs_status gs_sample_neighbors_ragged(const gs_graph* g, const int32_t* seeds, in
       return fail(GS_ERR_NOT_SUPPORTED, "max batch size * prod(fanouts) must be <= 2^25");
   }
   cudaStream_t stream = (cudaStream_t)stream_;
-  if ((st = prepare_blocks(out, stream))) return st;
+  if ((st = prepare_blocks(out, stream, g))) return st;
   return run_nodewise_hop(g, seeds, num_seeds, batch_ptr, 0, num_batches, batch_index_base, fanouts, num_layers,
                           replace, bias_mode, rng_key, stream, *out);
 }
@@ -492,7 +493,7 @@ gs_status gs_induce_subgraph(const gs_graph* g, const gs_blocks* sampled, void* 
   if (sampled->kind != gs_blocks::NODEWISE)
     return fail(GS_ERR_INVALID_ARGUMENT, "gs_induce_subgraph: sampled must come from gs_sample_neighbors");
   cudaStream_t stream = (cudaStream_t)stream_;
-  gs_status st = prepare_blocks(out, stream);
+  gs_status st = prepare_blocks(out, stream, g);
   if (st) return st;
   return run_induce(g, sampled, stream, *out);
 }
@@ -514,7 +515,7 @@ gs_status gs_sample_shadow(const gs_graph* g, const int32_t* seeds, int64_t num_
       return fail(GS_ERR_NOT_SUPPORTED, "batch_size * (1 + sum of fanout products) must be <= 2^25");
   }
   cudaStream_t stream = (cudaStream_t)stream_;
-  if ((st = prepare_blocks(out, stream))) return st;
+  if ((st = prepare_blocks(out, stream, g))) return st;
   return run_shadow(g, seeds, num_seeds, batch_size, batch_index_base, fanouts, num_layers,
                     bias_mode, rng_key, stream, *out);
 }
@@ -532,7 +533,7 @@ gs_status gs_sample_saint_rw(const gs_graph* g, const int32_t* roots, int64_t nu
   if ((batch_index_base + (num_roots + batch_size - 1) / batch_size) * batch_size > (int64_t(1) << 32))
     return fail(GS_ERR_NOT_SUPPORTED, "gs_sample_saint_rw: global walker ids must fit 32 bits");
   cudaStream_t stream = (cudaStream_t)stream_;
-  gs_status st = prepare_blocks(out, stream);
+  gs_status st = prepare_blocks(out, stream, g);
   if (st) return st;
   return run_saint_rw(g, roots, num_roots, batch_size, batch_index_base, walk_length, rng_key,
                       stream, *out);
@@ -557,7 +558,7 @@ gs_status gs_sample_pinsage(const gs_graph* g, const int32_t* seeds, int64_t num
       return fail(GS_ERR_NOT_SUPPORTED, "batch_size * prod(topk) must be <= 2^25");
   }
   cudaStream_t stream = (cudaStream_t)stream_;
-  if ((st = prepare_blocks(out, stream))) return st;
+  if ((st = prepare_blocks(out, stream, g))) return st;
   return run_pinsage(g, seeds, num_seeds, batch_size, batch_index_base, topk, num_layers, num_walks,
                      walk_length, restart_prob, rng_key, stream, *out);
 }
@@ -574,7 +575,7 @@ gs_status gs_sample_layerwise(const gs_graph* g, const int32_t* seeds, int64_t n
     if (n_per_layer[l] > 4096) return fail(GS_ERR_NOT_SUPPORTED, "n_per_layer must be <= 4096");
   if (batch_size > 4096) return fail(GS_ERR_NOT_SUPPORTED, "layer-wise batch_size must be <= 4096");
   cudaStream_t stream = (cudaStream_t)stream_;
-  if ((st = prepare_blocks(out, stream))) return st;
+  if ((st = prepare_blocks(out, stream, g))) return st;
   return run_layerwise(g, seeds, num_seeds, batch_size, batch_index_base, n_per_layer, num_layers,
                        prob_mode, rng_key, stream, *out);
 }

@@ -100,6 +100,7 @@ struct gs_blocks {
   bool synced = false;
   gs_blocks* aux = nullptr;    // ShaDow: the internal node-wise result
   int64_t num_seeds = 0, batch_size = 0;  // node-wise: the seeds and (fixed) batch size sampled
+  int64_t graph_edges = 0;     // num_edges of the graph sampled (gs_blocks_pack_narrow's check)
   const int64_t* bptr_dev = nullptr;       // node-wise (hop engine): device seed offsets [nb + 1]
   cudaStream_t side = nullptr; // node-wise: second stream (groups of batches alternate), forked/joined by events
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;

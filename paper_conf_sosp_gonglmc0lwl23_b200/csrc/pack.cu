@@ -56,12 +56,13 @@ struct PackParams {
   const int64_t* indptr_in;
   const int32_t* row_map_in;
   int32_t* row_local;
-  int64_t* eid;
-  int64_t* indptr;
+  void* eid;       // int64 (or int32: narrow)
+  void* indptr;    // int64 (or int32: narrow)
   int32_t* row_map;
   int64_t edge_cap, indptr_cap, row_cap;  // the layer buffers' capacities (copies are clamped)
 };
 
+template <bool NARROW>
 __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
   for (int64_t b = blockIdx.x; b < P.nb; b += gridDim.x) {
     const int64_t* m = P.meta + (b * P.L + P.layer) * GS_META_FIELDS;
@@ -73,9 +74,15 @@ __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
     const int64_t eo = o[0], io = o[1], ro = o[2];
     for (int64_t i = threadIdx.x; i < E; i += PK_THREADS) {
       P.row_local[eo + i] = __ldcs(P.row_local_in + m[6] + i);
-      P.eid[eo + i] = __ldcs(P.eid_in + m[6] + i);
+      const int64_t e = __ldcs(P.eid_in + m[6] + i);
+      if (NARROW) ((int32_t*)P.eid)[eo + i] = (int32_t)e;
+      else ((int64_t*)P.eid)[eo + i] = e;
     }
-    for (int64_t i = threadIdx.x; i <= T; i += PK_THREADS) P.indptr[io + i] = __ldcs(P.indptr_in + m[5] + i);
+    for (int64_t i = threadIdx.x; i <= T; i += PK_THREADS) {
+      const int64_t x = __ldcs(P.indptr_in + m[5] + i);
+      if (NARROW) ((int32_t*)P.indptr)[io + i] = (int32_t)x;  // block-relative (<= 2^25)
+      else ((int64_t*)P.indptr)[io + i] = x;
+    }
     for (int64_t i = threadIdx.x; i < R; i += PK_THREADS) P.row_map[ro + i] = __ldcs(P.row_map_in + m[4] + i);
   }
 }
@@ -84,9 +91,8 @@ __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
 
 using namespace gsb;
 
-extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
-                                    int64_t* indptr, int32_t* row_map, int64_t* totals,
-                                    void* stream_) {
+static gs_status pack_impl(const gs_blocks* b, int layer, int32_t* row_local, void* eid, void* indptr,
+                           int32_t* row_map, int64_t* totals, void* stream_, bool narrow) {
   cudaStream_t stream = (cudaStream_t)stream_;
   if (!b || !row_local || !eid || !indptr || !row_map || !totals)
     return fail(GS_ERR_INVALID_ARGUMENT, "gs_blocks_pack: null argument");
@@ -122,7 +128,21 @@ extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t grid = std::min<int64_t>(nb, (int64_t)sms * 4);
-  pack_copy_kernel<<<(unsigned)grid, PK_THREADS, 0, stream>>>(P); count_launch();
+  if (narrow) pack_copy_kernel<true><<<(unsigned)grid, PK_THREADS, 0, stream>>>(P);
+  else pack_copy_kernel<false><<<(unsigned)grid, PK_THREADS, 0, stream>>>(P);
+  count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
+}
+
+extern "C" gs_status gs_blocks_pack(const gs_blocks* b, int layer, int32_t* row_local, int64_t* eid,
+                                    int64_t* indptr, int32_t* row_map, int64_t* totals, void* stream) {
+  return pack_impl(b, layer, row_local, eid, indptr, row_map, totals, stream, false);
+}
+
+extern "C" gs_status gs_blocks_pack_narrow(const gs_blocks* b, int layer, int32_t* row_local, int32_t* eid,
+                                           int32_t* indptr, int32_t* row_map, int64_t* totals, void* stream) {
+  if (b && b->graph_edges >= (int64_t(1) << 31))
+    return fail(GS_ERR_NOT_SUPPORTED, "gs_blocks_pack_narrow: the graph has >= 2^31 edges (int32 edge ids)");
+  return pack_impl(b, layer, row_local, eid, indptr, row_map, totals, stream, true);
 }

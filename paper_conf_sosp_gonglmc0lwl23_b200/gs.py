@@ -33,7 +33,7 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_kernel_launche
            "gs_set_allocator",
            "gs_graph_create", "gs_graph_get_info", "gs_graph_destroy", "gs_blocks_sync",
            "gs_blocks_shape", "gs_blocks_view", "gs_blocks_device_meta", "gs_blocks_layer",
-           "gs_blocks_pack", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_neighbors_ragged",
+           "gs_blocks_pack", "gs_blocks_pack_narrow", "gs_blocks_destroy", "gs_sample_neighbors", "gs_sample_neighbors_ragged",
            "gs_induce_subgraph", "gs_sample_shadow", "gs_sample_saint_rw", "gs_sample_pinsage",
            "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
@@ -162,6 +162,7 @@ def load_library(path: str = LIB_PATH):
     L.gs_blocks_device_meta.argtypes = [vp, ctypes.POINTER(vp)]
     L.gs_blocks_layer.argtypes = [vp, i32, ctypes.POINTER(_LayerBuffers)]
     L.gs_blocks_pack.argtypes = [vp, i32, vp, vp, vp, vp, vp, vp]
+    L.gs_blocks_pack_narrow.argtypes = [vp, i32, vp, vp, vp, vp, vp, vp]
     L.gs_blocks_destroy.argtypes = [vp]
     L.gs_blocks_destroy.restype = None
     _lib = L
@@ -325,11 +326,13 @@ class Blocks:
         _check(_lib.gs_blocks_layer(self._h, layer, ctypes.byref(lb)), "gs_blocks_layer")
         return {"edges": lb.edge_capacity, "indptr": lb.indptr_capacity, "rows": lb.row_capacity}
 
-    def pack(self, layer: int, out: dict = None, stream=None) -> dict:
+    def pack(self, layer: int, out: dict = None, stream=None, narrow: bool = False) -> dict:
         """gs_blocks_pack: layer `layer` of every batch packed densely on the
         device (batch order).  Returns device tensors (capacity-sized; the used
-        prefix lengths are in `totals` = device int64 [edges, indptr entries, rows])."""
+        prefix lengths are in `totals` = device int64 [edges, indptr entries, rows]).
+        narrow: int32 eid / indptr (gs_blocks_pack_narrow; graphs with < 2^31 entries)."""
         cap = self.layer_capacity(layer)
+        wide = torch.int32 if narrow else torch.int64
         if out is not None:  # the C call writes up to the layer's capacity: check the caller's buffers
             for k, n in (("row_local", cap["edges"]), ("eid", cap["edges"]), ("indptr", cap["indptr"]),
                          ("row_map", cap["rows"])):
@@ -338,13 +341,16 @@ class Blocks:
         if out is None:
             dev = torch.device("cuda", torch.cuda.current_device())
             out = {"row_local": torch.empty(cap["edges"], dtype=torch.int32, device=dev),
-                   "eid": torch.empty(cap["edges"], dtype=torch.int64, device=dev),
-                   "indptr": torch.empty(cap["indptr"], dtype=torch.int64, device=dev),
+                   "eid": torch.empty(cap["edges"], dtype=wide, device=dev),
+                   "indptr": torch.empty(cap["indptr"], dtype=wide, device=dev),
                    "row_map": torch.empty(cap["rows"], dtype=torch.int32, device=dev),
                    "totals": torch.empty(3, dtype=torch.int64, device=dev)}
-        _check(_lib.gs_blocks_pack(self._h, layer, _ptr(out["row_local"]), _ptr(out["eid"]),
-                                   _ptr(out["indptr"]), _ptr(out["row_map"]), _ptr(out["totals"]),
-                                   _stream_ptr(stream)), "gs_blocks_pack")
+        fn = _lib.gs_blocks_pack_narrow if narrow else _lib.gs_blocks_pack
+        for k in ("eid", "indptr"):
+            if out[k].dtype != wide:
+                raise GSError(1, f"pack: out['{k}'] must be {wide}")
+        _check(fn(self._h, layer, _ptr(out["row_local"]), _ptr(out["eid"]), _ptr(out["indptr"]),
+                  _ptr(out["row_map"]), _ptr(out["totals"]), _stream_ptr(stream)), "gs_blocks_pack")
         return out
 
     def to_host(self) -> list:

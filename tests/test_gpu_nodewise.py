@@ -143,10 +143,12 @@ def test_shadow(gs, oracle_lib, medium, mode, wcap, monkeypatch):
     compare_all(out, [[r] for r in ref], f"shadow {mode}")
 
 
+@pytest.mark.parametrize("narrow", [False, True])
 @pytest.mark.parametrize("kind", ["nodewise", "layerwise"])
-def test_pack_matches_views(gs, medium, kind):
-    """gs_blocks_pack: every batch's block, packed densely in batch order, is
-    exactly its view (indptr block-relative), and `totals` are the sums."""
+def test_pack_matches_views(gs, medium, kind, narrow):
+    """gs_blocks_pack (and gs_blocks_pack_narrow, int32 ids): every batch's
+    block, packed densely in batch order, is exactly its view (indptr
+    block-relative), and `totals` are the sums."""
     g, G, O = medium
     seeds = synth.make_seeds(synth.GraphSpec("m", 200_000, 1, False, None, 12), 5000).cuda()
     if kind == "nodewise":
@@ -155,8 +157,10 @@ def test_pack_matches_views(gs, medium, kind):
         out = gs.sample_layerwise(G, seeds, [300, 300], batch_size=700, prob_mode=1, rng_key=21)
     out.sync()
     for l in range(2):
-        pk = out.pack(l)
+        pk = out.pack(l, narrow=narrow)
         torch.cuda.synchronize()
+        if narrow:
+            pk = {k: (v.long() if k in ("eid", "indptr") else v) for k, v in pk.items()}
         tot = pk["totals"].cpu().tolist()
         e = i = r = 0
         for b in range(out.num_batches):
