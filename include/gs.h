@@ -331,6 +331,42 @@ gs_status gs_matrix_elementwise(gs_matrix* m, int op, float v, void* stream);
 /* A.row() (Finalize; R3): distinct row ids ascending into out (device
  * int32, capacity >= min(nnz, num_nodes)); *n_out (host) = their number. */
 gs_status gs_matrix_row_ids(const gs_matrix* m, int32_t* out, int64_t* n_out, void* stream);
+/* A.individual_sample(K, probs) (Select): every column
+ * (frontier) samples K of its entries independently; returns the sub-matrix
+ * of the kept entries (ascending position; slot order with replacement).
+ * use_values 0: uniform -- without replacement Floyd (R5, all of a column with
+ * <= K entries), replace 1: K i.i.d. draws (R10); use_values 1: weighted
+ * without replacement on the matrix's values (A-Res, R6; values <= 0
+ * ineligible).  RNG: the samplers' keying (R4) with the column node, the
+ * entry's position in the column, `layer` and `batch_index` -- on A[:, F] the
+ * result is exactly that layer of gs_sample_neighbors (Extract-Select fusion,
+ * P:289).  1 <= K <= 32.  Synchronises the stream once (output size). */
+gs_status gs_matrix_individual_sample(const gs_matrix* in, int K, int use_values, int replace, uint64_t rng_key,
+                                      int layer, int64_t batch_index, void* stream, gs_matrix** out);
+/* A.collective_sample(K, node_probs) (Select): K of the
+ * matrix's row nodes by the bias node_probs (device float[num_nodes], indexed
+ * by global id, unnormalised) or, node_probs NULL, the rows' entry counts;
+ * b <= 0 ineligible; every eligible row when at most K (R24), else the K
+ * smallest A-Res keys (R6, layer-wise keying R4; ties -> smaller id); returns
+ * the sub-matrix of the entries whose row was selected (CSC order; its
+ * gs_matrix_row_ids = S ascending).  With node_probs = (A[:,F] ** 2).sum(1)
+ * it is one layer of gs_sample_layerwise(LADIES).  K <= 2048.  Synchronises. */
+gs_status gs_matrix_collective_sample(const gs_matrix* in, int K, const float* node_probs, uint64_t rng_key,
+                                      int layer, int64_t batch_index, void* stream, gs_matrix** out);
+/* Fused Edge-Map chain (+ Edge-Reduce): the element-wise
+ * operators (ops[i], scalars[i]), i < n_ops <= 8, applied in order to every
+ * entry value -- identical to n_ops gs_matrix_elementwise calls -- in one
+ * pass; axis -1: written back in place (Edge-Map fusion); axis 0 / 1: not
+ * written, summed per column / per global row into out (float[n_cols] /
+ * float[num_nodes], fp64 accumulation, Edge-MapReduce fusion). */
+gs_status gs_matrix_map_reduce(gs_matrix* m, const int* ops, const float* scalars, int n_ops, int axis, float* out,
+                               void* stream);
+/* AS-GCN-style learned layer-wise bias (Table 2; R30): out[u] =
+ * fp32(s(u) * relu(fp32(sum_f X[u][f] wg[f]))) with s = A.sum(axis=1) (fp64
+ * accumulation), X device bf16 [num_nodes][F] row-major, wg device float[F]
+ * (the trainable projection); 0 for nodes that are not rows of m.  The
+ * node_probs of gs_matrix_collective_sample. */
+gs_status gs_matrix_asgcn_bias(const gs_matrix* m, const void* X, int F, const float* wg, float* out, void* stream);
 gs_status gs_matrix_get_view(const gs_matrix* m, gs_matrix_view* out);
 void      gs_matrix_destroy(gs_matrix* m);
 

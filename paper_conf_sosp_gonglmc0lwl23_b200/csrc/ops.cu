@@ -22,6 +22,8 @@
 
 #include "common.cuh"
 #include "gs_internal.h"
+#include "nodewise_common.cuh"
+#include <cuda_bf16.h>
 
 struct gs_matrix {
   gsb::Allocator al;
@@ -329,6 +331,257 @@ __global__ void emit_rows_kernel(const uint32_t* __restrict__ bm, int64_t nw, co
   }
 }
 
+
+// ---- Select operators (Table 4; oracle/ops.py individual_sample,
+// collective_sample) ----
+// A.individual_sample, count pass: kept entries per column (R5 / R6 / R10).
+__global__ void isamp_count_kernel(const int64_t* __restrict__ ip, const float* __restrict__ val, int64_t n,
+                                   int K, int use_values, int replace, int64_t* __restrict__ out_ip) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t j = warp; j < n; j += nwarps) {
+    const int64_t lo = ip[j], hi = ip[j + 1], d = hi - lo;
+    int64_t c;
+    if (replace) {
+      c = d > 0 ? K : 0;
+    } else if (use_values) {
+      int64_t pos = 0;
+      for (int64_t i = lo + lane; i < hi; i += 32) pos += val[i] > 0.0f ? 1 : 0;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) pos += __shfl_xor_sync(0xffffffffu, pos, o);
+      c = pos < K ? pos : K;
+    } else {
+      c = d < K ? d : K;
+    }
+    if (lane == 0) out_ip[j + 1] = c;
+    if (j == 0 && lane == 0) out_ip[0] = 0;
+  }
+}
+
+// A.individual_sample, select + copy: a thread per column (the general,
+// unfused operator; the fused samplers are the fast path).
+__global__ void isamp_select_kernel(const int32_t* __restrict__ cols, const int64_t* __restrict__ ip,
+                                    const int32_t* __restrict__ row, const int64_t* __restrict__ eid,
+                                    const float* __restrict__ val, int64_t n, int K, int use_values, int replace,
+                                    uint64_t key, int layer, uint32_t batch, const int64_t* __restrict__ out_ip,
+                                    int32_t* __restrict__ orow, int64_t* __restrict__ oeid, float* __restrict__ oval) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = (uint32_t)cols[j];
+    const int64_t lo = ip[j], d = ip[j + 1] - lo;
+    int64_t o = out_ip[j];
+    const int64_t cnt = out_ip[j + 1] - o;
+    uint32_t pos[MAX_FANOUT];
+    double kk[MAX_FANOUT];
+    int n_sel = 0;
+    if (replace) {
+      for (int s = 0; s < (int)cnt; ++s) {
+        const U4 r = philox(v, (uint32_t)s, ctr2(layer, TAG_REPLACE), batch, key);
+        pos[n_sel++] = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
+      }
+    } else if (!use_values) {
+      if (d <= K) {
+        for (int i = 0; i < (int)d; ++i) pos[n_sel++] = (uint32_t)i;
+      } else {  // Floyd (R5), the list kept sorted
+        for (int s = 0; s < K; ++s) {
+          const U4 r = philox(v, (uint32_t)s, ctr2(layer, TAG_FLOYD), batch, key);
+          const uint32_t m = (uint32_t)(d - K + s);
+          const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
+          bool dup = false;
+          for (int q = 0; q < n_sel; ++q) dup |= pos[q] == t;
+          const uint32_t x = dup ? m : t;
+          int q = n_sel;
+          while (q > 0 && pos[q - 1] > x) {
+            pos[q] = pos[q - 1];
+            --q;
+          }
+          pos[q] = x;
+          ++n_sel;
+        }
+      }
+    } else {  // A-Res (R6): the cnt smallest (key, position) among the positive values
+      for (int64_t i = 0; i < d && cnt > 0; ++i) {
+        const float w = val[lo + i];
+        if (!(w > 0.0f)) continue;
+        const U4 r = philox(v, (uint32_t)(i >> 2), ctr2(layer, TAG_ARES_NODE), batch, key);
+        const double k2 = ares_key(sel_word(r, (int)(i & 3)), (double)w);
+        if (n_sel == cnt && !(k2 < kk[n_sel - 1])) continue;
+        int q = n_sel < cnt ? n_sel : (int)cnt - 1;
+        while (q > 0 && kk[q - 1] > k2) {
+          kk[q] = kk[q - 1];
+          pos[q] = pos[q - 1];
+          --q;
+        }
+        kk[q] = k2;
+        pos[q] = (uint32_t)i;
+        if (n_sel < cnt) ++n_sel;
+      }
+      for (int a = 1; a < n_sel; ++a) {  // positions ascending
+        const uint32_t x = pos[a];
+        int q = a;
+        while (q > 0 && pos[q - 1] > x) {
+          pos[q] = pos[q - 1];
+          --q;
+        }
+        pos[q] = x;
+      }
+    }
+    for (int q = 0; q < n_sel; ++q) {
+      const int64_t i = lo + pos[q];
+      orow[o] = row[i];
+      oeid[o] = eid[i];
+      oval[o] = val[i];
+      ++o;
+    }
+  }
+}
+
+// A.collective_sample helpers: per-row entry counts (node_probs omitted)
+__global__ void row_count_dense_kernel(const int32_t* __restrict__ row, int64_t nnz, float* __restrict__ cnt) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + __ldcs(row + i), 1.0f);  // exact: integer counts < 2^24
+}
+
+// keys of the candidates C (ascending ids): eligible (b > 0) -> (key, u); B;
+// count of keys below tau and the ones below tau collected (<= cap)
+__global__ void csamp_keys_kernel(const int32_t* __restrict__ C, int64_t nc, const float* __restrict__ b,
+                                  uint64_t key, int layer, uint32_t batch, double* __restrict__ ckey,
+                                  double* __restrict__ bsum, unsigned long long* __restrict__ nelig) {
+  double s = 0.0;
+  unsigned long long e = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = (uint32_t)C[i];
+    const float bias = b[u];
+    double k2 = INFINITY;
+    if (bias > 0.0f) {
+      const U4 r = philox(u, 0u, ctr2(layer, TAG_ARES_LAYER), batch, key);
+      k2 = ares_key(r.x, (double)bias);
+      ++e;
+    }
+    s += (double)bias;
+    ckey[i] = k2;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    s += __shfl_xor_sync(0xffffffffu, s, o);
+    e += __shfl_xor_sync(0xffffffffu, e, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicAdd(bsum, s);
+    atomicAdd(nelig, e);
+  }
+}
+
+__global__ void csamp_collect_kernel(const int32_t* __restrict__ C, const double* __restrict__ ckey, int64_t nc,
+                                     double tau, int cap, double* __restrict__ bk, int32_t* __restrict__ bu,
+                                     unsigned int* __restrict__ nb) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += (int64_t)gridDim.x * blockDim.x) {
+    const double k2 = ckey[i];
+    if (!(k2 < tau)) continue;
+    const unsigned int slot = atomicAdd(nb, 1u);
+    if ((int)slot < cap) {
+      bk[slot] = k2;
+      bu[slot] = C[i];
+    }
+  }
+}
+
+// one CTA: the K smallest (key, u) of n buffered candidates -> their rows'
+// bits in the bitmap (the sub-matrix is then A restricted to them)
+constexpr int CS_CAP = 4096;
+__global__ void __launch_bounds__(1024) csamp_select_kernel(const double* __restrict__ bk, const int32_t* __restrict__ bu,
+                                                          int n, int K, uint32_t* __restrict__ bm) {
+  __shared__ double sk[CS_CAP];
+  __shared__ int32_t su[CS_CAP];
+  int n2 = 1;
+  while (n2 < n) n2 <<= 1;
+  for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+    sk[i] = i < n ? bk[i] : INFINITY;
+    su[i] = i < n ? bu[i] : 0x7FFFFFFF;
+  }
+  __syncthreads();
+  for (int k = 2; k <= n2; k <<= 1)
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+        const int o = i ^ j;
+        if (o > i) {
+          const bool gt = sk[i] > sk[o] || (sk[i] == sk[o] && su[i] > su[o]);
+          if (gt == ((i & k) == 0)) {
+            const double t = sk[i]; sk[i] = sk[o]; sk[o] = t;
+            const int32_t tu = su[i]; su[i] = su[o]; su[o] = tu;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  for (int i = threadIdx.x; i < K && i < n; i += blockDim.x) atomicOr(bm + (su[i] >> 5), 1u << (su[i] & 31));
+}
+
+// eligible rows (b > 0) of C into the bitmap (at most K of them: all are taken, R24)
+__global__ void csamp_all_kernel(const int32_t* __restrict__ C, int64_t nc, const float* __restrict__ b,
+                                 uint32_t* __restrict__ bm) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t u = C[i];
+    if (b[u] > 0.0f) atomicOr(bm + (u >> 5), 1u << (u & 31));
+  }
+}
+
+// ---- fused Edge-Map chain (+ Edge-Reduce), P:291-294 ----
+constexpr int MR_MAX_OPS = 8;
+struct MapChain {
+  int n;
+  int op[MR_MAX_OPS];
+  float x[MR_MAX_OPS];
+};
+__device__ __forceinline__ float chain_apply(const MapChain& c, float v) {
+  for (int i = 0; i < c.n; ++i) v = apply_op(c.op[i], v, c.x[i]);
+  return v;
+}
+__global__ void map_chain_kernel(float* val, int64_t nnz, MapChain c) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
+    val[i] = chain_apply(c, val[i]);
+}
+__global__ void __launch_bounds__(OPS_THREADS) map_col_sum_kernel(const int64_t* __restrict__ ip,
+                                                                 const float* __restrict__ val, int64_t n,
+                                                                 MapChain c, float* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t j = warp; j < n; j += nwarps) {
+    double s = 0.0;
+    for (int64_t i = ip[j] + lane; i < ip[j + 1]; i += 32) s += (double)chain_apply(c, __ldcs(val + i));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) out[j] = (float)s;
+  }
+}
+__global__ void map_row_sum_kernel(const int32_t* __restrict__ row, const float* __restrict__ val, int64_t nnz,
+                                   MapChain c, double* __restrict__ acc) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(acc + __ldcs(row + i), (double)chain_apply(c, __ldcs(val + i)));
+}
+
+// ---- AS-GCN-style bias (R30): b(u) = fp32(s(u) * relu(fp32(sum_fp64 X[u] wg))) ----
+__global__ void asgcn_bias_kernel(const double* __restrict__ s, const __nv_bfloat16* __restrict__ X, int F,
+                                  const float* __restrict__ wg, int64_t N, float* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < N; u += nwarps) {
+    const float su = (float)s[u];
+    if (su == 0.0f) {  // not a row of the matrix (or a zero sum): b = 0
+      if (lane == 0) out[u] = 0.0f;
+      continue;
+    }
+    double dot = 0.0;
+    for (int f = lane; f < F; f += 32) dot += (double)__bfloat162float(X[u * F + f]) * (double)wg[f];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, o);
+    if (lane == 0) {
+      const float g = (float)dot;
+      out[u] = __fmul_rn(su, g > 0.0f ? g : 0.0f);
+    }
+  }
+}
 }  // namespace gsb
 
 using namespace gsb;
@@ -531,6 +784,216 @@ gs_status gs_matrix_row_ids(const gs_matrix* m, int32_t* out, int64_t* n_out, vo
   bm.reset(m->al, s);
   cnt.reset(m->al, s);
   return st;
+}
+
+
+gs_status gs_matrix_individual_sample(const gs_matrix* in, int K, int use_values, int replace, uint64_t rng_key,
+                                      int layer, int64_t batch_index, void* stream_, gs_matrix** out) {
+  if (!in || !out || *out == in || K < 1 || K > MAX_FANOUT || (replace && use_values) || layer < 0 ||
+      layer >= (1 << 24) || batch_index < 0)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_individual_sample: bad argument (1 <= K <= %d, no weighted "
+                "replacement, out != in)", MAX_FANOUT);
+  cudaStream_t s = (cudaStream_t)stream_;
+  gs_status st = new_matrix(out, in->num_nodes);
+  if (st) return st;
+  gs_matrix* m = *out;
+  const int64_t n = in->n_cols;
+  if (!m->b_indptr.ensure(m->al, (size_t)(n + 1) * 8, s))
+    return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (individual_sample)");
+  int64_t* ip = (int64_t*)m->b_indptr.ptr;
+  GS_CUDA_TRY(cudaMemsetAsync(ip, 0, 8, s));
+  if (n > 0) {
+    isamp_count_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>((const int64_t*)in->b_indptr.ptr,
+                                                           (const float*)in->b_val.ptr, n, K, use_values, replace, ip);
+    count_launch();
+    GS_CUDA_TRY(cudaGetLastError());
+    if ((st = scan_inclusive(ip + 1, n, m->al, s))) return st;
+  }
+  int64_t nnz = 0;
+  GS_CUDA_TRY(cudaMemcpyAsync(&nnz, ip + n, 8, cudaMemcpyDeviceToHost, s));
+  GS_CUDA_TRY(cudaStreamSynchronize(s));
+  if ((st = alloc_entries(m, n, nnz, s))) return st;
+  if (n > 0) {
+    GS_CUDA_TRY(cudaMemcpyAsync(m->b_cols.ptr, in->b_cols.ptr, n * 4, cudaMemcpyDeviceToDevice, s));
+    isamp_select_kernel<<<grid_for(n, 128), 128, 0, s>>>(
+        (const int32_t*)in->b_cols.ptr, (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr,
+        (const int64_t*)in->b_eid.ptr, (const float*)in->b_val.ptr, n, K, use_values, replace, rng_key, layer,
+        (uint32_t)batch_index, ip, (int32_t*)m->b_row.ptr, (int64_t*)m->b_eid.ptr, (float*)m->b_val.ptr);
+    count_launch();
+    GS_CUDA_TRY(cudaGetLastError());
+  }
+  return GS_OK;
+}
+
+gs_status gs_matrix_collective_sample(const gs_matrix* in, int K, const float* node_probs, uint64_t rng_key,
+                                      int layer, int64_t batch_index, void* stream_, gs_matrix** out) {
+  if (!in || !out || *out == in || K < 1 || layer < 0 || layer >= (1 << 24) || batch_index < 0)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_collective_sample: bad argument (K >= 1, out != in)");
+  cudaStream_t s = (cudaStream_t)stream_;
+  const int64_t N = in->num_nodes, nw = (N + 31) / 32;
+  const Allocator al = in->al;
+  // C = row(): the distinct rows ascending
+  DevBuf cbuf, bias, keys, sel, bbuf, misc;
+  if (!cbuf.ensure(al, (size_t)std::max<int64_t>(std::min(in->nnz, N), 1) * 4, s) ||
+      !misc.ensure(al, 64, s) || !sel.ensure(al, (size_t)std::max<int64_t>(nw, 1) * 4, s))
+    return fail(GS_ERR_OUT_OF_MEMORY, "collective_sample workspace");
+  auto cleanup = [&](gs_status st) {
+    cbuf.reset(al, s); bias.reset(al, s); keys.reset(al, s); sel.reset(al, s); bbuf.reset(al, s); misc.reset(al, s);
+    return st;
+  };
+  int64_t nc = 0;
+  gs_status st = gs_matrix_row_ids(in, (int32_t*)cbuf.ptr, &nc, stream_);
+  if (st) return cleanup(st);
+  const float* b = node_probs;
+  if (!b) {  // "the sampling bias on each edge is 1 and automatically aggregates"
+    if (!bias.ensure(al, (size_t)std::max<int64_t>(N, 1) * 4, s)) return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "bias"));
+    GS_CUDA_TRY(cudaMemsetAsync(bias.ptr, 0, (size_t)std::max<int64_t>(N, 1) * 4, s));
+    if (in->nnz > 0) {
+      row_count_dense_kernel<<<grid_for(in->nnz, 256), 256, 0, s>>>((const int32_t*)in->b_row.ptr, in->nnz,
+                                                                    (float*)bias.ptr);
+      count_launch();
+    }
+    b = (const float*)bias.ptr;
+  }
+  GS_CUDA_TRY(cudaMemsetAsync(sel.ptr, 0, (size_t)std::max<int64_t>(nw, 1) * 4, s));
+  GS_CUDA_TRY(cudaMemsetAsync(misc.ptr, 0, 64, s));
+  double* bsum = (double*)misc.ptr;
+  unsigned long long* nelig = (unsigned long long*)((char*)misc.ptr + 8);
+  unsigned int* nbuf = (unsigned int*)((char*)misc.ptr + 16);
+  if (nc > 0) {
+    if (!keys.ensure(al, (size_t)nc * 8, s)) return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "keys"));
+    csamp_keys_kernel<<<grid_for(nc, 256), 256, 0, s>>>((const int32_t*)cbuf.ptr, nc, b, rng_key, layer,
+                                                        (uint32_t)batch_index, (double*)keys.ptr, bsum, nelig);
+    count_launch();
+    double hb = 0.0;
+    unsigned long long he = 0;
+    GS_CUDA_TRY(cudaMemcpyAsync(&hb, bsum, 8, cudaMemcpyDeviceToHost, s));
+    GS_CUDA_TRY(cudaMemcpyAsync(&he, nelig, 8, cudaMemcpyDeviceToHost, s));
+    GS_CUDA_TRY(cudaStreamSynchronize(s));
+    if ((int64_t)he <= K) {  // every eligible row (R24)
+      csamp_all_kernel<<<grid_for(nc, 256), 256, 0, s>>>((const int32_t*)cbuf.ptr, nc, b, (uint32_t*)sel.ptr);
+      count_launch();
+    } else {
+      // threshold: keys below tau (expected ~2K of them), widened / narrowed
+      // until K <= count <= CS_CAP, then the K smallest in one CTA
+      if (K > CS_CAP / 2) return cleanup(fail(GS_ERR_NOT_SUPPORTED, "collective_sample: K <= %d", CS_CAP / 2));
+      if (!bbuf.ensure(al, (size_t)CS_CAP * 12, s)) return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "buffer"));
+      double tau = hb > 0.0 ? 2.0 * K / hb : 1.0, lo = 0.0, hi = 0.0;
+      unsigned int cnt = 0;
+      for (int att = 0; att < 200; ++att) {
+        GS_CUDA_TRY(cudaMemsetAsync(nbuf, 0, 4, s));
+        csamp_collect_kernel<<<grid_for(nc, 256), 256, 0, s>>>((const int32_t*)cbuf.ptr, (const double*)keys.ptr,
+                                                               nc, tau, CS_CAP, (double*)bbuf.ptr,
+                                                               (int32_t*)((char*)bbuf.ptr + CS_CAP * 8), nbuf);
+        count_launch();
+        GS_CUDA_TRY(cudaMemcpyAsync(&cnt, nbuf, 4, cudaMemcpyDeviceToHost, s));
+        GS_CUDA_TRY(cudaStreamSynchronize(s));
+        if ((int)cnt >= K && (int)cnt <= CS_CAP) break;
+        if ((int)cnt < K) lo = tau;
+        else hi = tau;
+        tau = (lo > 0.0 && hi > 0.0) ? 0.5 * (lo + hi) : (lo > 0.0 ? lo * 4.0 : hi * 0.5);
+      }
+      if ((int)cnt < K || (int)cnt > CS_CAP) return cleanup(fail(GS_ERR_CUDA, "collective_sample: threshold search failed"));
+      csamp_select_kernel<<<1, 1024, 0, s>>>((const double*)bbuf.ptr, (const int32_t*)((char*)bbuf.ptr + CS_CAP * 8),
+                                             (int)cnt, K, (uint32_t*)sel.ptr);
+      count_launch();
+    }
+    GS_CUDA_TRY(cudaGetLastError());
+  }
+  // the sub-matrix: the entries whose row was selected (CSC order), as A[rows, :]
+  st = new_matrix(out, N);
+  if (st) return cleanup(st);
+  gs_matrix* m = *out;
+  const int64_t n = in->n_cols;
+  if (!m->b_indptr.ensure(m->al, (size_t)(n + 1) * 8, s)) return cleanup(fail(GS_ERR_OUT_OF_MEMORY, "indptr"));
+  int64_t* ip = (int64_t*)m->b_indptr.ptr;
+  GS_CUDA_TRY(cudaMemsetAsync(ip, 0, 8, s));
+  if (n > 0) {
+    row_count_kernel<<<grid_for(n * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
+        (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr, n, (const uint32_t*)sel.ptr, ip);
+    count_launch();
+    if ((st = scan_inclusive(ip + 1, n, m->al, s))) return cleanup(st);
+  }
+  int64_t nnz = 0;
+  GS_CUDA_TRY(cudaMemcpyAsync(&nnz, ip + n, 8, cudaMemcpyDeviceToHost, s));
+  GS_CUDA_TRY(cudaStreamSynchronize(s));
+  if ((st = alloc_entries(m, n, nnz, s))) return cleanup(st);
+  if (n > 0) {
+    GS_CUDA_TRY(cudaMemcpyAsync(m->b_cols.ptr, in->b_cols.ptr, n * 4, cudaMemcpyDeviceToDevice, s));
+    row_copy_kernel<<<grid_for(n * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
+        (const int64_t*)in->b_indptr.ptr, (const int32_t*)in->b_row.ptr, (const int64_t*)in->b_eid.ptr,
+        (const float*)in->b_val.ptr, n, (const uint32_t*)sel.ptr, ip, (int32_t*)m->b_row.ptr, (int64_t*)m->b_eid.ptr,
+        (float*)m->b_val.ptr);
+    count_launch();
+    GS_CUDA_TRY(cudaGetLastError());
+  }
+  return cleanup(GS_OK);
+}
+
+gs_status gs_matrix_map_reduce(gs_matrix* m, const int* ops, const float* scalars, int n_ops, int axis, float* out,
+                               void* stream_) {
+  if (!m || (n_ops > 0 && (!ops || !scalars)) || n_ops < 0 || n_ops > MR_MAX_OPS || axis < -1 || axis > 1 ||
+      (axis >= 0 && !out))
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_map_reduce: bad argument (<= %d ops, axis -1/0/1)", MR_MAX_OPS);
+  MapChain c = {};
+  c.n = n_ops;
+  for (int i = 0; i < n_ops; ++i) {
+    if (ops[i] < GS_OP_ADD || ops[i] > GS_OP_POW) return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_map_reduce: op");
+    c.op[i] = ops[i];
+    c.x[i] = scalars[i];
+  }
+  cudaStream_t s = (cudaStream_t)stream_;
+  if (axis < 0) {  // Edge-Map fusion: the chain applied in place in one pass
+    if (m->nnz > 0) {
+      map_chain_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((float*)m->b_val.ptr, m->nnz, c);
+      count_launch();
+    }
+  } else if (axis == 0) {
+    if (m->n_cols > 0) {
+      map_col_sum_kernel<<<grid_for(m->n_cols * 32, OPS_THREADS), OPS_THREADS, 0, s>>>(
+          (const int64_t*)m->b_indptr.ptr, (const float*)m->b_val.ptr, m->n_cols, c, out);
+      count_launch();
+    }
+  } else {
+    const int64_t N = m->num_nodes;
+    DevBuf acc;
+    if (!acc.ensure(m->al, (size_t)std::max<int64_t>(N, 1) * 8, s)) return fail(GS_ERR_OUT_OF_MEMORY, "map_reduce acc");
+    GS_CUDA_TRY(cudaMemsetAsync(acc.ptr, 0, (size_t)std::max<int64_t>(N, 1) * 8, s));
+    if (m->nnz > 0) {
+      map_row_sum_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((const int32_t*)m->b_row.ptr, (const float*)m->b_val.ptr,
+                                                               m->nnz, c, (double*)acc.ptr);
+      count_launch();
+    }
+    if (N > 0) {
+      to_float_kernel<<<grid_for(N, 256), 256, 0, s>>>((const double*)acc.ptr, N, out);
+      count_launch();
+    }
+    acc.reset(m->al, s);
+  }
+  GS_CUDA_TRY(cudaGetLastError());
+  return GS_OK;
+}
+
+gs_status gs_matrix_asgcn_bias(const gs_matrix* m, const void* X, int F, const float* wg, float* out, void* stream_) {
+  if (!m || !X || !wg || !out || F <= 0) return fail(GS_ERR_INVALID_ARGUMENT, "gs_matrix_asgcn_bias: bad argument");
+  cudaStream_t s = (cudaStream_t)stream_;
+  const int64_t N = m->num_nodes;
+  DevBuf acc;
+  if (!acc.ensure(m->al, (size_t)std::max<int64_t>(N, 1) * 8, s)) return fail(GS_ERR_OUT_OF_MEMORY, "asgcn acc");
+  GS_CUDA_TRY(cudaMemsetAsync(acc.ptr, 0, (size_t)std::max<int64_t>(N, 1) * 8, s));
+  if (m->nnz > 0) {
+    row_sum_kernel<<<grid_for(m->nnz, 256), 256, 0, s>>>((const int32_t*)m->b_row.ptr, (const float*)m->b_val.ptr,
+                                                         m->nnz, (double*)acc.ptr);
+    count_launch();
+  }
+  if (N > 0) {
+    asgcn_bias_kernel<<<grid_for(N * 32, 256), 256, 0, s>>>((const double*)acc.ptr, (const __nv_bfloat16*)X, F, wg,
+                                                             N, out);
+    count_launch();
+  }
+  GS_CUDA_TRY(cudaGetLastError());
+  acc.reset(m->al, s);
+  return GS_OK;
 }
 
 gs_status gs_matrix_get_view(const gs_matrix* m, gs_matrix_view* out) {

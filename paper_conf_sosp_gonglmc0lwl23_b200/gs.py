@@ -38,7 +38,8 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_kernel_launche
            "gs_sample_layerwise",
            "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
            "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
-           "gs_matrix_get_view", "gs_matrix_destroy", "gs_pass_attention", "gs_graph_set_weights"]
+           "gs_matrix_get_view", "gs_matrix_destroy", "gs_matrix_individual_sample",
+           "gs_matrix_collective_sample", "gs_matrix_map_reduce", "gs_matrix_asgcn_bias", "gs_pass_attention", "gs_graph_set_weights"]
 OP_ADD, OP_SUB, OP_MUL, OP_DIV, OP_POW = 0, 1, 2, 3, 4
 
 
@@ -144,6 +145,10 @@ def load_library(path: str = LIB_PATH):
     L.gs_matrix_slice_columns.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_slice_rows.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_sum.argtypes = [vp, i32, vp, vp]
+    L.gs_matrix_individual_sample.argtypes = [vp, i32, i32, i32, u64, i32, i64, vp, ctypes.POINTER(vp)]
+    L.gs_matrix_collective_sample.argtypes = [vp, i32, vp, u64, i32, i64, vp, ctypes.POINTER(vp)]
+    L.gs_matrix_map_reduce.argtypes = [vp, vp, vp, i32, i32, vp, vp]
+    L.gs_matrix_asgcn_bias.argtypes = [vp, vp, i32, vp, vp, vp]
     L.gs_matrix_broadcast.argtypes = [vp, i32, vp, i32, vp]
     L.gs_matrix_elementwise.argtypes = [vp, i32, ctypes.c_float, vp]
     L.gs_matrix_row_ids.argtypes = [vp, vp, ctypes.POINTER(i64), vp]
@@ -530,6 +535,51 @@ class Matrix:
         _check(_lib.gs_matrix_elementwise(self._h, int(op), float(x), _stream_ptr(stream)),
                "gs_matrix_elementwise")
         return self
+
+    def individual_sample(self, K: int, use_values=False, replace=False, rng_key=0, layer=0, batch_index=0,
+                          stream=None) -> "Matrix":
+        """A.individual_sample(K, probs) (probs = the values when use_values)."""
+        h = ctypes.c_void_p()
+        _check(_lib.gs_matrix_individual_sample(self._h, int(K), int(bool(use_values)), int(bool(replace)),
+                                                ctypes.c_uint64(rng_key), int(layer), int(batch_index),
+                                                _stream_ptr(stream), ctypes.byref(h)),
+               "gs_matrix_individual_sample")
+        return Matrix(h, self._keep)
+
+    def collective_sample(self, K: int, node_probs: torch.Tensor = None, rng_key=0, layer=0, batch_index=0,
+                          stream=None) -> "Matrix":
+        """A.collective_sample(K, node_probs) (node_probs: dense float per global id, or None)."""
+        h = ctypes.c_void_p()
+        p = None if node_probs is None else node_probs.to(torch.float32).contiguous()
+        _check(_lib.gs_matrix_collective_sample(self._h, int(K), None if p is None else _ptr(p),
+                                                ctypes.c_uint64(rng_key), int(layer), int(batch_index),
+                                                _stream_ptr(stream), ctypes.byref(h)),
+               "gs_matrix_collective_sample")
+        return Matrix(h, self._keep)
+
+    def map_reduce(self, ops, scalars, axis=None, stream=None):
+        """Fused element-wise chain; axis None: in place (returns self), 0/1: the sums."""
+        o = (ctypes.c_int * len(ops))(*[int(x) for x in ops])
+        sc = (ctypes.c_float * len(scalars))(*[float(x) for x in scalars])
+        if axis is None:
+            _check(_lib.gs_matrix_map_reduce(self._h, o, sc, len(ops), -1, None, _stream_ptr(stream)),
+                   "gs_matrix_map_reduce")
+            return self
+        v = self.view()
+        n = v["cols"].numel() if axis == 0 else v["num_nodes"]
+        out = torch.empty(n, dtype=torch.float32, device="cuda")
+        _check(_lib.gs_matrix_map_reduce(self._h, o, sc, len(ops), int(axis), _ptr(out), _stream_ptr(stream)),
+               "gs_matrix_map_reduce")
+        return out
+
+    def asgcn_bias(self, X: torch.Tensor, wg: torch.Tensor, stream=None) -> torch.Tensor:
+        """AS-GCN-style node bias (R30): dense float[num_nodes]."""
+        X = X.to(torch.bfloat16).contiguous()
+        wg = wg.to(torch.float32).contiguous()
+        out = torch.empty(self.view()["num_nodes"], dtype=torch.float32, device="cuda")
+        _check(_lib.gs_matrix_asgcn_bias(self._h, _ptr(X), X.shape[1], _ptr(wg), _ptr(out), _stream_ptr(stream)),
+               "gs_matrix_asgcn_bias")
+        return out
 
     def row_ids(self, stream=None) -> torch.Tensor:
         """A.row(): distinct row ids ascending."""
