@@ -95,12 +95,14 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
                            int64_t batch_base, const int32_t* fanouts, int L, int replace, int bias,
                            uint64_t key, cudaStream_t stream, gs_blocks* blk);
 // node-wise engine: the hop-synchronous kernels (default) or the round-1
-// single-launch wave kernel (GS_NODEWISE=wave; kept for comparison)
+// single-launch wave kernel (GS_NODEWISE=wave; host-mapped graphs)
 gs_status run_nodewise(const gs_graph* g, const int32_t* seeds, int64_t num_seeds,
                        int64_t batch_size, int64_t batch_base, const int32_t* fanouts, int L,
                        int replace, int bias, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
+  // host-mapped (UVA) graphs: the wave kernel (PD, index array in host
+  // memory: 31.5 ms vs 81.6 for the hop engine's per-lane register gathers)
   const char* e = getenv("GS_NODEWISE");
-  if (e && e[0] == 'w')
+  if ((e && e[0] == 'w') || (g->host_mapped && !(e && e[0] == 'h')))
     return run_nodewise_wave(g, seeds, num_seeds, batch_size, batch_base, fanouts, L, replace, bias, key,
                              stream, blk);
   return run_nodewise_hop(g, seeds, num_seeds, nullptr, batch_size, (num_seeds + batch_size - 1) / batch_size,

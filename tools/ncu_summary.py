@@ -41,6 +41,7 @@ def main():
     hdr, units = rows[0], rows[1]
     lines = [f"# ncu summary: {os.path.basename(rep)}", ""]
     traffic = None
+    total = 0.0  # summed over every captured launch (e.g. the select kernel of each hop of one step)
     for r in rows[2:]:
         name = r[hdr.index("Kernel Name")] if "Kernel Name" in hdr else "?"
         lines.append(f"## {name}")
@@ -72,10 +73,14 @@ def main():
                 v = float(r[i])
                 return v * {"Tbyte": 1e12, "Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0}.get(units[i], 1.0)
             traffic = gb("dram__bytes_read.sum") + gb("dram__bytes_write.sum")
+            total += traffic
             lines.append(f"DRAM bytes (read + write) per launch: {traffic:.4g}")
             lines.append("")
         except (ValueError, KeyError):
             pass
+    if len(rows) > 3:
+        lines.append(f"DRAM bytes (read + write) summed over the {len(rows) - 2} captured launches: {total:.4g}")
+        traffic = total
     with open(out, "w") as f:
         f.write("\n".join(lines) + "\n")
     if workload and traffic is not None:
