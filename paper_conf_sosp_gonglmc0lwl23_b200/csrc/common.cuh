@@ -28,6 +28,13 @@ __device__ __forceinline__ U4 philox(uint32_t c0, uint32_t c1, uint32_t c2, uint
   return U4{c0, c1, c2, c3};
 }
 
+// Out-of-line copies for the weighted select kernels: inlined at every call
+// site they made the kernel ~9k instructions and its warps stalled on
+// instruction fetch (ncu: no_instructions the top stall reason).
+static __device__ __noinline__ U4 philox_nl(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3, uint64_t key) {
+  return philox(c0, c1, c2, c3, key);
+}
+
 enum : uint32_t { TAG_FLOYD = 1, TAG_REPLACE = 2, TAG_ARES_NODE = 3, TAG_ARES_LAYER = 4,
                   TAG_DEEPWALK = 5, TAG_NODE2VEC = 6 };
 
@@ -46,6 +53,7 @@ __device__ __forceinline__ double ares_key(uint32_t r, double bias) {
   double u = ((double)r + 0.5) * 0x1p-32;
   return -log(u) / bias;
 }
+static __device__ __noinline__ double ares_key_nl(uint32_t r, double bias) { return ares_key(r, bias); }
 
 // (key, pos) lexicographic order: smaller key wins, ties -> smaller position.
 __device__ __forceinline__ bool key_less(double ka, int64_t pa, double kb, int64_t pb) {

@@ -78,6 +78,18 @@ __device__ __forceinline__ int warp_excl(int v, int* total) {
   return inc - v;
 }
 
+__device__ __forceinline__ long long warp_excl_ll(long long v, long long* total) {
+  const int lane = threadIdx.x & 31;
+  long long inc = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const long long n = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += n;
+  }
+  *total = __shfl_sync(0xffffffffu, inc, 31);
+  return inc - v;
+}
+
 // ---------------------------------------------------------------------------
 // A-Res by candidate filtering (R6).  The k smallest exact keys
 // key_i = -ln((r_i + 0.5) 2^-32) / w_i (fp64, as the oracle) are found among
@@ -141,7 +153,7 @@ __device__ __forceinline__ void ares_filter(const NWCore& P, int32_t v, int64_t 
     float w[4] = {0.f, 0.f, 0.f, 0.f};
     uint32_t r[4] = {0u, 0u, 0u, 0u};
     if (i0 < d) {
-      const U4 R = philox((uint32_t)v, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.key);
+      const U4 R = philox_nl((uint32_t)v, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.key);
       r[0] = R.x; r[1] = R.y; r[2] = R.z; r[3] = R.w;
 #pragma unroll
       for (int q = 0; q < 4; ++q)
@@ -182,9 +194,9 @@ __device__ __forceinline__ int ares_exact(const NWCore& P, int32_t v, int64_t of
   int below = 0;
   for (int j = lane; j < m; j += 32) {
     const uint32_t p = pos[j];
-    const U4 R = philox((uint32_t)v, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.key);
+    const U4 R = philox_nl((uint32_t)v, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.key);
     const float w = P.weights ? __ldg(P.weights + off + p) : 1.0f;
-    const double kk = ares_key(sel_word(R, (int)(p & 3)), (double)w);
+    const double kk = ares_key_nl(sel_word(R, (int)(p & 3)), (double)w);
     key[j] = kk;
     below += (tau < 0.0f || kk < (double)tau) ? 1 : 0;
   }

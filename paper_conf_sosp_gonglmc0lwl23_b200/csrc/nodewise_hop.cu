@@ -83,6 +83,9 @@ struct HopParams {
   int64_t nw, nwp, nsw;      // words used / allocated per batch, summary words
   int sel_nq, sel_claim;     // select: claim queues, chunks per claim
   int sel_ld;                // select: gather load flavour (0 nc, 1 cg, 2 nc no-L1-allocate)
+  int ares_split;            // A-Res columns with d > 64: 1 hop_ares_big_kernel, 0 in select
+  int ares_tau;              // hop_ares_big_kernel's first threshold: 0 normal, 1 too tight,
+                             // 2 too loose (tests: every widen / narrow step runs)
   int wsh;                   // bitmap word index shift: 1 = 64-bit words (global finalize), 0 = 32-bit (cluster)
 };
 
@@ -304,7 +307,7 @@ struct HSmem {
 // the lane's sampled rows gathered 16 at a time, bitmap bits set, edge id / row
 // id staged slot-major in shared memory, then written out coalesced.
 template <bool WEIGHTED, int KCAP>
-__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_MINB : 2))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
+__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_MINB : 2))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
                                                                  unsigned int* claim) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = HSmem<WEIGHTED, KCAP>;
@@ -376,6 +379,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
     const int64_t ebase = __ldcg(P.indptr_out[l] + cb + b + jb);  // first edge of the chunk
     int cnt = 0;
     bool all = false;
+    bool defer = false;  // weighted, d > 64: written by hop_ares_big_kernel
     float csum = 1.0f;
     uint32_t a[KCAP];  // positions (compile-time indexed registers)
 #pragma unroll
@@ -417,7 +421,102 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
           if (!wts || __ldg(wts + off + i) > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
       }
       HWarpA& A = reinterpret_cast<HWarpA*>(&sm + 1)[warp];
-      uint32_t med = __ballot_sync(0xffffffffu, d > k);
+      // k < d <= 64: four columns at a time, eight lanes each; every eligible
+      // edge's exact key is held in registers (lane s: positions 32 t + 4 s + q)
+      // and the want = min(k, eligible) smallest (key, position) pairs are
+      // taken by want rounds of a group argmin
+      uint32_t sml = __ballot_sync(0xffffffffu, d > k && d <= 64);
+      const int g8 = lane >> 3, s8 = lane & 7;
+      while (sml) {
+        int cc = -1;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const int bt = __ffs(sml) - 1;
+          if (sml) {
+            sml &= sml - 1u;
+            if (t == g8) cc = bt;
+          }
+        }
+        const int src = cc < 0 ? 0 : cc;
+        const int32_t vc = __shfl_sync(0xffffffffu, v, src);
+        const int64_t oc = __shfl_sync(0xffffffffu, off, src);
+        const int dsrc = __shfl_sync(0xffffffffu, (int)d, src);
+        const int dc = cc < 0 ? 0 : dsrc;
+        double kk[8];
+        int elig = 0;
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+          const int i0 = 32 * t + 4 * s8;
+          U4 R{0u, 0u, 0u, 0u};
+          if (i0 < dc) R = philox_nl((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.core.key);
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const float w = i0 + q < dc ? (wts ? __ldg(wts + oc + i0 + q) : 1.0f) : 0.0f;
+            kk[4 * t + q] = w > 0.0f ? ares_key_nl(sel_word(R, q), (double)w) : INFINITY;
+            elig += w > 0.0f ? 1 : 0;
+          }
+        }
+        elig += __shfl_xor_sync(0xffffffffu, elig, 4);
+        elig += __shfl_xor_sync(0xffffffffu, elig, 2);
+        elig += __shfl_xor_sync(0xffffffffu, elig, 1);
+        const int want = min(k, elig);
+        int rounds = want;
+        rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, 8));
+        rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, 16));
+        for (int r = 0; r < rounds; ++r) {
+          double bk = INFINITY;
+          uint32_t bp = 0xFFFFFFFFu;
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const uint32_t pj = (uint32_t)(32 * (j >> 2) + 4 * s8 + (j & 3));
+            if (key_less(kk[j], pj, bk, bp)) { bk = kk[j]; bp = pj; }
+          }
+#pragma unroll
+          for (int o = 4; o > 0; o >>= 1) {
+            const double ok = __shfl_xor_sync(0xffffffffu, bk, o);
+            const uint32_t op = __shfl_xor_sync(0xffffffffu, bp, o);
+            if (key_less(ok, op, bk, bp)) { bk = ok; bp = op; }
+          }
+          if (r < want) {
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              if ((uint32_t)(32 * (j >> 2) + 4 * s8 + (j & 3)) == bp) kk[j] = INFINITY;
+            if (s8 == 0) C.list[r][cc] = bp;
+          }
+        }
+        __syncwarp();
+        // the want winners of column cc in ascending position order
+        uint32_t wp[(KCAP + 7) / 8];
+#pragma unroll
+        for (int t = 0; t < (KCAP + 7) / 8; ++t) {
+          const int j = s8 + 8 * t;
+          wp[t] = j < want ? C.list[j][src] : 0xFFFFFFFFu;
+        }
+        int rk8[(KCAP + 7) / 8];
+#pragma unroll
+        for (int t = 0; t < (KCAP + 7) / 8; ++t) rk8[t] = 0;
+        for (int i = 0; i < want; ++i) {
+          const uint32_t pi = C.list[i][src];
+#pragma unroll
+          for (int t = 0; t < (KCAP + 7) / 8; ++t) rk8[t] += pi < wp[t] ? 1 : 0;
+        }
+        __syncwarp();
+#pragma unroll
+        for (int t = 0; t < (KCAP + 7) / 8; ++t)
+          if (s8 + 8 * t < want) C.list[rk8[t]][cc] = wp[t];
+        if (cc >= 0 && s8 == 0) A.rk[cc] = want;
+        __syncwarp();
+      }
+      if (d > k && d <= 64) cnt = A.rk[lane];
+      __syncwarp();
+      // d > 64: the heavy-column kernel (hop_ares_big_kernel) selects, gathers
+      // and writes these columns; here only their output range is reserved
+      const bool big = d > 64;
+      if (big && P.ares_split) {
+        defer = true;
+        cnt = min(k, P.poscnt && wts ? __ldg(P.poscnt + v) : (int)d);
+      }
+      uint32_t med = __ballot_sync(0xffffffffu, big && !defer);
       while (med) {
         const int cc = __ffs(med) - 1;
         med &= med - 1u;
@@ -463,7 +562,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
         const int i = h + q;
         const uint32_t ps = all ? (uint32_t)i : a[i];
         u[q] = 0u;
-        if (i < cnt) {
+        if (i < cnt && !defer) {
           const int32_t* ap = P.core.indices + off + ps;
           if (P.sel_ld == 1) u[q] = (uint32_t)ldh(ap, pf);  // L2 only
           else if (P.sel_ld == 2)
@@ -474,7 +573,9 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
 #pragma unroll
       for (int q = 0; q < 16 && h + q < KCAP; ++q) {
         const int i = h + q;
-        if (i < cnt) {
+        if (i < cnt && defer) {
+          C.se[pre + i] = ~0ull;  // reserved (hop_ares_big_kernel)
+        } else if (i < cnt) {
           const uint32_t ps = all ? (uint32_t)i : a[i];
           C.se[pre + i] = (unsigned long long)(off + ps);
           C.su[pre + i] = u[q];
@@ -497,6 +598,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
     int64_t* eid_out = P.eid[l] + rb + ebase;
     float* val_out = P.val[l] ? P.val[l] + rb + ebase : nullptr;
     for (int f = lane; f < total; f += 32) {
+      if (WEIGHTED && C.se[f] == ~0ull) continue;
       sth(eid_out + f, (int64_t)C.se[f], pf);
       sth(rl_out + f, (int32_t)C.su[f], pf);
       if constexpr (WEIGHTED) {
@@ -507,6 +609,247 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 1 : (KCAP <= 16 ? SEL_
     if (++c >= cend) {
       c = grab();
       cend = c < 0 ? -1 : min(min(c + CLAIM, (long long)(q + 1) * qlen), nchunks);
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// A-Res (R6) for the heavy columns (d > 64) of a hop: a warp per column, in a
+// lean kernel of its own (2 KB of shared memory and <= 64 registers per warp,
+// so 32 warps per SM hide the weight stream's latency; inside the select
+// kernel the same loop ran at 16 warps per SM and stalled on instruction
+// fetch).  Candidate filter (one Philox per 4 edges, the next 128 edges'
+// weights loaded while the current ones are tested), exact fp64 keys of the
+// <= 128 candidates held in registers, want = min(k, eligible) rounds of a
+// warp argmin over (key, position), then the winners in position order are
+// gathered and written to the block's reserved CSC range (hop_select left it
+// untouched) and their rows' bitmap bits set.
+// ---------------------------------------------------------------------------
+constexpr int AB_THREADS = 256;
+constexpr int AB_WARPS = AB_THREADS / 32;
+constexpr int AB_CAP = 128;  // candidates per column pass (4 per lane)
+
+__global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P, int l, int64_t b0, int nbg,
+                                                                     unsigned int* claim) {
+  __shared__ long long cpre[MAX_GROUP + 1];
+  __shared__ long long scr[40];
+  __shared__ uint32_t cpos[AB_WARPS][AB_CAP];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  {
+    long long run = 0;
+    for (int i0 = 0; i0 < nbg; i0 += AB_THREADS) {
+      const int i = i0 + threadIdx.x;
+      const long long c = i < nbg ? (hp_T(P, b0 + i, l) + 31) / 32 : 0;
+      long long tot;
+      const long long ex = block_exclusive_scan<long long>(c, scr, &tot);
+      if (i < nbg) cpre[i] = run + ex;
+      run += tot;
+    }
+    if (threadIdx.x == 0) cpre[nbg] = run;
+    __syncthreads();
+  }
+  const long long nchunks = cpre[nbg];
+  const int k = P.k[l];
+  const uint64_t pf = pol_first();
+  const float* wts = P.core.weights;
+  uint32_t* pos = cpos[warp];
+  int lo = 0;
+  for (;;) {
+    unsigned int x = 0;
+    if (lane == 0) x = atomicAdd(claim, 1u);
+    const long long c = (long long)__shfl_sync(0xffffffffu, x, 0);
+    if (c >= nchunks) break;
+    if (!(cpre[lo] <= c && c < cpre[lo + 1])) {
+      int lo2 = 0, hi2 = nbg - 1;
+      while (lo2 < hi2) {
+        const int mid = (lo2 + hi2 + 1) >> 1;
+        if (cpre[mid] <= c) lo2 = mid;
+        else hi2 = mid - 1;
+      }
+      lo = lo2;
+    }
+    const int64_t b = b0 + lo;
+    const long long T = hp_T(P, b, l);
+    const long long jb = (c - cpre[lo]) * 32;
+    const int64_t cb = hp_cbase(P, b, l);
+    const int64_t rb = __ldg(P.bptr + b) * P.K[l];
+    const uint32_t gb = (uint32_t)(P.batch_base + b);
+    const long long jcol = jb + lane;
+    const bool active = jcol < T;
+    const int64_t d = active ? (int64_t)__ldcg(P.dcol + cb + jcol) : 0;
+    uint32_t bigm = __ballot_sync(0xffffffffu, d > 64);
+    if (!bigm) continue;
+    const int32_t* F = hp_frontier(P, b, l);
+    const int32_t v = active ? __ldcg(F + jcol) : -1;
+    const int64_t off = active ? __ldcg(P.coff + cb + jcol) : 0;
+    const int64_t slot = b - b0;
+    uint32_t* bits = (uint32_t*)(P.bm + slot * P.nwp);
+    uint32_t* summ = P.summ + slot * P.nsw;
+    const int use_sum = P.use_sum[l];
+    while (bigm) {
+      const int cc = __ffs(bigm) - 1;
+      bigm &= bigm - 1u;
+      const int32_t vc = __shfl_sync(0xffffffffu, v, cc);
+      const int64_t oc = __shfl_sync(0xffffffffu, off, cc);
+      const int dc = (int)__shfl_sync(0xffffffffu, d, cc);
+      const int elig = P.poscnt && wts ? __ldg(P.poscnt + vc) : dc;
+      const int want = min(k, elig);
+      if (want == 0) continue;
+      const float W = wts ? __ldg(P.core.colsum + vc) : (float)dc;
+      // tau ~ (k + 8) / W expects k + 8 keys below it (widened when fewer
+      // than want, narrowed when the candidates overflow); tau < 0: every
+      // eligible edge is a candidate
+      const float tau0 = W > 0.0f ? (float)(k + 8) / W : -1.0f;
+      float tau = tau0 < 0.0f ? -1.0f : (P.ares_tau == 1 ? 0.25f * tau0 : (P.ares_tau == 2 ? 16.0f * tau0 : tau0));
+      TauSearch ts{tau, 0.0f, 0.0f};
+      const float* wc = wts ? wts + oc : nullptr;
+      double kk[4];
+      uint32_t pp[4];
+      int M = 0;
+      bool good = false;
+      const unsigned lt = (1u << lane) - 1u;
+      for (int it = 0; it < 64 && !good; ++it) {
+        tau = ts.tau;
+        const float t101 = __fmul_rn(tau, 1.01f);
+        // filter: candidate iff E_lb(r) <= tau w (1 + 1%), with
+        // E(r) = -ln(1 - x) >= x + x^2 / 2, x = (2^32 - r - 0.5) 2^-32
+        M = 0;
+        float wn[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const int i = 4 * lane + q;
+          wn[q] = i < dc ? (wc ? ldg_h(wc + i, pf) : 1.0f) : 0.0f;
+        }
+        for (int base = 0; base < dc; base += 128) {
+          float w[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) w[q] = wn[q];
+          const int i0 = base + 4 * lane;
+          if (base + 128 < dc) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int i = i0 + 128 + q;
+              wn[q] = i < dc ? (wc ? ldg_h(wc + i, pf) : 1.0f) : 0.0f;
+            }
+          }
+          unsigned fl = 0u;
+          if (tau < 0.0f) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) fl |= w[q] > 0.0f ? (1u << q) : 0u;
+          } else {
+            const U4 R = philox((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.core.key);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const float x = __fmul_rn(__uint2float_rn(~sel_word(R, q)) + 0.5f, 2.3283064365386963e-10f);
+              const bool cnd = w[q] > 0.0f && __fmaf_rn(0.5f * x, x, x) <= __fmul_rn(t101, w[q]);
+              fl |= cnd ? (1u << q) : 0u;
+            }
+          }
+          // append in (lane, q) order: prefix of the per-lane counts by bit ballots
+          const int n = __popc(fl);
+          const unsigned b0 = __ballot_sync(0xffffffffu, n & 1), b1 = __ballot_sync(0xffffffffu, n & 2),
+                         b2 = __ballot_sync(0xffffffffu, n & 4);
+          if (b0 | b1 | b2) {
+            int o = M + __popc(b0 & lt) + 2 * __popc(b1 & lt) + 4 * __popc(b2 & lt);
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              if (fl & (1u << q)) {
+                if (o < AB_CAP) pos[o] = (uint32_t)(i0 + q);
+                ++o;
+              }
+            M += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2);
+          }
+        }
+        __syncwarp();
+        if (M > AB_CAP) {  // too many candidates: narrow
+          if (!ts.next(-2, tau0)) break;
+          continue;
+        }
+        // exact keys (fp64, as the oracle)
+        int below = 0;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const int j = lane + 32 * t;
+          kk[t] = INFINITY;
+          pp[t] = 0xFFFFFFFFu;
+          if (32 * t < M && j < M) {
+            const uint32_t p = pos[j];
+            const U4 R = philox((uint32_t)vc, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.core.key);
+            const float wj = wc ? __ldg(wc + p) : 1.0f;
+            kk[t] = ares_key(sel_word(R, (int)(p & 3)), (double)wj);
+            pp[t] = p;
+            below += (tau < 0.0f || kk[t] < (double)tau) ? 1 : 0;
+          }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) below += __shfl_xor_sync(0xffffffffu, below, o);
+        __syncwarp();
+        if (below < want) {  // too few keys below tau: widen
+          if (!ts.next(-1, tau0)) break;
+          continue;
+        }
+        good = true;
+      }
+      if (!good) {
+        if (lane == 0) atomicOr(P.core.err, ERR_INTERNAL);
+        continue;
+      }
+      uint32_t mine = 0xFFFFFFFFu;
+      if (M <= 32) {
+        // one candidate per lane: bitonic sort of (key, position) across the
+        // warp; lanes 0 .. want-1 then hold the want smallest
+        double K = kk[0];
+        uint32_t Q = pp[0];
+#pragma unroll
+        for (int size = 2; size <= 32; size <<= 1) {
+#pragma unroll
+          for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            const double ok = __shfl_xor_sync(0xffffffffu, K, stride);
+            const uint32_t oq = __shfl_xor_sync(0xffffffffu, Q, stride);
+            const bool asc = (lane & size) == 0 || size == 32;
+            const bool low = (lane & stride) == 0;
+            const bool ol = key_less(ok, oq, K, Q);
+            if (low == asc ? ol : (!ol && !(ok == K && oq == Q))) { K = ok; Q = oq; }
+          }
+        }
+        if (lane < want) mine = Q;
+      } else {
+        // want rounds of a warp argmin over (key, position)
+        for (int r = 0; r < want; ++r) {
+          double bk = INFINITY;
+          uint32_t bp = 0xFFFFFFFFu;
+#pragma unroll
+          for (int t = 0; t < 4; ++t)
+            if (key_less(kk[t], pp[t], bk, bp)) { bk = kk[t]; bp = pp[t]; }
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) {
+            const double ok = __shfl_xor_sync(0xffffffffu, bk, o);
+            const uint32_t op = __shfl_xor_sync(0xffffffffu, bp, o);
+            if (key_less(ok, op, bk, bp)) { bk = ok; bp = op; }
+          }
+#pragma unroll
+          for (int t = 0; t < 4; ++t)
+            if (pp[t] == bp) { kk[t] = INFINITY; pp[t] = 0xFFFFFFFFu; }
+          if (lane == r) mine = bp;
+        }
+      }
+      // the winners in position order, gathered and written out
+      int o = 0;
+      for (int s2 = 0; s2 < want; ++s2) o += __shfl_sync(0xffffffffu, mine, s2) < mine ? 1 : 0;
+      if (lane < want) {
+        const int64_t ce = __ldcg(P.indptr_out[l] + cb + b + jb + cc);  // the column's first edge
+        const int64_t e = oc + mine;
+        const uint32_t u = (uint32_t)ldg_h(P.core.indices + e, pf);
+        sth(P.eid[l] + rb + ce + o, (int64_t)e, pf);
+        sth(P.row_local[l] + rb + ce + o, (int32_t)u, pf);
+        if (P.val[l]) {
+          const float w = wts ? __ldg(wts + e) : 1.0f;
+          sth(P.val[l] + rb + ce + o, w / W, pf);
+        }
+        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + ((u >> 5) << P.wsh)), "r"(1u << (u & 31)) : "memory");
+        if (use_sum)
+          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (u >> 10)), "r"(1u << ((u >> 5) & 31)) : "memory");
+      }
     }
   }
 }
@@ -747,6 +1090,10 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.sel_claim = 2;
   P.sel_ld = 0;
   if (const char* e = getenv("GS_SEL_LD")) P.sel_ld = atoi(e);
+  P.ares_split = 1;
+  if (const char* e = getenv("GS_ARES_SPLIT")) P.ares_split = atoi(e);
+  P.ares_tau = 0;
+  if (const char* e = getenv("GS_ARES_TAU")) P.ares_tau = atoi(e);
   if (const char* e = getenv("GS_SEL_NQ")) P.sel_nq = std::max(1, std::min(32, atoi(e)));
   if (const char* e = getenv("GS_SEL_CLAIM")) P.sel_claim = std::max(1, atoi(e));
   int ntile[MAX_LAYERS];
@@ -802,7 +1149,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   int64_t stat_words = 0;
   for (int l = 0; l < L; ++l) stat_words += WB * (nseg_max[l] + ntile[l]);
   const int64_t ctr_q_off = std::max<int64_t>(G * L, 1) * 4 + G * stat_words * 2;  // in uints
-  const int64_t ctr_bytes = a256h(ctr_q_off * 4 + std::max<int64_t>(G * L, 1) * 4096);
+  const int64_t ctr_bytes = a256h(ctr_q_off * 4 + std::max<int64_t>(G * L, 1) * 8192);
   const int64_t bptr_bytes = a256h((nbatch + 1) * 8);
   ok = ok && need(blk->b_meta, nbatch * L * 8 * 8) && need(blk->b_err, 16) &&
        need(blk->b_sched, ctr_bytes + bptr_bytes);
@@ -908,7 +1255,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     P.summ = P0.summ + si * WB * P.nsw;
     for (int l = 0; l < L; ++l) {
       unsigned int* c4 = ctr + (gi * L + l) * 4;
-      unsigned int* cq = ctr + ctr_q_off + (gi * L + l) * 1024;
+      unsigned int* cq = ctr + ctr_q_off + (gi * L + l) * 2048;  // select queues, then the heavy-column counter
       const Scan snp{c4 + 0, st};
       st += WB * nseg_max[l];
       const Scan srow{c4 + 1, st};
@@ -930,6 +1277,20 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       }
       if (rc) return rc;
       mark("select", l);
+      if (weighted && P.ares_split) {
+        static int grid_big = 0;
+        if (grid_big == 0) {
+          int per_sm = 0, dev = 0, sms = 148;
+          GS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hop_ares_big_kernel, AB_THREADS, 0));
+          cudaGetDevice(&dev);
+          cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+          grid_big = std::max(1, per_sm) * sms;
+          if (getenv("GS_VERBOSE")) fprintf(stderr, "hop_ares_big: %d CTAs/SM\n", per_sm);
+        }
+        hop_ares_big_kernel<<<grid_big, AB_THREADS, 0, stream>>>(P, l, b0, nbg, cq + 1024); count_launch();
+        GS_CUDA_TRY(cudaGetLastError());
+        mark("ares", l);
+      }
       hop_rows_kernel<<<(unsigned)(nbg * ntile[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, ntile[l], srow); count_launch();
       GS_CUDA_TRY(cudaGetLastError());
       mark("rows", l);

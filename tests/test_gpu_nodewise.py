@@ -69,8 +69,15 @@ def test_kgcn_replace(gs, oracle_lib, medium):
     compare_all(out, ref, "kgcn")
 
 
-@pytest.mark.parametrize("mode", [1, 2])
-def test_weighted_ares_and_pass(gs, oracle_lib, medium, mode):
+@pytest.mark.parametrize("mode,split,tau", [(1, "1", "0"), (2, "1", "0"), (1, "0", "0"),
+                                            (1, "1", "1"), (1, "1", "2")])
+def test_weighted_ares_and_pass(gs, oracle_lib, medium, mode, split, tau, monkeypatch):
+    """A-Res / PASS-style.  GS_ARES_SPLIT: 1 heavy columns (d > 64) in their
+    own kernel (default), 0 inside the select kernel; GS_ARES_TAU 1 / 2 start
+    the heavy-column threshold too tight / too loose so that every widen and
+    narrow step of the search runs."""
+    monkeypatch.setenv("GS_ARES_SPLIT", split)
+    monkeypatch.setenv("GS_ARES_TAU", tau)
     g, G, O = medium
     seeds = synth.make_seeds(synth.GraphSpec("m", 200_000, 1, True, None, 5), 2048)
     out = gs.sample_neighbors(G, seeds.cuda(), [10, 10], batch_size=1024, bias_mode=mode,
