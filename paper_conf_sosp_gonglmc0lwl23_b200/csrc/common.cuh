@@ -28,6 +28,34 @@ __device__ __forceinline__ U4 philox(uint32_t c0, uint32_t c1, uint32_t c2, uint
   return U4{c0, c1, c2, c3};
 }
 
+// The same generator with the ten round keys precomputed (philox_keys, on the
+// host): kept in kernel-parameter space they are constant-bank operands of the
+// round's XOR, so a round is two wide multiplies and two LOP3s.
+struct PhiloxKeys { uint32_t k[20]; };
+inline PhiloxKeys philox_keys(uint64_t key) {
+  PhiloxKeys r;
+  uint32_t k0 = (uint32_t)key, k1 = (uint32_t)(key >> 32);
+  for (int i = 0; i < 10; ++i) {
+    r.k[2 * i] = k0;
+    r.k[2 * i + 1] = k1;
+    k0 += 0x9E3779B9u;
+    k1 += 0xBB67AE85u;
+  }
+  return r;
+}
+__device__ __forceinline__ U4 philox_k(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3, const PhiloxKeys& K) {
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    const uint64_t p0 = (uint64_t)0xD2511F53u * c0, p1 = (uint64_t)0xCD9E8D57u * c2;
+    const uint32_t n0 = (uint32_t)(p1 >> 32) ^ c1 ^ K.k[2 * r], n2 = (uint32_t)(p0 >> 32) ^ c3 ^ K.k[2 * r + 1];
+    c1 = (uint32_t)p1;
+    c3 = (uint32_t)p0;
+    c0 = n0;
+    c2 = n2;
+  }
+  return U4{c0, c1, c2, c3};
+}
+
 // Out-of-line copies for the weighted select kernels: inlined at every call
 // site they made the kernel ~9k instructions and its warps stalled on
 // instruction fetch (ncu: no_instructions the top stall reason).

@@ -59,6 +59,7 @@ constexpr int ROW_STAGE = 4096;             // rows of a tile staged in smem for
 
 struct HopParams {
   NWCore core;
+  PhiloxKeys pk;             // round keys of core.key
   const int32_t* poscnt;     // weighted graphs: #{w > 0} per column (a0), else NULL
   const int32_t* seeds;
   const int64_t* bptr;       // [nb + 1] seed offsets of the batches (device)
@@ -388,7 +389,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
       if (P.core.replace) {  // KGCN (R10): k i.i.d. positions in slot order
         cnt = d > 0 ? k : 0;
         for (int s = 0; s < cnt; ++s) {
-          const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.core.key);
+          const U4 r = philox_k((uint32_t)v, (uint32_t)s, ctr2(l, TAG_REPLACE), gb, P.pk);
           const uint32_t x = (uint32_t)draw_below((uint64_t)d, r.x, r.y);
 #pragma unroll
           for (int i = 0; i < KCAP; ++i) if (i == s) a[i] = x;
@@ -399,7 +400,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
       } else {  // GraphSAGE (R5): Floyd (membership test against the unsorted set), then sorted
         cnt = k;
         for (int s = 0; s < k; ++s) {
-          const U4 r = philox((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.core.key);
+          const U4 r = philox_k((uint32_t)v, (uint32_t)s, ctr2(l, TAG_FLOYD), gb, P.pk);
           const uint32_t m = (uint32_t)(d - k + s);
           const uint32_t t = (uint32_t)draw_below((uint64_t)m + 1, r.x, r.y);
           bool dup = false;
@@ -628,12 +629,17 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
 constexpr int AB_THREADS = 256;
 constexpr int AB_WARPS = AB_THREADS / 32;
 constexpr int AB_CAP = 128;  // candidates per column pass (4 per lane)
+#ifndef AB_MINB
+#define AB_MINB 3            // CTAs per SM (80 registers; 4 -> 64 registers spills)
+#endif
 
-__global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P, int l, int64_t b0, int nbg,
+__global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopParams P, int l, int64_t b0, int nbg,
                                                                      unsigned int* claim) {
   __shared__ long long cpre[MAX_GROUP + 1];
   __shared__ long long scr[40];
-  __shared__ uint32_t cpos[AB_WARPS][AB_CAP];
+  __shared__ uint32_t cpos[AB_WARPS][AB_CAP];  // candidates: position, random word, weight
+  __shared__ uint32_t crnd[AB_WARPS][AB_CAP];
+  __shared__ float cwt[AB_WARPS][AB_CAP];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   {
     long long run = 0;
@@ -653,6 +659,8 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
   const uint64_t pf = pol_first();
   const float* wts = P.core.weights;
   uint32_t* pos = cpos[warp];
+  uint32_t* rnd = crnd[warp];
+  float* cw = cwt[warp];
   int lo = 0;
   for (;;) {
     unsigned int x = 0;
@@ -686,16 +694,23 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
     uint32_t* bits = (uint32_t*)(P.bm + slot * P.nwp);
     uint32_t* summ = P.summ + slot * P.nsw;
     const int use_sum = P.use_sum[l];
+    // per-column a0 values and output offsets, loaded for all heavy columns
+    // of the chunk at once (one latency per chunk, not three per column)
+    const bool mybig = d > 64;
+    const int my_elig = mybig ? (P.poscnt && wts ? __ldg(P.poscnt + v) : (int)d) : 0;
+    const float my_W = mybig ? (wts ? __ldg(P.core.colsum + v) : (float)d) : 0.0f;
+    const int64_t my_ce = mybig ? __ldcg(P.indptr_out[l] + cb + b + jcol) : 0;  // the column's first edge
     while (bigm) {
       const int cc = __ffs(bigm) - 1;
       bigm &= bigm - 1u;
       const int32_t vc = __shfl_sync(0xffffffffu, v, cc);
       const int64_t oc = __shfl_sync(0xffffffffu, off, cc);
       const int dc = (int)__shfl_sync(0xffffffffu, d, cc);
-      const int elig = P.poscnt && wts ? __ldg(P.poscnt + vc) : dc;
+      const int elig = __shfl_sync(0xffffffffu, my_elig, cc);
+      const float W = __shfl_sync(0xffffffffu, my_W, cc);
+      const int64_t ce = __shfl_sync(0xffffffffu, my_ce, cc);
       const int want = min(k, elig);
       if (want == 0) continue;
-      const float W = wts ? __ldg(P.core.colsum + vc) : (float)dc;
       // tau ~ (k + 8) / W expects k + 8 keys below it (widened when fewer
       // than want, narrowed when the candidates overflow); tau < 0: every
       // eligible edge is a candidate
@@ -710,9 +725,9 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
       const unsigned lt = (1u << lane) - 1u;
       for (int it = 0; it < 64 && !good; ++it) {
         tau = ts.tau;
-        const float t101 = __fmul_rn(tau, 1.01f);
-        // filter: candidate iff E_lb(r) <= tau w (1 + 1%), with
-        // E(r) = -ln(1 - x) >= x + x^2 / 2, x = (2^32 - r - 0.5) 2^-32
+        const float t32 = __fmul_rn(__fmul_rn(tau, 1.01f), 4294967296.0f);
+        // filter: candidate iff x <= tau w (1 + 1%), x = (2^32 - r - 0.5) 2^-32:
+        // E(r) = -ln(1 - x) >= x, so every key below tau is a candidate
         M = 0;
         float wn[4];
 #pragma unroll
@@ -733,19 +748,16 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
             }
           }
           unsigned fl = 0u;
-          if (tau < 0.0f) {
+          const U4 R = philox_k((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.pk);
 #pragma unroll
-            for (int q = 0; q < 4; ++q) fl |= w[q] > 0.0f ? (1u << q) : 0u;
-          } else {
-            const U4 R = philox((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.core.key);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              const float x = __fmul_rn(__uint2float_rn(~sel_word(R, q)) + 0.5f, 2.3283064365386963e-10f);
-              const bool cnd = w[q] > 0.0f && __fmaf_rn(0.5f * x, x, x) <= __fmul_rn(t101, w[q]);
-              fl |= cnd ? (1u << q) : 0u;
-            }
+          for (int q = 0; q < 4; ++q) {
+            // x <= tau w (1 + 1%) in units of 2^-32 (w = 0: the bound is < 0)
+            const bool cnd = tau < 0.0f ? w[q] > 0.0f
+                                        : __uint2float_rn(~sel_word(R, q)) <= __fmaf_rn(t32, w[q], -0.5f);
+            fl |= cnd ? (1u << q) : 0u;
           }
-          // append in (lane, q) order: prefix of the per-lane counts by bit ballots
+          // append in (lane, q) order -- position order -- with the prefix of
+          // the per-lane counts from bit ballots
           const int n = __popc(fl);
           const unsigned b0 = __ballot_sync(0xffffffffu, n & 1), b1 = __ballot_sync(0xffffffffu, n & 2),
                          b2 = __ballot_sync(0xffffffffu, n & 4);
@@ -754,7 +766,11 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
 #pragma unroll
             for (int q = 0; q < 4; ++q)
               if (fl & (1u << q)) {
-                if (o < AB_CAP) pos[o] = (uint32_t)(i0 + q);
+                if (o < AB_CAP) {
+                  pos[o] = (uint32_t)(i0 + q);
+                  rnd[o] = sel_word(R, q);
+                  cw[o] = w[q];
+                }
                 ++o;
               }
             M += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2);
@@ -773,11 +789,8 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
           kk[t] = INFINITY;
           pp[t] = 0xFFFFFFFFu;
           if (32 * t < M && j < M) {
-            const uint32_t p = pos[j];
-            const U4 R = philox((uint32_t)vc, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.core.key);
-            const float wj = wc ? __ldg(wc + p) : 1.0f;
-            kk[t] = ares_key(sel_word(R, (int)(p & 3)), (double)wj);
-            pp[t] = p;
+            kk[t] = ares_key(rnd[j], (double)cw[j]);
+            pp[t] = pos[j];
             below += (tau < 0.0f || kk[t] < (double)tau) ? 1 : 0;
           }
         }
@@ -794,50 +807,67 @@ __global__ void __launch_bounds__(AB_THREADS, 4) hop_ares_big_kernel(HopParams P
         if (lane == 0) atomicOr(P.core.err, ERR_INTERNAL);
         continue;
       }
-      uint32_t mine = 0xFFFFFFFFu;
-      if (M <= 32) {
-        // one candidate per lane: bitonic sort of (key, position) across the
-        // warp; lanes 0 .. want-1 then hold the want smallest
-        double K = kk[0];
-        uint32_t Q = pp[0];
-#pragma unroll
-        for (int size = 2; size <= 32; size <<= 1) {
-#pragma unroll
-          for (int stride = size >> 1; stride > 0; stride >>= 1) {
-            const double ok = __shfl_xor_sync(0xffffffffu, K, stride);
-            const uint32_t oq = __shfl_xor_sync(0xffffffffu, Q, stride);
-            const bool asc = (lane & size) == 0 || size == 32;
-            const bool low = (lane & stride) == 0;
-            const bool ol = key_less(ok, oq, K, Q);
-            if (low == asc ? ol : (!ol && !(ok == K && oq == Q))) { K = ok; Q = oq; }
-          }
+      uint32_t mine = 0xFFFFFFFFu;  // a winner's position
+      int o = 0;                     // its rank in position order
+      bool sel = false;
+      if (M <= 20) {
+        // rank of each candidate by (key, position) against all M; the pool
+        // is in position order, so the winners' order is their lane order
+        const double K = kk[0];
+        const uint32_t Q = pp[0];
+        int r = 0;
+        for (int i = 0; i < M; ++i) {
+          const double ok = __shfl_sync(0xffffffffu, K, i);
+          const uint32_t oq = __shfl_sync(0xffffffffu, Q, i);
+          r += key_less(ok, oq, K, Q) ? 1 : 0;
         }
-        if (lane < want) mine = Q;
+        sel = lane < M && r < want;
+        o = __popc(__ballot_sync(0xffffffffu, sel) & lt);
+        mine = Q;
       } else {
-        // want rounds of a warp argmin over (key, position)
-        for (int r = 0; r < want; ++r) {
-          double bk = INFINITY;
-          uint32_t bp = 0xFFFFFFFFu;
+        if (M <= 32) {
+          // one candidate per lane: bitonic sort of (key, position) across
+          // the warp; lanes 0 .. want-1 then hold the want smallest
+          double K = kk[0];
+          uint32_t Q = pp[0];
 #pragma unroll
-          for (int t = 0; t < 4; ++t)
-            if (key_less(kk[t], pp[t], bk, bp)) { bk = kk[t]; bp = pp[t]; }
+          for (int size = 2; size <= 32; size <<= 1) {
 #pragma unroll
-          for (int o = 16; o > 0; o >>= 1) {
-            const double ok = __shfl_xor_sync(0xffffffffu, bk, o);
-            const uint32_t op = __shfl_xor_sync(0xffffffffu, bp, o);
-            if (key_less(ok, op, bk, bp)) { bk = ok; bp = op; }
+            for (int stride = size >> 1; stride > 0; stride >>= 1) {
+              const double ok = __shfl_xor_sync(0xffffffffu, K, stride);
+              const uint32_t oq = __shfl_xor_sync(0xffffffffu, Q, stride);
+              const bool asc = (lane & size) == 0 || size == 32;
+              const bool low = (lane & stride) == 0;
+              const bool ol = key_less(ok, oq, K, Q);
+              if (low == asc ? ol : (!ol && !(ok == K && oq == Q))) { K = ok; Q = oq; }
+            }
           }
+          if (lane < want) mine = Q;
+        } else {
+          // want rounds of a warp argmin over (key, position)
+          for (int r = 0; r < want; ++r) {
+            double bk = INFINITY;
+            uint32_t bp = 0xFFFFFFFFu;
 #pragma unroll
-          for (int t = 0; t < 4; ++t)
-            if (pp[t] == bp) { kk[t] = INFINITY; pp[t] = 0xFFFFFFFFu; }
-          if (lane == r) mine = bp;
+            for (int t = 0; t < 4; ++t)
+              if (key_less(kk[t], pp[t], bk, bp)) { bk = kk[t]; bp = pp[t]; }
+#pragma unroll
+            for (int o2 = 16; o2 > 0; o2 >>= 1) {
+              const double ok = __shfl_xor_sync(0xffffffffu, bk, o2);
+              const uint32_t op = __shfl_xor_sync(0xffffffffu, bp, o2);
+              if (key_less(ok, op, bk, bp)) { bk = ok; bp = op; }
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+              if (pp[t] == bp) { kk[t] = INFINITY; pp[t] = 0xFFFFFFFFu; }
+            if (lane == r) mine = bp;
+          }
         }
+        for (int s2 = 0; s2 < want; ++s2) o += __shfl_sync(0xffffffffu, mine, s2) < mine ? 1 : 0;
+        sel = lane < want;
       }
-      // the winners in position order, gathered and written out
-      int o = 0;
-      for (int s2 = 0; s2 < want; ++s2) o += __shfl_sync(0xffffffffu, mine, s2) < mine ? 1 : 0;
-      if (lane < want) {
-        const int64_t ce = __ldcg(P.indptr_out[l] + cb + b + jb + cc);  // the column's first edge
+      // the winners, gathered and written out in position order
+      if (sel) {
         const int64_t e = oc + mine;
         const uint32_t u = (uint32_t)ldg_h(P.core.indices + e, pf);
         sth(P.eid[l] + rb + ce + o, (int64_t)e, pf);
@@ -1061,6 +1091,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.core.replace = replace;
   P.core.bias = bias;
   P.core.key = key;
+  P.pk = philox_keys(key);
   const bool weighted = !replace && bias != GS_W_UNIFORM;
   P.poscnt = weighted && g->weights ? g->poscnt : nullptr;
   if (weighted && g->weights && !g->poscnt)
