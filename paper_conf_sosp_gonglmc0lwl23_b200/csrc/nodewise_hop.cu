@@ -422,12 +422,22 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
           if (!wts || __ldg(wts + off + i) > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
       }
       HWarpA& A = reinterpret_cast<HWarpA*>(&sm + 1)[warp];
-      // k < d <= 64: four columns at a time, eight lanes each; every eligible
-      // edge's exact key is held in registers (lane s: positions 32 t + 4 s + q)
-      // and the want = min(k, eligible) smallest (key, position) pairs are
-      // taken by want rounds of a group argmin
+      // k < d <= 64: four columns at a time, eight lanes each (lane s holds
+      // positions 32 t + 4 s + q).  Candidates x <= tau w (1 + 1%), tau =
+      // (k + 8) / W, get exact fp64 keys; a group with fewer than want keys
+      // below tau retakes every eligible edge.  The candidates are listed in
+      // position order in shared memory (the idle staging area), each is
+      // ranked by (key, position) against its group's list, and the want
+      // winners are written in list order = position order.
+      static_assert(sizeof(C.se) >= 4 * 64 * 12 && sizeof(C.su) >= 4 * 64 * 5 && sizeof(C.sv) >= 4 * 64 * 4,
+                    "group lists");
       uint32_t sml = __ballot_sync(0xffffffffu, d > k && d <= 64);
       const int g8 = lane >> 3, s8 = lane & 7;
+      double* gkey = reinterpret_cast<double*>(C.se) + g8 * 64;
+      uint32_t* gpos = reinterpret_cast<uint32_t*>(reinterpret_cast<double*>(C.se) + 4 * 64) + g8 * 64;
+      uint32_t* grnd = reinterpret_cast<uint32_t*>(C.su) + g8 * 64;
+      uint8_t* gwin = reinterpret_cast<uint8_t*>(reinterpret_cast<uint32_t*>(C.su) + 4 * 64) + g8 * 64;
+      float* gw = reinterpret_cast<float*>(C.sv) + g8 * 64;
       while (sml) {
         int cc = -1;
 #pragma unroll
@@ -443,68 +453,94 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
         const int64_t oc = __shfl_sync(0xffffffffu, off, src);
         const int dsrc = __shfl_sync(0xffffffffu, (int)d, src);
         const int dc = cc < 0 ? 0 : dsrc;
-        double kk[8];
+        const float W = dc > 0 ? (wts ? __ldg(P.core.colsum + vc) : (float)dc) : 0.0f;
+        uint32_t rw[8];
+        float w8[8];
         int elig = 0;
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
           const int i0 = 32 * t + 4 * s8;
           U4 R{0u, 0u, 0u, 0u};
-          if (i0 < dc) R = philox_nl((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.core.key);
+          if (i0 < dc) R = philox_k((uint32_t)vc, (uint32_t)(i0 >> 2), ctr2(l, TAG_ARES_NODE), gb, P.pk);
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
-            const float w = i0 + q < dc ? (wts ? __ldg(wts + oc + i0 + q) : 1.0f) : 0.0f;
-            kk[4 * t + q] = w > 0.0f ? ares_key_nl(sel_word(R, q), (double)w) : INFINITY;
-            elig += w > 0.0f ? 1 : 0;
+            w8[4 * t + q] = i0 + q < dc ? (wts ? __ldg(wts + oc + i0 + q) : 1.0f) : 0.0f;
+            rw[4 * t + q] = sel_word(R, q);
+            elig += w8[4 * t + q] > 0.0f ? 1 : 0;
           }
         }
         elig += __shfl_xor_sync(0xffffffffu, elig, 4);
         elig += __shfl_xor_sync(0xffffffffu, elig, 2);
         elig += __shfl_xor_sync(0xffffffffu, elig, 1);
         const int want = min(k, elig);
-        int rounds = want;
-        rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, 8));
-        rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, 16));
-        for (int r = 0; r < rounds; ++r) {
-          double bk = INFINITY;
-          uint32_t bp = 0xFFFFFFFFu;
+        float tau = W > 0.0f ? (float)(k + 8) / W : -1.0f;
+        if (P.ares_tau == 1) tau *= 0.25f;
+        int M = 0;
+        for (int pass = 0; pass < 2; ++pass) {
+          // candidates (no logarithm yet), listed in position order (t, lane, q)
+          const float t32 = __fmul_rn(__fmul_rn(tau, 1.01f), 4294967296.0f);
+          unsigned cm = 0u;
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
-            const uint32_t pj = (uint32_t)(32 * (j >> 2) + 4 * s8 + (j & 3));
-            if (key_less(kk[j], pj, bk, bp)) { bk = kk[j]; bp = pj; }
+            const bool cnd = w8[j] > 0.0f && (tau < 0.0f || __uint2float_rn(~rw[j]) <= __fmaf_rn(t32, w8[j], -0.5f));
+            cm |= cnd ? (1u << j) : 0u;
           }
+          __syncwarp();
+          M = 0;
 #pragma unroll
-          for (int o = 4; o > 0; o >>= 1) {
-            const double ok = __shfl_xor_sync(0xffffffffu, bk, o);
-            const uint32_t op = __shfl_xor_sync(0xffffffffu, bp, o);
-            if (key_less(ok, op, bk, bp)) { bk = ok; bp = op; }
-          }
-          if (r < want) {
+          for (int t = 0; t < 2; ++t) {
+            const int c = __popc((cm >> (4 * t)) & 0xFu);
+            int x = c;
 #pragma unroll
-            for (int j = 0; j < 8; ++j)
-              if ((uint32_t)(32 * (j >> 2) + 4 * s8 + (j & 3)) == bp) kk[j] = INFINITY;
-            if (s8 == 0) C.list[r][cc] = bp;
+            for (int o = 1; o < 8; o <<= 1) {
+              const int y = __shfl_up_sync(0xffffffffu, x, o, 8);
+              if (s8 >= o) x += y;
+            }
+            int o = M + x - c;
+            M += __shfl_sync(0xffffffffu, x, 7, 8);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int j = 4 * t + q;
+              if (cm & (1u << j)) {
+                gpos[o] = (uint32_t)(32 * t + 4 * s8 + q);
+                grnd[o] = rw[j];
+                gw[o] = w8[j];
+                ++o;
+              }
+            }
           }
+          __syncwarp();
+          // exact keys of the listed candidates, eight lanes per group
+          int below = 0;
+          for (int e = s8; e < M; e += 8) {
+            const double ke = ares_key_nl(grnd[e], (double)gw[e]);
+            gkey[e] = ke;
+            below += (tau < 0.0f || ke < (double)tau) ? 1 : 0;
+          }
+          below += __shfl_xor_sync(0xffffffffu, below, 4);
+          below += __shfl_xor_sync(0xffffffffu, below, 2);
+          below += __shfl_xor_sync(0xffffffffu, below, 1);
+          const bool redo = below < want;
+          if (!__any_sync(0xffffffffu, redo)) break;
+          if (redo) tau = -1.0f;  // every eligible edge (the others recompute the same)
         }
         __syncwarp();
-        // the want winners of column cc in ascending position order
-        uint32_t wp[(KCAP + 7) / 8];
-#pragma unroll
-        for (int t = 0; t < (KCAP + 7) / 8; ++t) {
-          const int j = s8 + 8 * t;
-          wp[t] = j < want ? C.list[j][src] : 0xFFFFFFFFu;
-        }
-        int rk8[(KCAP + 7) / 8];
-#pragma unroll
-        for (int t = 0; t < (KCAP + 7) / 8; ++t) rk8[t] = 0;
-        for (int i = 0; i < want; ++i) {
-          const uint32_t pi = C.list[i][src];
-#pragma unroll
-          for (int t = 0; t < (KCAP + 7) / 8; ++t) rk8[t] += pi < wp[t] ? 1 : 0;
+        // rank the list entries s, s + 8, ... of the group against all M
+        for (int e = s8; e < M; e += 8) {
+          const double ke = gkey[e];
+          const uint32_t pe = gpos[e];
+          int r = 0;
+          for (int i = 0; i < M; ++i) r += key_less(gkey[i], gpos[i], ke, pe) ? 1 : 0;
+          gwin[e] = r < want ? 1 : 0;
         }
         __syncwarp();
-#pragma unroll
-        for (int t = 0; t < (KCAP + 7) / 8; ++t)
-          if (s8 + 8 * t < want) C.list[rk8[t]][cc] = wp[t];
+        for (int e = s8; e < M; e += 8) {
+          if (gwin[e]) {
+            int o = 0;
+            for (int i = 0; i < e; ++i) o += gwin[i];
+            C.list[o][cc] = gpos[e];
+          }
+        }
         if (cc >= 0 && s8 == 0) A.rk[cc] = want;
         __syncwarp();
       }
