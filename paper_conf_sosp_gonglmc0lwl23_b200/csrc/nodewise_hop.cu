@@ -417,9 +417,13 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
       // columns one at a time by the whole warp (candidate filtering)
       const float* wts = P.core.weights;
       if (d > 0 && P.core.bias == GS_W_PASS_COLNORM) csum = wts ? __ldg(P.core.colsum + v) : (float)d;
-      if (d <= k) {
-        for (int i = 0; i < (int)d; ++i)
-          if (!wts || __ldg(wts + off + i) > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
+      if (d <= k) {  // the d weights loaded at once (unrolled), then the eligible ones listed
+        float wl[KCAP];
+#pragma unroll
+        for (int i = 0; i < KCAP; ++i) wl[i] = i < d ? (wts ? __ldg(wts + off + i) : 1.0f) : 0.0f;
+#pragma unroll
+        for (int i = 0; i < KCAP; ++i)
+          if (wl[i] > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
       }
       HWarpA& A = reinterpret_cast<HWarpA*>(&sm + 1)[warp];
       // k < d <= 64: four columns at a time, eight lanes each (lane s holds
