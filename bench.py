@@ -697,12 +697,17 @@ def run_gpu(args, wl, world, rank, device):
     achieved = bytes_per_launch / (statistics.mean(times) / 1000.0) / 1e9
     line_bytes = (model_bytes + 96 * rnd_secs) / args.steps  # random 32-B sectors as 128-B lines
     line_achieved = line_bytes / (statistics.mean(times) / 1000.0) / 1e9
-    sel_ms = sum(v for k, v in kernel_ms.items() if k.startswith("hop_select"))
+    # the Extract+Select stage: hop_select (+ hop_ares_big, which takes the
+    # weighted heavy columns' filter, select and gather off it)
+    sel_ms = sum(v for k, v in kernel_ms.items() if k.startswith("hop_select") or k.startswith("hop_ares"))
+    has_ares = any(k.startswith("hop_ares") for k in kernel_ms)
     dom = None
     if sel_ms > 0:
         prof_total = sum(kernel_ms.values())
-        dom = {"kernel": "gsb::hop_select_kernel (every hop; Extract+Select+gather: frontier ids, sampled "
-                         "sectors, eid + row id written)",
+        dom = {"kernel": ("gsb::hop_select_kernel + gsb::hop_ares_big_kernel" if has_ares else
+                          "gsb::hop_select_kernel") +
+                         " (every hop; Extract+Select+gather: frontier ids, sampled sectors"
+                         + (", weights streamed" if has_ares else "") + ", eid + row id written)",
                "bytes_per_step": sel_bytes / args.steps, "ms_per_step": sel_ms,
                "achieved": sel_bytes / args.steps / (sel_ms / 1000.0) / 1e9,
                "share_of_step": sel_ms / prof_total if prof_total > 0 else None,
