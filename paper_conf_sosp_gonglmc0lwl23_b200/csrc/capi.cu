@@ -633,6 +633,7 @@ gs_status gs_blocks_sync(gs_blocks* b) {
       for (int l = 0; l < b->num_layers; ++l)
         b->lw_edge_hint[l] = std::max<int64_t>(b->lw_edge_hint[l], (int64_t)(ctr[l] + ctr[l] / 4 + 1024));
       b->lw_tab_hint = std::max<int64_t>(b->lw_tab_hint, (int64_t)ctr[MAX_LAYERS]);
+      if (ctr[MAX_LAYERS + 1]) b->lw_big = true;  // re-run on the global-table kernel
     }
     return fail(GS_ERR_CAPACITY,
                 "a device-side capacity was exceeded; call again with this gs_blocks (it has grown)");

@@ -97,6 +97,7 @@ struct gs_blocks {
   int ws_kind_prev = 0;        // workspace layout tag of the previous launch (per kernel family)
   int64_t lw_edge_hint[gsb::MAX_LAYERS] = {};  // layer-wise edge capacity learnt from an overflow
   int64_t lw_tab_hint = 0;     // layer-wise per-CTA table size learnt from an overflow
+  bool lw_big = false;         // a batch-layer outgrew the shared-memory layer-wise kernel
   bool synced = false;
   gs_blocks* aux = nullptr;    // ShaDow: the internal node-wise result
   int64_t num_seeds = 0, batch_size = 0;  // node-wise: the seeds and (fixed) batch size sampled

@@ -508,10 +508,9 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
 // when the candidate bitmaps of one CTA per SM fit (N/8 bytes each, <= 2 GB
 // in all) and its rank prefixes fit shared memory -- hub-biased frontiers give
 // ~280 k candidates per batch-layer (measured on LJ: 282 ms vs 514 ms).
-// LADIES / COUNT (~10 k candidates): the global hash-table kernel below (31 ms
-// vs 69 ms for the bitmap kernel: four dense bitmap scans per batch-layer cost
-// more than the table; the shared-memory kernel of layerwise_sm.cu, 30-53 ms,
-// on request).
+// LADIES / COUNT (~10 k candidates) with K and batch size <= 1024: the
+// shared-memory kernel of layerwise_sm.cu; larger: the global hash-table
+// kernel below (31 ms vs 69 ms for the bitmap kernel on LJ).
 // GS_LW_PATH=old|bm forces one (experiments / tests).
 gs_status run_layerwise_sm(const gs_graph* g, const int32_t* seeds, int64_t num_seeds, int64_t batch_size,
                            int64_t batch_base, const int32_t* n_per_layer, int L, int prob_mode, uint64_t key,
@@ -521,16 +520,14 @@ gs_status run_layerwise(const gs_graph* g, const int32_t* seeds, int64_t num_see
                         int64_t batch_size, int64_t batch_base, const int32_t* n_per_layer,
                         int L, int prob_mode, uint64_t key, cudaStream_t stream, gs_blocks* blk) {
   {
-    // LADIES / COUNT with frontiers and K <= 512: every per-batch table in
-    // shared memory (layerwise_sm.cu), on request
+    // LADIES / COUNT with frontiers and K <= 1024: every per-batch table in
+    // shared memory, the extracted edges in registers (layerwise_sm.cu)
     int maxK0 = 1;
     for (int l = 0; l < L; ++l) maxK0 = std::max(maxK0, n_per_layer[l]);
     const char* path0 = getenv("GS_LW_PATH");
-    // measured (LJ, 512 x 3): 30-53 ms vs the global-table kernel's 31 ms --
-    // per-batch-layer phases are barrier- and latency-bound; kept as an option
-    // (GS_LW_PATH=sm) until it wins
-    const bool sm_ok = prob_mode != GS_PROB_DEGREE && maxK0 <= 512 && batch_size <= 512;
-    if (sm_ok && path0 && !strcmp(path0, "sm"))
+    const bool sm_ok = prob_mode != GS_PROB_DEGREE && maxK0 <= 1024 && batch_size <= 1024 && !blk->lw_big;
+    const bool forced_other = path0 && (!strcmp(path0, "old") || !strcmp(path0, "bm"));
+    if (sm_ok && !forced_other)
       return run_layerwise_sm(g, seeds, num_seeds, batch_size, batch_base, n_per_layer, L, prob_mode, key,
                               stream, blk);
   }

@@ -134,3 +134,41 @@ def test_fastgcn_emit_restream(gs, oracle_lib, ljlike, monkeypatch, lw_path):
         ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [512, 512], batch_size=512, prob_mode=mode,
                                           rng_key=5)
         compare_all(out.to_host(), ref, f"restream emit mode {mode}")
+
+
+def test_sm_big_frontier(gs, oracle_lib, ljlike, lw_path):
+    """Shared-memory kernel (layerwise_sm.cu) with 1024-column frontiers and
+    K = 1024: batch-layers of more than one register chunk (re-streamed per
+    pass) and several hash partitions, besides the one-chunk / one-partition
+    common case."""
+    if lw_path != "sm":
+        pytest.skip("shared-memory kernel path")
+    cfg = "1024x12"
+    g, G, O = ljlike
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 21), 1024 * 5 + 300)
+    for mode in (0, 2):
+        out = gs.sample_layerwise(G, seeds.cuda(), [1024, 1024], batch_size=1024, prob_mode=mode,
+                                  rng_key=77)
+        ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [1024, 1024], batch_size=1024,
+                                          prob_mode=mode, rng_key=77)
+        compare_all(out.to_host(), ref, f"sm cfg {cfg} mode {mode}")
+
+
+@pytest.fixture(scope="module")
+def hubby(gs, oracle_lib):
+    # undirected power-law graph: LADIES frontiers pick hubs, so the later
+    # layers extract tens of thousands of edges per batch (many chunks and
+    # partitions in the shared-memory kernel)
+    g = synth.small_graph(100_000, 3_000_000, undirected=True, weights="gcn", seed=23, device="cuda")
+    return g, gs.Graph(g["indptr"], g["indices"], g["weights"]), oracle_lib.Graph(*host_graph(g))
+
+
+def test_ladies_hub_frontiers(gs, oracle_lib, hubby, lw_path):
+    if lw_path == "bm":
+        pytest.skip("LADIES on the bitmap kernel is covered above")
+    g, G, O = hubby
+    seeds = synth.make_seeds(synth.GraphSpec("pd", 100_000, 1, True, None, 5), 512 * 4 + 17)
+    out = gs.sample_layerwise(G, seeds.cuda(), [512, 256, 512], batch_size=512, prob_mode=0, rng_key=8)
+    ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [512, 256, 512], batch_size=512, prob_mode=0,
+                                      rng_key=8)
+    compare_all(out.to_host(), ref, "ladies hub frontiers")
