@@ -64,8 +64,9 @@ struct gs_graph {
   int sorted = 0;
   int64_t max_in_degree = 0;
   gsb::Allocator al;
-  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_poscnt, b_err, b_deg;
+  gsb::DevBuf b_indptr, b_indices, b_weights, b_colsum, b_poscnt, b_err, b_deg, b_degsrc;
   int32_t* deg = nullptr;    // FastGCN a0 pre-processing: in-degree per node (built on first use)
+  int32_t* degsrc = nullptr; // FastGCN a0: in-degree of every CSC entry's row (deg[indices[e]]), if it fits
   gsb::DevBuf b_walk;        // walk index (walk.cu): 16 B per CSC entry, built on the first walk
   const int4* walk_rec = nullptr;
   bool walk_index_failed = false;

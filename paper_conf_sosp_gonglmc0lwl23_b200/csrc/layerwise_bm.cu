@@ -49,6 +49,7 @@ constexpr int LB_WARPS = LB_THREADS / 32;
 constexpr int LB_CAP = 4096;        // A-Res candidate buffer (select), >= max K
 constexpr int LB_HS = 8192;         // hash of S (aliases the candidate buffer)
 constexpr int LB_ILP = 4;           // flat edges per thread in flight
+constexpr int LB_ILP5 = 8;          // ... in the finalize re-stream (L5a)
 constexpr int LB_MAX_K = 4096;
 constexpr int LB_SCAP = 512;        // kept edges a warp stages in L5a (more: L5b streams again)
 
@@ -57,6 +58,7 @@ struct LBParams {
   const int32_t* indices;
   const float* weights;
   const int32_t* deg;               // a0: in-degree per node (FastGCN)
+  const int32_t* degsrc;            // a0: deg[indices[e]] per CSC entry (FastGCN), or null
   int64_t N;
   const int32_t* seeds;
   int64_t num_seeds, batch_size, num_batches, batch_base;
@@ -64,6 +66,7 @@ struct LBParams {
   int K[MAX_LAYERS];
   int mode;
   uint64_t key;
+  PhiloxKeys pk;
   int32_t* col0;
   int32_t* row_map[MAX_LAYERS];
   float* row_prob[MAX_LAYERS];
@@ -203,43 +206,69 @@ __device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, i
   const int g_beg = min(warp * gpw, P.ng), g_end = min((warp + 1) * gpw, P.ng);
   const int64_t i_beg = (int64_t)g_beg * gq, i_end = (int64_t)g_end * gq;
   int run = 0;
-  double bsum = 0.0;
+  long long bsum = 0;  // B = sum of integer in-degrees (exact; = the oracle's fp64 sum)
   int elig = 0;
+  const float tau_f = (float)tau_est;
   for (int64_t i0 = i_beg; i0 < i_end; i0 += 32) {
     const int64_t i = i0 + lane;
     const uint4 x = i < i_end ? __ldcg(bm4 + i) : make_uint4(0, 0, 0, 0);
     const int pc = popc4(x);
     const int inc = warp_inclusive_scan(pc);
     if (i < i_end && (lane & (gq - 1)) == 0) s_gp[i >> (P.gw_log - 2)] = run + inc - pc;
-    run += __shfl_sync(0xffffffffu, inc, 31);
-    if (degree && pc) {
+    const int total = __shfl_sync(0xffffffffu, inc, 31);
+    run += total;
+    if (!degree) continue;
+    // the warp's candidates, 32 at a time across the lanes (balanced: no lane
+    // walks its own bits while the others wait): candidate k -> its owner lane
+    // (binary search of the inclusive scan) and bit (fns)
+    auto locate = [&](int k) -> uint32_t {  // the warp's k-th candidate (all lanes call)
+      int o = 0;
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        uint32_t w = word4(x, j);
-        while (w) {
-          const int bpos = __ffs(w) - 1;
-          w &= w - 1u;
-          const uint32_t u = (uint32_t)((i * 4 + j) * 32 + bpos);
-          const int32_t dg = __ldg(P.deg + u);
-          bsum += (double)(float)dg;
-          elig += dg > 0 ? 1 : 0;
-          if (tau_est > 0.0 && dg > 0) {
-            const float bb = (float)dg;
-            const U4 R = philox(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.key);
-            if (ares_maybe_below(R.x, (float)(tau_est * (double)bb) * 1.01f)) {
-              const double kk = ares_key(R.x, (double)bb);
-              if (kk < tau_est) {
-                const int slot = atomicAdd(&sh.misc[6], 1);
-                if (slot < LB_CAP) {
-                  buf.k[slot] = (unsigned long long)__double_as_longlong(kk);
-                  buf.u[slot] = u;
-                  buf.b[slot] = bb;
-                }
-              }
+      for (int step = 16; step > 0; step >>= 1) {
+        const int ip = __shfl_sync(0xffffffffu, inc, o + step - 1);
+        if (ip <= k) o += step;
+      }
+      const uint32_t w0 = __shfl_sync(0xffffffffu, x.x, o), w1 = __shfl_sync(0xffffffffu, x.y, o);
+      const uint32_t w2 = __shfl_sync(0xffffffffu, x.z, o), w3 = __shfl_sync(0xffffffffu, x.w, o);
+      const int ex_o = __shfl_sync(0xffffffffu, inc - pc, o);
+      if (k >= total) return 0xFFFFFFFFu;
+      int r = k - ex_o;
+      int j = 0;
+      uint32_t wd = w0;
+      const int p0 = __popc(w0), p1 = __popc(w1), p2 = __popc(w2);
+      if (r >= p0) { r -= p0; j = 1; wd = w1;
+        if (r >= p1) { r -= p1; j = 2; wd = w2;
+          if (r >= p2) { r -= p2; j = 3; wd = w3; } } }
+      uint32_t bpos;
+      asm("fns.b32 %0, %1, 0, %2;" : "=r"(bpos) : "r"(wd), "r"(r + 1));
+      return (uint32_t)(((i0 + o) * 4 + j) * 32 + bpos);
+    };
+    auto take = [&](uint32_t u, int32_t dg) {
+      bsum += dg;
+      elig += dg > 0 ? 1 : 0;
+      if (tau_est > 0.0 && dg > 0) {
+        const float bb = (float)dg;
+        const uint32_t R = philox_k(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.pk).x;
+        if (ares_maybe_below(R, __fmul_rn(__fmul_rn(tau_f, bb), 1.01f))) {
+          const double kk = ares_key(R, (double)bb);
+          if (kk < tau_est) {
+            const int slot = atomicAdd(&sh.misc[6], 1);
+            if (slot < LB_CAP) {
+              buf.k[slot] = (unsigned long long)__double_as_longlong(kk);
+              buf.u[slot] = u;
+              buf.b[slot] = bb;
             }
           }
         }
       }
+    };
+    // two candidates per lane in flight (their degree loads overlap)
+    for (int k0 = 0; k0 < total; k0 += 64) {
+      const uint32_t ua = locate(k0 + lane), ub = locate(k0 + 32 + lane);
+      const int32_t da = ua != 0xFFFFFFFFu ? __ldg(P.deg + ua) : 0;
+      const int32_t db = ub != 0xFFFFFFFFu ? __ldg(P.deg + ub) : 0;
+      if (ua != 0xFFFFFFFFu) take(ua, da);
+      if (ub != 0xFFFFFFFFu) take(ub, db);
     }
   }
   if (lane == 0) sh.wtot[warp] = run;
@@ -256,7 +285,7 @@ __device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, i
   if (warp == 0 && lane == 0) s_gp[P.ng] = sh.misc[5];
   const int64_t total = sh.misc[5];
   if (degree) {
-    *B_out = block_reduce_sum(bsum, sh.dred);
+    *B_out = (double)block_reduce_sum((unsigned long long)bsum, sh.scan);
     *nelig_out = (int64_t)block_reduce_sum((double)elig, sh.dred);
   } else {
     __syncthreads();
@@ -264,27 +293,50 @@ __device__ int64_t lb_ranks(const LBParams& P, LBShared& sh, const uint4* bm4, i
   return total;
 }
 
-// Bitonic sort of n2 (power of two) 64-bit keys with a 32-bit payload,
-// ascending by (key, payload).
-__device__ void lb_sort_kv(unsigned long long* k, uint32_t* v, float* b, int n2) {
-  for (int kk = 2; kk <= n2; kk <<= 1) {
-    for (int jj = kk >> 1; jj > 0; jj >>= 1) {
-      for (int i = threadIdx.x; i < n2; i += blockDim.x) {
-        const int ixj = i ^ jj;
-        if (ixj > i) {
-          const unsigned long long ka = k[i], kc = k[ixj];
-          const uint32_t va = v[i], vc = v[ixj];
-          const bool gt = ka > kc || (ka == kc && va > vc);
-          if (gt == ((i & kk) == 0)) {
-            k[i] = kc; k[ixj] = ka;
-            v[i] = vc; v[ixj] = va;
-            if (b) { const float t = b[i]; b[i] = b[ixj]; b[ixj] = t; }
-          }
-        }
-      }
-      __syncthreads();
+__device__ __forceinline__ double block_reduce_max(double v, double* scratch) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  if (lane == 0) scratch[wid] = v;
+  __syncthreads();
+  double r = 0.0;
+  for (int w = 0; w < nw; ++w) r = fmax(r, scratch[w]);
+  __syncthreads();
+  return r;
+}
+
+// Counting-sort rank of n <= LB_CAP items on LB_THREADS bins (bin(i) monotone
+// in the order; less(j, i) the exact order inside a bin): rank[i] for every
+// item with take(i).  Every thread of the CTA calls it.
+template <class Bin, class Less, class Take>
+__device__ __forceinline__ void lb_csrank(int n, int* hist, int* fill, int16_t* ord, int16_t* rank, Bin bin,
+                                          Less less, Take take, unsigned long long* scan) {
+  const int t = threadIdx.x;
+  hist[t] = 0;
+  fill[t] = 0;
+  __syncthreads();
+  for (int i = t; i < n; i += LB_THREADS)
+    if (take(i)) atomicAdd(&hist[bin(i)], 1);
+  __syncthreads();
+  unsigned long long tot;
+  const int c = hist[t];
+  const int st = (int)block_exclusive_scan<unsigned long long>((unsigned long long)c, scan, &tot);
+  hist[t] = st;
+  __syncthreads();
+  for (int i = t; i < n; i += LB_THREADS)
+    if (take(i)) {
+      const int bb = bin(i);
+      ord[hist[bb] + atomicAdd(&fill[bb], 1)] = (int16_t)i;
     }
-  }
+  __syncthreads();
+  for (int i = t; i < n; i += LB_THREADS)
+    if (take(i)) {
+      const int bb = bin(i), s0 = hist[bb], s1 = s0 + fill[bb];
+      int r = s0;
+      for (int k = s0; k < s1; ++k) r += less(ord[k], i) ? 1 : 0;
+      rank[i] = (int16_t)r;
+    }
+  __syncthreads();
 }
 
 __device__ __forceinline__ uint32_t lb_hash(uint32_t u) { return (u * 0x9E3779B1u) >> 19; }  // 13 bits
@@ -366,39 +418,92 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       const int Ti = (int)T;
       const int64_t nflat = T > 0 ? (int64_t)sh.u64[1] : 0;
 
-      // ---- L1: Extract, the rows' bits (one red.or per distinct row per warp round) ----
+      // ---- L1: Extract, the rows' bits (one red.or per distinct row per warp
+      // round).  FastGCN with the a0 per-entry degrees: b(u) travels with u, so
+      // the edge that sets a row's bit also adds b(u) to B, counts it eligible
+      // and runs the fused A-Res filter against the previous batch's threshold
+      // (no per-candidate degree lookups, no pass over the bitmap) ----
+      const double tau_est = degree ? sh.tau_est[l] : 0.0;
+      const float tau_f = (float)tau_est;
+      const bool l1_deg = degree && P.degsrc != nullptr;
+      unsigned long long l1_b = 0, l1_e = 0;
+      if (threadIdx.x == 0) sh.misc[6] = 0;
+      __syncthreads();
       {
         LBStream st(nflat);
         for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
           uint32_t u[LB_ILP];
+          int32_t dg[LB_ILP];
 #pragma unroll
           for (int q = 0; q < LB_ILP; ++q) {
             const int64_t e = e0 + 32 * q + lane;
             u[q] = 0xFFFFFFFFu;
+            dg[q] = 0;
             if (e < st.end) {
               const int c = st.col(s_fstart, Ti, e);
-              u[q] = (uint32_t)__ldg(P.indices + s_off[c] + (e - s_fstart[c]));
+              const int64_t pos = s_off[c] + (e - s_fstart[c]);
+              u[q] = (uint32_t)__ldg(P.indices + pos);
+              if (l1_deg) dg[q] = __ldg(P.degsrc + pos);
             }
           }
 #pragma unroll
           for (int q = 0; q < LB_ILP; ++q) {
             const uint32_t peers = __match_any_sync(0xffffffffu, u[q]);
-            if (u[q] != 0xFFFFFFFFu && (__ffs(peers) - 1) == lane)
-              atomicOr(bm + (u[q] >> 5), 1u << (u[q] & 31));
+            if (u[q] == 0xFFFFFFFFu || (__ffs(peers) - 1) != lane) continue;
+            const uint32_t bit = 1u << (u[q] & 31);
+            if (!l1_deg) {
+              atomicOr(bm + (u[q] >> 5), bit);
+              continue;
+            }
+            if (atomicOr(bm + (u[q] >> 5), bit) & bit) continue;  // not new
+            l1_b += (unsigned long long)dg[q];
+            if (dg[q] <= 0) continue;
+            ++l1_e;
+            if (!(tau_est > 0.0)) continue;
+            const float bb = (float)dg[q];
+            const uint32_t R = philox_k(u[q], 0u, ctr2(l, TAG_ARES_LAYER), gb, P.pk).x;
+            if (!ares_maybe_below(R, __fmul_rn(__fmul_rn(tau_f, bb), 1.01f))) continue;
+            const double kk = ares_key(R, (double)bb);
+            if (!(kk < tau_est)) continue;
+            const int slot = atomicAdd(&sh.misc[6], 1);
+            if (slot < LB_CAP) {
+              s_bk[slot] = (unsigned long long)__double_as_longlong(kk);
+              s_bu[slot] = u[q];
+              s_bb[slot] = bb;
+            }
           }
         }
       }
       __syncthreads();
 
-      // ---- L2: rank groups (FastGCN: b(u) = in-degree, B, eligible) ----
+      // ---- L2: rank groups (FastGCN: b(u) = in-degree, B, eligible; skipped
+      // when L1 already holds B and a usable fused selection) ----
       double Btot = 0.0;
       int64_t nelig = 0;
-      if (threadIdx.x == 0) sh.misc[6] = 0;
-      __syncthreads();
-      const double tau_est = degree ? sh.tau_est[l] : 0.0;
-      const int64_t nc = lb_ranks(P, sh, bm4, s_gp, degree, &Btot, &nelig, tau_est, l, gb,
-                                  LBBuf{s_bk, s_bu, s_bb});
-      const int m_fused = sh.misc[6];
+      int m_fused = 0;
+      bool skip_ranks = false;
+      if (l1_deg) {
+        Btot = (double)block_reduce_sum(l1_b, sh.scan);
+        nelig = (int64_t)block_reduce_sum(l1_e, sh.scan);
+        m_fused = sh.misc[6];
+        skip_ranks = tau_est > 0.0 && m_fused >= K && m_fused <= LB_CAP && nelig > K;
+      }
+      int64_t nc = 0;
+      if (!skip_ranks) {
+        if (threadIdx.x == 0) sh.misc[6] = 0;
+        __syncthreads();
+        double Bx = 0.0;
+        int64_t nx = 0;
+        nc = lb_ranks(P, sh, bm4, s_gp, degree, &Bx, &nx, l1_deg ? 0.0 : tau_est, l, gb,
+                      LBBuf{s_bk, s_bu, s_bb});
+        if (!l1_deg) {
+          Btot = Bx;
+          nelig = nx;
+          m_fused = sh.misc[6];
+        } else {
+          m_fused = 0;  // L1's fused selection was not usable: the select filters the bitmap
+        }
+      }
       bool acc_ok = true;
       if (!degree && nc > P.acc_cap) {
         if (threadIdx.x == 0) {
@@ -453,7 +558,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       };
       if (threadIdx.x == 0) sh.misc[0] = 0;
       __syncthreads();
-      int nsel = 0;
+      int nsel = 0, ncand = 0;
       if (nelig <= K) {  // every eligible candidate (R24)
         if (nelig > 0) {
           lb_for_bits(P, bm4, s_gp, [&](uint32_t u, int64_t r) {
@@ -466,6 +571,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
           });
         }
         nsel = (int)nelig;
+        ncand = nsel;
         __syncthreads();
       } else {
         // threshold filter: keys below tau, ~2K of them (R6: exact fp64 key)
@@ -479,10 +585,10 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
           lb_for_bits(P, bm4, s_gp, [&](uint32_t u, int64_t r) {
             const float bb = bias_of(u, r);
             if (!(bb > 0.0f)) return;
-            const U4 R = philox(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.key);
+            const uint32_t R = philox_k(u, 0u, ctr2(l, TAG_ARES_LAYER), gb, P.pk).x;
             const float t = (float)(tau * (double)bb) * 1.01f;
-            if (!ares_maybe_below(R.x, t)) return;
-            const double kk = ares_key(R.x, (double)bb);
+            if (!ares_maybe_below(R, t)) return;
+            const double kk = ares_key(R, (double)bb);
             if (!(kk < tau)) return;
             const int slot = atomicAdd(&sh.misc[0], 1);
             if (slot < LB_CAP) {
@@ -503,38 +609,46 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
             m = min(m, LB_CAP);
           }
         }
-        int n2 = 1;
-        while (n2 < m) n2 <<= 1;
-        for (int i = m + threadIdx.x; i < n2; i += blockDim.x) {
-          s_bk[i] = ~0ull;
-          s_bu[i] = 0xFFFFFFFFu;
-        }
-        __syncthreads();
-        lb_sort_kv(s_bk, s_bu, s_bb, n2);  // (key, u) ascending: the K smallest first
-        nsel = min(K, m);
+        ncand = min(m, LB_CAP);
+        nsel = min(K, ncand);
         // next batch at this layer: ~3K expected candidates below the estimate
         if (degree && threadIdx.x == 0) sh.tau_est[l] = 3.0 * K / Btot;
       }
-      // S sorted by node id (R3): (u << 32 | bias bits)
-      int n2 = 1;
-      while (n2 < nsel) n2 <<= 1;
-      for (int i = threadIdx.x; i < n2; i += blockDim.x)
-        s_sel[i] = i < nsel ? (((unsigned long long)s_bu[i] << 32) | __float_as_uint(s_bb[i])) : ~0ull;
-      __syncthreads();
-      for (int kk = 2; kk <= n2; kk <<= 1) {
-        for (int jj = kk >> 1; jj > 0; jj >>= 1) {
-          for (int i = threadIdx.x; i < n2; i += blockDim.x) {
-            const int ixj = i ^ jj;
-            if (ixj > i) {
-              const unsigned long long a = s_sel[i], c = s_sel[ixj];
-              if ((a > c) == ((i & kk) == 0)) {
-                s_sel[i] = c;
-                s_sel[ixj] = a;
-              }
-            }
-          }
-          __syncthreads();
+      // the K smallest (key, u) of the candidates, then S sorted by node id
+      // (R3) as (u << 32 | bias bits): counting-sort ranks (a handful of
+      // barriers instead of bitonic networks); scratch in s_sel's region
+      {
+        int* c_hist = reinterpret_cast<int*>(s_sel);
+        int* c_fill = c_hist + LB_THREADS;
+        int16_t* c_ord = reinterpret_cast<int16_t*>(c_fill + LB_THREADS);
+        int16_t* c_rank = c_ord + LB_CAP;
+        uint8_t* c_sel = reinterpret_cast<uint8_t*>(c_rank + LB_CAP);
+        if (nsel < ncand) {
+          double km = 0.0;
+          for (int i = threadIdx.x; i < ncand; i += blockDim.x) km = fmax(km, __longlong_as_double((long long)s_bk[i]));
+          km = block_reduce_max(km, sh.dred);
+          const double scale = km > 0.0 ? (double)(LB_THREADS - 1) / km : 0.0;
+          lb_csrank(
+              ncand, c_hist, c_fill, c_ord, c_rank,
+              [&](int i) { return min(LB_THREADS - 1, (int)(__longlong_as_double((long long)s_bk[i]) * scale)); },
+              [&](int j, int i) { return s_bk[j] < s_bk[i] || (s_bk[j] == s_bk[i] && s_bu[j] < s_bu[i]); },
+              [&](int) { return true; }, sh.scan);
+          for (int i = threadIdx.x; i < ncand; i += blockDim.x) c_sel[i] = c_rank[i] < nsel ? 1 : 0;
+        } else {
+          for (int i = threadIdx.x; i < ncand; i += blockDim.x) c_sel[i] = 1;
         }
+        __syncthreads();
+        const uint64_t NN = (uint64_t)P.N;
+        lb_csrank(
+            ncand, c_hist, c_fill, c_ord, c_rank,
+            [&](int i) { return (int)(((uint64_t)s_bu[i] * LB_THREADS) / NN); },
+            [&](int j, int i) { return s_bu[j] < s_bu[i]; },
+            [&](int i) { return c_sel[i] != 0; }, sh.scan);
+        for (int i = threadIdx.x; i < ncand; i += blockDim.x)
+          if (c_sel[i]) s_bk[c_rank[i]] = ((unsigned long long)s_bu[i] << 32) | __float_as_uint(s_bb[i]);
+        __syncthreads();
+        for (int i = threadIdx.x; i < nsel; i += blockDim.x) s_sel[i] = s_bk[i];
+        __syncthreads();
       }
       // p(u) = b(u) / B (R7); hash of S for the finalize
       for (int i = threadIdx.x; i < LB_HS; i += blockDim.x) s_hk[i] = -1;
@@ -571,12 +685,12 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       __syncthreads();
       {
         LBStream st(nflat);
-        for (int64_t e0 = st.beg; e0 < st.end && nsel > 0; e0 += 32 * LB_ILP) {
-          uint32_t u[LB_ILP];
-          int c[LB_ILP];
-          int64_t pos[LB_ILP];
+        for (int64_t e0 = st.beg; e0 < st.end && nsel > 0; e0 += 32 * LB_ILP5) {
+          uint32_t u[LB_ILP5];
+          int c[LB_ILP5];
+          int64_t pos[LB_ILP5];
 #pragma unroll
-          for (int q = 0; q < LB_ILP; ++q) {
+          for (int q = 0; q < LB_ILP5; ++q) {
             const int64_t e = e0 + 32 * q + lane;
             u[q] = 0xFFFFFFFFu;
             c[q] = 0;
@@ -588,7 +702,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
             }
           }
 #pragma unroll
-          for (int q = 0; q < LB_ILP; ++q) {
+          for (int q = 0; q < LB_ILP5; ++q) {
             const int lid = u[q] == 0xFFFFFFFFu ? -1 : lb_lookup(s_hk, s_hv, u[q]);
             const unsigned bal = __ballot_sync(0xffffffffu, lid >= 0);
             if (lid >= 0) {
@@ -689,6 +803,14 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
   }
 }
 
+// a0 pre-processing ("degree of each node in FastGCN"): the row's degree
+// beside every CSC entry, so the extract stream carries b(u) with u.
+__global__ void degsrc_kernel(const int32_t* __restrict__ indices, const int32_t* __restrict__ deg, int64_t nnz,
+                              int32_t* __restrict__ out) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x)
+    out[e] = deg[indices[e]];
+}
+
 // a0 pre-processing ("degree of each node in FastGCN"): deg[u] = in-degree.
 __global__ void degree_kernel(const int64_t* __restrict__ indptr, int64_t N, int32_t* __restrict__ deg) {
   for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < N; u += (int64_t)gridDim.x * blockDim.x)
@@ -707,6 +829,14 @@ gs_status layerwise_degree_array(const gs_graph* g, cudaStream_t stream) {
   const int64_t blocks = std::min<int64_t>((g->num_nodes + 255) / 256, 148 * 16);
   if (g->num_nodes > 0) {
     degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
+    count_launch();
+  }
+  // the per-entry copy (4 B per CSC entry) when memory allows; without it the
+  // kernel looks b(u) up per candidate
+  if (g->num_edges > 0 && !gm->degsrc && gm->b_degsrc.ensure(gm->al, (size_t)g->num_edges * 4, stream)) {
+    gm->degsrc = (int32_t*)gm->b_degsrc.ptr;
+    const int64_t b2 = std::min<int64_t>((g->num_edges + 255) / 256, 148 * 16);
+    degsrc_kernel<<<(unsigned)b2, 256, 0, stream>>>(g->indices, gm->deg, g->num_edges, gm->degsrc);
     count_launch();
   }
   GS_CUDA_TRY(cudaGetLastError());
@@ -748,6 +878,7 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.L = L;
   P.mode = prob_mode;
   P.key = key;
+  P.pk = philox_keys(key);
   P.gw_log = gw_log;
   P.ng = ng;
   P.n4 = n4;
@@ -763,6 +894,7 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
     if (st) return st;
   }
   P.deg = g->deg;
+  P.degsrc = g->degsrc;
   blk->kind = gs_blocks::LAYERWISE;
   blk->num_batches = nbatch;
   blk->num_layers = L;
