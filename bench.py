@@ -731,6 +731,15 @@ KERNEL_OF = {"nodewise": "node-wise engine (nodewise_hop.cu: nprep / select / ro
              "layerwise": "gsb::layerwise_kernel", "walk": "gsb::walk_kernel"}
 
 
+def kernel_name(kind, wl):
+    if kind == "layerwise":  # layerwise.cu run_layerwise: which kernel takes the call
+        if wl.get("mode", 0) == 1:
+            return "gsb::layerwise_bm_kernel (FastGCN: candidate bitmaps)"
+        if max(wl["n_per_layer"]) <= 1024 and wl["batch"] <= 1024:
+            return "gsb::layerwise_sm_kernel<1024, 12> (LADIES / COUNT: shared-memory tables)"
+    return KERNEL_OF[kind]
+
+
 def ncu_traffic(workload):
     """DRAM bytes per launch of the dominant kernel from the committed ncu --set full capture."""
     try:
@@ -796,7 +805,7 @@ def main():
             "roofline": {"bound": "hbm", "achieved": r["achieved"], "peak": r["peak"],
                          "unit": "GB/s", "frac": r["achieved"] / r["peak"],
                          "traffic": ncu_traffic(args.workload), "peak_source": r["peak_src"],
-                         "kernel": KERNEL_OF[kind],
+                         "kernel": kernel_name(kind, wl),
                          "algorithmic_bytes_per_launch": r["bytes_per_launch"],
                          "random_sector_ceiling_gbs": RANDOM_SECTOR_GBS,
                          "frac_of_random_sector_ceiling": r["achieved"] / RANDOM_SECTOR_GBS,
