@@ -98,6 +98,8 @@ typedef struct gs_graph_info {
   const int32_t* indices;  /* device */
   const float* weights;    /* device or NULL */
   int host_mapped;         /* indices / weights are mapped host memory (GS_GRAPH_HOST_MAPPED) */
+  int64_t cached_pages;    /* HBM cache of a host-mapped graph (gs_graph_cache_hot): pages held, */
+  int64_t cache_page_entries; /* CSC entries per page                                           */
 } gs_graph_info;
 gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out);
 /* Replaces the edge weights (device float[num_edges]) and recomputes the a0
@@ -105,6 +107,17 @@ gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out);
  * kept alive by the caller).  Structure, validation and derived index arrays
  * are unchanged.  Used to sample over a computed bias (PASS att, R29). */
 gs_status gs_graph_set_weights(gs_graph* g, const float* weights, uint32_t flags, void* stream);
+/* Hot-column cache of a host-mapped graph (GS_GRAPH_HOST_MAPPED; P:490's
+ * "caching hot data in GPU"): copies the hottest pages of the
+ * index (and weight) array -- pages of 16,384 CSC entries, scored by the sum
+ * over their entries of min(32, in-degree of the entry's column), i.e. the
+ * expected node-wise accesses per entry when frontier nodes are drawn in
+ * proportion to degree -- into HBM, at most budget_bytes of them; the
+ * node-wise sampler then reads cached entries from HBM and the rest over the
+ * host link.  Results are unchanged (tested).  A second call replaces the
+ * cache; budget_bytes = 0 drops it.  GS_ERR_INVALID_ARGUMENT for a graph that
+ * is not host-mapped.  Synchronises the stream (page scores come to the host). */
+gs_status gs_graph_cache_hot(gs_graph* g, int64_t budget_bytes, void* stream);
 void gs_graph_destroy(gs_graph* g);
 
 /* ------------------------------------------------------------------------ */

@@ -9,6 +9,7 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <vector>
 #include <new>
 
 #include "gs_internal.h"
@@ -389,6 +390,94 @@ gs_status gs_graph_get_info(const gs_graph* g, gs_graph_info* out) {
   out->indices = g->indices;
   out->weights = g->weights;
   out->host_mapped = g->host_mapped ? 1 : 0;
+  out->cached_pages = g->ptab ? g->cached_pages : 0;
+  out->cache_page_entries = int64_t(1) << g->cpsh;
+  return GS_OK;
+}
+
+// Hot-page cache (gs_graph_cache_hot): score[p] = sum over the CSC entries of
+// page p of min(32, in-degree of the entry's column) -- the expected
+// node-wise accesses of an entry when frontier nodes come in proportion to
+// degree and a column access reads min(k, d) of its d entries.
+__global__ void page_score_kernel(const int64_t* __restrict__ indptr, int64_t N, int psh,
+                                  unsigned long long* __restrict__ score) {
+  for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = indptr[v], b = indptr[v + 1];
+    if (b <= a) continue;
+    const unsigned long long wgt = (unsigned long long)(b - a < 32 ? b - a : 32);
+    for (int64_t p = a >> psh; p <= (b - 1) >> psh; ++p) {
+      const int64_t lo = max(a, p << psh), hi = min(b, (p + 1) << psh);
+      atomicAdd(score + p, (unsigned long long)(hi - lo) * wgt);
+    }
+  }
+}
+
+// Copies page slot_page[s] of the (host-mapped) index / weight arrays into slot s.
+__global__ void page_copy_kernel(const int32_t* __restrict__ idx, const float* __restrict__ w, int64_t nnz, int psh,
+                                 const int32_t* __restrict__ slot_page, int32_t* __restrict__ cidx,
+                                 float* __restrict__ cw) {
+  const int64_t s = blockIdx.x;
+  const int64_t p = slot_page[s];
+  const int64_t a = p << psh, b = min(nnz, (p + 1) << psh);
+  for (int64_t i = a + threadIdx.x; i < b; i += blockDim.x) {
+    cidx[(s << psh) + (i - a)] = idx[i];
+    if (w) cw[(s << psh) + (i - a)] = w[i];
+  }
+}
+
+gs_status gs_graph_cache_hot(gs_graph* g, int64_t budget_bytes, void* stream_) {
+  if (!g || !g->host_mapped || budget_bytes < 0)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_graph_cache_hot: needs a host-mapped graph and budget >= 0");
+  cudaStream_t stream = (cudaStream_t)stream_;
+  g->ptab = nullptr;
+  g->cidx = nullptr;
+  g->cw = nullptr;
+  g->cached_pages = 0;
+  const int psh = g->cpsh;
+  const int64_t npages = (g->num_edges + (int64_t(1) << psh) - 1) >> psh;
+  const int64_t page_bytes = (int64_t(1) << psh) * (g->weights ? 8 : 4);
+  const int64_t nsel = std::min<int64_t>(npages, budget_bytes / page_bytes);
+  if (nsel <= 0) return GS_OK;
+  // page scores on the device, ranked on the host
+  gsb::DevBuf sc;
+  if (!sc.ensure(g->al, (size_t)npages * 8, stream, true))
+    return fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_cache_hot: device allocation failed");
+  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((g->num_nodes + 255) / 256, (int64_t)num_sms() * 16));
+  page_score_kernel<<<(unsigned)blocks, 256, 0, stream>>>(g->indptr, g->num_nodes, psh,
+                                                           (unsigned long long*)sc.ptr);
+  count_launch();
+  std::vector<unsigned long long> score((size_t)npages);
+  GS_CUDA_TRY(cudaMemcpyAsync(score.data(), sc.ptr, (size_t)npages * 8, cudaMemcpyDeviceToHost, stream));
+  GS_CUDA_TRY(cudaStreamSynchronize(stream));
+  sc.reset(g->al, stream);
+  std::vector<int32_t> order((size_t)npages);
+  for (int64_t p = 0; p < npages; ++p) order[(size_t)p] = (int32_t)p;
+  std::partial_sort(order.begin(), order.begin() + nsel, order.end(), [&](int32_t a, int32_t b) {
+    return score[(size_t)a] > score[(size_t)b] || (score[(size_t)a] == score[(size_t)b] && a < b);
+  });
+  order.resize((size_t)nsel);
+  std::sort(order.begin(), order.end());  // slots in page order
+  std::vector<int32_t> ptab((size_t)npages, -1);
+  for (int64_t s = 0; s < nsel; ++s) ptab[(size_t)order[(size_t)s]] = (int32_t)s;
+  gsb::DevBuf sp;
+  if (!g->b_ptab.ensure(g->al, (size_t)npages * 4, stream) ||
+      !g->b_cidx.ensure(g->al, (size_t)nsel << psh << 2, stream) ||
+      (g->weights && !g->b_cw.ensure(g->al, (size_t)nsel << psh << 2, stream)) ||
+      !sp.ensure(g->al, (size_t)nsel * 4, stream))
+    return fail(GS_ERR_OUT_OF_MEMORY, "gs_graph_cache_hot: device allocation failed (cache)");
+  GS_CUDA_TRY(cudaMemcpyAsync(g->b_ptab.ptr, ptab.data(), (size_t)npages * 4, cudaMemcpyHostToDevice, stream));
+  GS_CUDA_TRY(cudaMemcpyAsync(sp.ptr, order.data(), (size_t)nsel * 4, cudaMemcpyHostToDevice, stream));
+  page_copy_kernel<<<(unsigned)nsel, 512, 0, stream>>>(g->indices, g->weights, g->num_edges, psh,
+                                                       (const int32_t*)sp.ptr, (int32_t*)g->b_cidx.ptr,
+                                                       g->weights ? (float*)g->b_cw.ptr : nullptr);
+  count_launch();
+  GS_CUDA_TRY(cudaGetLastError());
+  GS_CUDA_TRY(cudaStreamSynchronize(stream));  // the host vectors above die with this call
+  sp.reset(g->al, stream);
+  g->ptab = (int32_t*)g->b_ptab.ptr;
+  g->cidx = (int32_t*)g->b_cidx.ptr;
+  g->cw = g->weights ? (float*)g->b_cw.ptr : nullptr;
+  g->cached_pages = nsel;
   return GS_OK;
 }
 
@@ -401,8 +490,12 @@ void gs_graph_destroy(gs_graph* g) {
   g->b_colsum.reset(g->al, s);
   g->b_poscnt.reset(g->al, s);
   g->b_deg.reset(g->al, s);
+  g->b_degsrc.reset(g->al, s);
   g->b_walk.reset(g->al, s);
   g->b_err.reset(g->al, s);
+  g->b_ptab.reset(g->al, s);
+  g->b_cidx.reset(g->al, s);
+  g->b_cw.reset(g->al, s);
   for (int k = 0; k < g->n_reg; ++k) cudaHostUnregister(g->host_reg[k]);
   delete g;
 }

@@ -73,6 +73,14 @@ struct gs_graph {
   int* d_err = nullptr;  // walk error word
   bool host_mapped = false;  // indices (+ weights) read from pinned host memory (UVA)
   void* host_reg[2] = {nullptr, nullptr};  // ranges this graph registered (unregistered at destroy)
+  // hot-page HBM cache of a host-mapped graph (gs_graph_cache_hot): ptab[page] =
+  // slot of the page in cidx / cw, or -1; pages of 1 << cpsh entries
+  gsb::DevBuf b_ptab, b_cidx, b_cw;
+  int32_t* ptab = nullptr;
+  int32_t* cidx = nullptr;
+  float* cw = nullptr;
+  int cpsh = 14;
+  int64_t cached_pages = 0;
   int n_reg = 0;
 };
 

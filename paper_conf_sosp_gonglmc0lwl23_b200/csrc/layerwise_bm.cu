@@ -831,9 +831,10 @@ gs_status layerwise_degree_array(const gs_graph* g, cudaStream_t stream) {
     degree_kernel<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(g->indptr, g->num_nodes, gm->deg);
     count_launch();
   }
-  // the per-entry copy (4 B per CSC entry) when memory allows; without it the
+  // the per-entry copy (4 B per CSC entry) when memory allows (not for
+  // host-mapped graphs: it is as large as their index array); without it the
   // kernel looks b(u) up per candidate
-  if (g->num_edges > 0 && !gm->degsrc && gm->b_degsrc.ensure(gm->al, (size_t)g->num_edges * 4, stream)) {
+  if (g->num_edges > 0 && !gm->degsrc && !g->host_mapped && gm->b_degsrc.ensure(gm->al, (size_t)g->num_edges * 4, stream)) {
     gm->degsrc = (int32_t*)gm->b_degsrc.ptr;
     const int64_t b2 = std::min<int64_t>((g->num_edges + 255) / 256, 148 * 16);
     degsrc_kernel<<<(unsigned)b2, 256, 0, stream>>>(g->indices, gm->deg, g->num_edges, gm->degsrc);

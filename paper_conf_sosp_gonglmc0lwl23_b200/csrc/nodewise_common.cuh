@@ -21,7 +21,29 @@ struct NWCore {
   int* err;
   int replace, bias;
   uint64_t key;
+  // host-mapped graphs: HBM copies of the hot pages (gs_graph_cache_hot), or NULL
+  const int32_t* ptab;  // page -> slot in cidx / cw, -1 if not cached
+  const int32_t* cidx;
+  const float* cw;
+  int cpsh;             // log2 entries per page
 };
+
+// Address of CSC entry pos of the index / weight array: its HBM copy when the
+// page is cached (host-mapped graphs), else the array itself.
+__device__ __forceinline__ const int32_t* nw_idx(const NWCore& P, int64_t pos) {
+  if (P.ptab) {
+    const int s = __ldg(P.ptab + (pos >> P.cpsh));
+    if (s >= 0) return P.cidx + (((int64_t)s << P.cpsh) | (pos & ((int64_t(1) << P.cpsh) - 1)));
+  }
+  return P.indices + pos;
+}
+__device__ __forceinline__ const float* nw_w(const NWCore& P, int64_t pos) {
+  if (P.ptab && P.cw) {
+    const int s = __ldg(P.ptab + (pos >> P.cpsh));
+    if (s >= 0) return P.cw + (((int64_t)s << P.cpsh) | (pos & ((int64_t(1) << P.cpsh) - 1)));
+  }
+  return P.weights + pos;
+}
 
 // Shared memory of one warp's chunk of 32 columns.
 struct WarpChunk {
@@ -157,7 +179,7 @@ __device__ __forceinline__ void ares_filter(const NWCore& P, int32_t v, int64_t 
       r[0] = R.x; r[1] = R.y; r[2] = R.z; r[3] = R.w;
 #pragma unroll
       for (int q = 0; q < 4; ++q)
-        w[q] = i0 + q < d ? (P.weights ? ldg_h(P.weights + off + i0 + q, pf) : 1.0f) : 0.0f;
+        w[q] = i0 + q < d ? (P.weights ? ldg_h(nw_w(P, off + i0 + q), pf) : 1.0f) : 0.0f;
     }
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
@@ -195,7 +217,7 @@ __device__ __forceinline__ int ares_exact(const NWCore& P, int32_t v, int64_t of
   for (int j = lane; j < m; j += 32) {
     const uint32_t p = pos[j];
     const U4 R = philox_nl((uint32_t)v, p >> 2, ctr2(l, TAG_ARES_NODE), gb, P.key);
-    const float w = P.weights ? __ldg(P.weights + off + p) : 1.0f;
+    const float w = P.weights ? __ldg(nw_w(P, off + p)) : 1.0f;
     const double kk = ares_key_nl(sel_word(R, (int)(p & 3)), (double)w);
     key[j] = kk;
     below += (tau < 0.0f || kk < (double)tau) ? 1 : 0;

@@ -284,7 +284,7 @@ __device__ void nv_select_weighted(const NVParams& P, SM& sm, NVWeighted& W, War
   int cnt = 0;
   if (d <= k) {
     for (int i = 0; i < (int)d; ++i) {
-      const float w = P.core.weights ? __ldg(P.core.weights + off + i) : 1.0f;
+      const float w = P.core.weights ? __ldg(nw_w(P.core, off + i)) : 1.0f;
       if (w > 0.0f) C.list[cnt++][lane] = (uint32_t)i;
     }
   }
@@ -395,12 +395,12 @@ __device__ int nv_gather(const NVParams& P, WarpChunk& C, const NVSeg& sg, long 
     const uint32_t p = (uint32_t)((jb + c) * k + q);
     sth(S.pos + p, ps, pl);
     if (S.val) {
-      const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
+      const float w = P.core.weights ? __ldg(nw_w(P.core, C.coff[c] + ps)) : 1.0f;
       sth(S.val + p, w / C.csum[c], pl);
     }
     const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
     asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
-                 "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
+                 "l"(nw_idx(P.core, C.coff[c] + ps)), "l"(pf)
                  : "memory");
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
@@ -509,12 +509,12 @@ __device__ int nv_chunk_uniform(const NVParams& P, WarpChunk& C, const NVSeg& sg
     const uint32_t p = (uint32_t)((jb + c) * k + q);
     sth(S.pos + p, ps, pl);
     if (S.val) {
-      const float w = P.core.weights ? __ldg(P.core.weights + C.coff[c] + ps) : 1.0f;
+      const float w = P.core.weights ? __ldg(nw_w(P.core, C.coff[c] + ps)) : 1.0f;
       sth(S.val + p, w / C.csum[c], pl);
     }
     const unsigned dst = (unsigned)__cvta_generic_to_shared(&C.list[q][c]);
     asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst),
-                 "l"(P.core.indices + C.coff[c] + ps), "l"(pf)
+                 "l"(nw_idx(P.core, C.coff[c] + ps)), "l"(pf)
                  : "memory");
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
@@ -803,6 +803,10 @@ gs_status run_nodewise_wave(const gs_graph* g, const int32_t* seeds, int64_t num
   P.core.indptr = g->indptr;
   P.core.indices = g->indices;
   P.core.weights = g->weights;
+  P.core.ptab = g->ptab;
+  P.core.cidx = g->cidx;
+  P.core.cw = g->cw;
+  P.core.cpsh = g->cpsh;
   P.core.colsum = g->colsum;
   P.core.N = g->num_nodes;
   P.core.replace = replace;

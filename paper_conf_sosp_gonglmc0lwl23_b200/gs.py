@@ -39,7 +39,8 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_kernel_launche
            "gs_random_walk", "gs_walk_check", "gs_matrix_slice_columns", "gs_matrix_slice_rows",
            "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
            "gs_matrix_get_view", "gs_matrix_destroy", "gs_matrix_individual_sample",
-           "gs_matrix_collective_sample", "gs_matrix_map_reduce", "gs_matrix_asgcn_bias", "gs_pass_attention", "gs_graph_set_weights"]
+           "gs_matrix_collective_sample", "gs_matrix_map_reduce", "gs_matrix_asgcn_bias", "gs_pass_attention", "gs_graph_set_weights",
+           "gs_graph_cache_hot"]
 OP_ADD, OP_SUB, OP_MUL, OP_DIV, OP_POW = 0, 1, 2, 3, 4
 
 
@@ -67,7 +68,8 @@ class _GraphInfo(ctypes.Structure):
                 ("weighted", ctypes.c_int), ("sorted", ctypes.c_int),
                 ("max_in_degree", ctypes.c_int64), ("indptr", ctypes.c_void_p),
                 ("indices", ctypes.c_void_p), ("weights", ctypes.c_void_p),
-                ("host_mapped", ctypes.c_int)]
+                ("host_mapped", ctypes.c_int), ("cached_pages", ctypes.c_int64),
+                ("cache_page_entries", ctypes.c_int64)]
 
 
 class _LayerBuffers(ctypes.Structure):
@@ -142,6 +144,7 @@ def load_library(path: str = LIB_PATH):
                                     vp, ctypes.POINTER(vp)]
     L.gs_pass_attention.argtypes = [vp, vp, i32, vp, vp, i32, vp, vp, vp]
     L.gs_graph_set_weights.argtypes = [vp, vp, ctypes.c_uint32, vp]
+    L.gs_graph_cache_hot.argtypes = [vp, i64, vp]
     L.gs_matrix_slice_columns.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_slice_rows.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_sum.argtypes = [vp, i32, vp, vp]
@@ -267,6 +270,17 @@ class Graph:
     @property
     def handle(self):
         return self._h
+
+    def cache_hot(self, budget_bytes: int, stream=None) -> int:
+        """Host-mapped graphs: copies the hottest pages of the index / weight
+        arrays into HBM (gs_graph_cache_hot, at most budget_bytes); returns the
+        number of cached CSC entries."""
+        L = load_library()
+        _check(L.gs_graph_cache_hot(self._h, ctypes.c_int64(int(budget_bytes)), _stream_ptr(stream)),
+               "gs_graph_cache_hot")
+        info = _GraphInfo()
+        _check(L.gs_graph_get_info(self._h, ctypes.byref(info)))
+        return int(info.cached_pages * info.cache_page_entries)
 
     def set_weights(self, weights: torch.Tensor, borrow: bool = True, stream=None) -> "Graph":
         """Replaces the edge weights (e.g. PASS att) and recomputes the a0 column sums."""

@@ -66,3 +66,35 @@ def test_uva_walks(gs, graphs):
         a = gs.random_walk(Gh, st, 20, p=pq[0], q=pq[1], rng_key=9)
         b = gs.random_walk(Gd, st, 20, p=pq[0], q=pq[1], rng_key=9)
         assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("budget_frac", [0.0, 0.3, 1.0])
+def test_uva_hot_page_cache(gs, budget_frac, oracle_lib):
+    """gs_graph_cache_hot: the node-wise sampler reads cached pages from HBM and
+    the rest over the host link -- the same blocks as without a cache (and as
+    the oracle), uniform, weighted and PASS-style, whatever the budget."""
+    g = synth.small_graph(200_000, 3_000_000, undirected=True, weights="uniform", seed=78, device="cuda")
+    Gd = gs.Graph(g["indptr"], g["indices"], g["weights"])
+    Gh = gs.Graph(g["indptr"], g["indices"], g["weights"], host_mapped=True)
+    budget = int(budget_frac * g["indices"].numel() * 8)
+    cached = Gh.cache_hot(budget)
+    if budget_frac == 1.0:
+        assert cached >= g["indices"].numel()
+    elif budget_frac == 0.0:
+        assert cached == 0
+    else:
+        assert 0 < cached < g["indices"].numel()
+    for bias in (0, 1, 2):
+        a = gs.sample_neighbors(Gh, seeds(3000, 8), [10, 5], batch_size=1024, bias_mode=bias, rng_key=9).to_host()
+        b = gs.sample_neighbors(Gd, seeds(3000, 8), [10, 5], batch_size=1024, bias_mode=bias, rng_key=9).to_host()
+        compare_all(a, b, f"uva cache {budget_frac} bias={bias}")
+    O = oracle_lib.Graph(*host_graph(g))
+    ref = oracle_lib.sample_neighbors(O, seeds(3000, 8).cpu().numpy(), [10, 5], batch_size=1024, rng_key=9)
+    a = gs.sample_neighbors(Gh, seeds(3000, 8), [10, 5], batch_size=1024, rng_key=9).to_host()
+    compare_all(a, ref, f"uva cache {budget_frac} vs oracle")
+
+
+def test_uva_cache_rejects_hbm_graph(gs, graphs):
+    g, Gd, Gh = graphs
+    with pytest.raises(gs.GSError):
+        Gd.cache_hot(1 << 20)
