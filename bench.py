@@ -61,6 +61,12 @@ WORKLOADS = {
                              desc="GraphSAGE [25,10] as graphsage_pd with the CSC index array in "
                                   "pinned host memory read over the host link (UVA, P:415; "
                                   "SURVEY 8(f) f4)"),
+    "graphsage_pd_uva_cache": dict(kind="nodewise", graph="PD", fanouts=[25, 10], batch=1024,
+                                   seeds=196_615, replace=False, bias=0, host_mapped=True,
+                                   cache_frac=0.25,
+                                   desc="GraphSAGE [25,10] as graphsage_pd_uva with the hottest quarter "
+                                        "of the index array cached in HBM (gs_graph_cache_hot, P:490; "
+                                        "SURVEY 8(f) f4)"),
     "graphsage_tiny": dict(kind="nodewise", graph="tiny", fanouts=[5, 5], batch=512, seeds=512,
                            replace=False, bias=0,
                            desc="GraphSAGE [5,5] uniform, 512 seeds, 10k-node/100k-edge R-MAT"),
@@ -388,6 +394,8 @@ def run_gpu(args, wl, world, rank, device):
     g = make_graph_dist(wl["graph"], world, rank, device)
     gen_s = time.time() - t0
     G = gs.Graph(g["indptr"], g["indices"], g["weights"], host_mapped=wl.get("host_mapped", False))
+    if wl.get("cache_frac"):
+        G.cache_hot(int(wl["cache_frac"] * g["indices"].numel() * (8 if g["weights"] is not None else 4)))
     all_inputs = workload_inputs(wl, g, device)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=device)  # > 126 MB L2
     out = gs.Blocks()

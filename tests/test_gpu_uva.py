@@ -76,7 +76,7 @@ def test_uva_hot_page_cache(gs, budget_frac, oracle_lib):
     g = synth.small_graph(200_000, 3_000_000, undirected=True, weights="uniform", seed=78, device="cuda")
     Gd = gs.Graph(g["indptr"], g["indices"], g["weights"])
     Gh = gs.Graph(g["indptr"], g["indices"], g["weights"], host_mapped=True)
-    budget = int(budget_frac * g["indices"].numel() * 8)
+    budget = int(budget_frac * (g["indices"].numel() + 16384) * 8)  # whole pages
     cached = Gh.cache_hot(budget)
     if budget_frac == 1.0:
         assert cached >= g["indices"].numel()
