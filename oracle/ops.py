@@ -273,3 +273,49 @@ def asgcn_bias(m, X, wg, num_nodes):
         g = g if g > 0 else np.float32(0.0)
         out[u] = np.float32(np.float32(s[u]) * g)
     return out
+
+
+# ---------------------------------------------------------------------------
+# Heterogeneous graphs ("each type of edges is modeled as a sparse
+# matrix to conduct the same sampling workflow as homogeneous graphs"; SURVEY
+# 8(f) f4).  Relation r is its own CSC matrix whose columns are nodes of type
+# dst[r] and whose rows are nodes of type src[r] (ids local to each type).
+# Layer l: every relation r samples fanouts[l][r] entries of each frontier
+# column of type dst[r] (A_r[:, F_dst].individual_sample, uniform without
+# replacement, R5) with the relation's key (R33); the next frontier of type t
+# is the union of the rows of the relations whose src is t, ascending (A.row()
+# of each, merged).
+# ---------------------------------------------------------------------------
+def relation_key(rng_key, r):
+    """R33: the RNG key of relation r -- rng_key XOR (r + 1) times the 64-bit
+    golden ratio, so relations never share a Philox stream."""
+    return (int(rng_key) ^ ((0x9E3779B97F4A7C15 * (r + 1)) & 0xFFFFFFFFFFFFFFFF)) & 0xFFFFFFFFFFFFFFFF
+
+
+def hetero_sample_neighbors(rels, num_nodes, seeds, fanouts, rng_key):
+    """rels[r] = (src_type, dst_type, indptr, indices); num_nodes[t]; seeds[t]
+    (int32 array, possibly empty); fanouts[l][r] (0: relation skipped at l).
+    Returns (blocks, frontiers): blocks[l][r] the sampled sub-matrix (or None),
+    frontiers[l][t] for l = 0 .. L (frontiers[0] = the seeds)."""
+    T = len(num_nodes)
+    frontiers = [[np.asarray(seeds[t], np.int32) for t in range(T)]]
+    blocks = []
+    for l, fl in enumerate(fanouts):
+        bl = []
+        for r, (st, dt, ip, ix) in enumerate(rels):
+            F = frontiers[l][dt]
+            if fl[r] == 0 or len(F) == 0:
+                bl.append(None)
+                continue
+            m = slice_columns(ip, ix, None, F)
+            bl.append(individual_sample(m, fl[r], relation_key(rng_key, r), layer=l, batch=0))
+        blocks.append(bl)
+        nxt = []
+        for t in range(T):
+            rows = set()
+            for r, (st, dt, ip, ix) in enumerate(rels):
+                if st == t and bl[r] is not None:
+                    rows |= set(row_ids(bl[r]).tolist())
+            nxt.append(np.array(sorted(rows), np.int32))
+        frontiers.append(nxt)
+    return blocks, frontiers
