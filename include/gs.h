@@ -383,6 +383,40 @@ gs_status gs_matrix_asgcn_bias(const gs_matrix* m, const void* X, int F, const f
 gs_status gs_matrix_get_view(const gs_matrix* m, gs_matrix_view* out);
 void      gs_matrix_destroy(gs_matrix* m);
 
+/* ------------------------------------------------------------------------ */
+/* Heterogeneous graphs ("each type of edges is modeled as a sparse    */
+/* matrix to conduct the same sampling workflow as homogeneous graphs";      */
+/* SURVEY 8(f) f4).                                                           */
+/* ------------------------------------------------------------------------ */
+typedef struct gs_hetero gs_hetero;
+/* One mini-batch of node-wise (GraphSAGE, R5) sampling over num_relations
+ * edge types.  Relation r: graphs[r] is the CSC matrix of that edge type --
+ * column v = the in-neighbours of destination node v of type dst_type[r], row
+ * ids = source nodes of type src_type[r], both in per-type local ids; it has
+ * max(num_nodes[src], num_nodes[dst]) columns (columns past the destination
+ * type's count empty).  seeds[t] (device int32[num_seeds[t]], NULL when 0) are
+ * the layer-0 frontier of node type t.  Layer l, relation r: every frontier
+ * node of type dst_type[r] samples fanouts[l * num_relations + r] (0..32; 0
+ * skips the relation at that layer) of its in-neighbours in graphs[r] --
+ * A_r[:, F].individual_sample(k), so the RNG keying is the homogeneous one
+ * (R4, layer l, batch 0) under the key rng_key XOR (r + 1) * 0x9E3779B97F4A7C15
+ * (R33); the frontier of type t at layer l + 1 is the union of the sampled
+ * rows of every relation with src_type == t, ascending (A.row()).
+ * Results: gs_hetero_block (layer, relation) -> the sampled sub-matrix (global
+ * per-type ids, COO + CSC over the frontier; NULL when skipped), borrowed
+ * from the gs_hetero; gs_hetero_frontier (layer 0..num_layers, type) -> device
+ * ids + count.  Synchronises the stream (sizes).  Errors: GS_ERR_INVALID_ARGUMENT
+ * (counts, types, fanouts, a graph with too few columns), GS_ERR_INDEX_OUT_OF_RANGE
+ * (a seed or row id outside its type). */
+gs_status gs_sample_neighbors_hetero(const gs_graph* const* graphs, const int32_t* src_type,
+                                     const int32_t* dst_type, int num_relations, int num_node_types,
+                                     const int64_t* num_nodes, const int32_t* const* seeds,
+                                     const int64_t* num_seeds, const int32_t* fanouts, int num_layers,
+                                     uint64_t rng_key, void* stream, gs_hetero** out);
+gs_status gs_hetero_block(const gs_hetero* h, int layer, int relation, const gs_matrix** out);
+gs_status gs_hetero_frontier(const gs_hetero* h, int layer, int node_type, const int32_t** ids, int64_t* n);
+void      gs_hetero_destroy(gs_hetero* h);
+
 /* PASS learned bias in full (Fig. 3(c) lines 3-9; DESIGN R29; SURVEY
  * 8(f) f2).  att[e] for every edge e = (u -> v) of g (weight w_e, 1 if unweighted):
  *   A1 = w_e <X_u W1, X_v W1>, A2 = w_e <X_u W2, X_v W2>, A3 = fp32(w_e / colsum_v),

@@ -19,6 +19,7 @@
 
 #include <algorithm>
 #include <new>
+#include <vector>
 
 #include "common.cuh"
 #include "gs_internal.h"
@@ -1021,3 +1022,157 @@ void gs_matrix_destroy(gs_matrix* m) {
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------------------
+// Heterogeneous node-wise sampling (each edge type is a sparse matrix
+// sampled by the same workflow; oracle/ops.py
+// hetero_sample_neighbors).  Per layer and relation r: A_r[:, F_dst(r)]
+// (gs_matrix_slice_columns) .individual_sample(k) (Floyd, R5) under the
+// relation's key (R33); the next frontier of every node type is the union of
+// the rows of the relations out of that type, ascending (A.row() of each,
+// merged in one bitmap: mark -> popcount scan -> emit).
+// ---------------------------------------------------------------------------
+struct gs_hetero {
+  gsb::Allocator al;
+  int L = 0, R = 0, T = 0;
+  std::vector<gs_matrix*> blocks;    // [L][R], NULL where skipped
+  std::vector<gsb::DevBuf> fr;       // [L + 1][T] frontier ids
+  std::vector<int64_t> nfr;          // [L + 1][T]
+};
+
+namespace gsb {
+static uint64_t relation_key(uint64_t key, int r) {  // R33
+  return key ^ (0x9E3779B97F4A7C15ull * (uint64_t)(r + 1));
+}
+}  // namespace gsb
+
+void gs_hetero_destroy(gs_hetero* h) {
+  if (!h) return;
+  for (gs_matrix* m : h->blocks) gs_matrix_destroy(m);
+  for (auto& b : h->fr) b.reset(h->al, nullptr);
+  delete h;
+}
+
+gs_status gs_sample_neighbors_hetero(const gs_graph* const* graphs, const int32_t* src_type, const int32_t* dst_type,
+                                     int num_relations, int num_node_types, const int64_t* num_nodes,
+                                     const int32_t* const* seeds, const int64_t* num_seeds, const int32_t* fanouts,
+                                     int num_layers, uint64_t rng_key, void* stream_, gs_hetero** out) {
+  if (!graphs || !src_type || !dst_type || !num_nodes || !seeds || !num_seeds || !fanouts || !out ||
+      num_relations < 1 || num_node_types < 1 || num_layers < 1 || num_layers > MAX_LAYERS)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_neighbors_hetero: null pointer or bad count");
+  for (int r = 0; r < num_relations; ++r) {
+    if (!graphs[r] || src_type[r] < 0 || src_type[r] >= num_node_types || dst_type[r] < 0 ||
+        dst_type[r] >= num_node_types)
+      return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_neighbors_hetero: relation %d: bad graph or node type", r);
+    if (graphs[r]->num_nodes < num_nodes[dst_type[r]] || graphs[r]->num_nodes < num_nodes[src_type[r]])
+      return fail(GS_ERR_INVALID_ARGUMENT,
+                  "gs_sample_neighbors_hetero: relation %d: its graph needs max(|src|, |dst|) columns", r);
+  }
+  for (int l = 0; l < num_layers; ++l)
+    for (int r = 0; r < num_relations; ++r)
+      if (fanouts[l * num_relations + r] < 0 || fanouts[l * num_relations + r] > MAX_FANOUT)
+        return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_neighbors_hetero: fanouts in [0, %d]", MAX_FANOUT);
+  for (int t = 0; t < num_node_types; ++t)
+    if (num_seeds[t] < 0 || (num_seeds[t] > 0 && !seeds[t]) || num_nodes[t] < 0)
+      return fail(GS_ERR_INVALID_ARGUMENT, "gs_sample_neighbors_hetero: node type %d: bad seeds", t);
+  cudaStream_t s = (cudaStream_t)stream_;
+  gs_hetero* h = new (std::nothrow) gs_hetero();
+  if (!h) return fail(GS_ERR_OUT_OF_MEMORY, "gs_sample_neighbors_hetero: host allocation failed");
+  h->al = current_allocator();
+  h->L = num_layers;
+  h->R = num_relations;
+  h->T = num_node_types;
+  h->blocks.assign((size_t)num_layers * num_relations, nullptr);
+  h->fr.resize((size_t)(num_layers + 1) * num_node_types);
+  h->nfr.assign((size_t)(num_layers + 1) * num_node_types, 0);
+  auto bail = [&](gs_status st) {
+    gs_hetero_destroy(h);
+    return st;
+  };
+  for (int t = 0; t < num_node_types; ++t) {
+    DevBuf& b = h->fr[(size_t)t];
+    if (!b.ensure(h->al, (size_t)std::max<int64_t>(num_seeds[t], 1) * 4, s))
+      return bail(fail(GS_ERR_OUT_OF_MEMORY, "hetero frontier"));
+    if (num_seeds[t] > 0)
+      if (cudaMemcpyAsync(b.ptr, seeds[t], (size_t)num_seeds[t] * 4, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        return bail(fail(GS_ERR_CUDA, "hetero seed copy"));
+    h->nfr[(size_t)t] = num_seeds[t];
+  }
+  DevBuf bm, cnt, err;
+  int64_t maxn = 1;
+  for (int t = 0; t < num_node_types; ++t) maxn = std::max<int64_t>(maxn, num_nodes[t]);
+  const int64_t maxw = (maxn + 31) / 32;
+  if (!bm.ensure(h->al, (size_t)maxw * 4, s) || !cnt.ensure(h->al, (size_t)maxw * 8, s) ||
+      !err.ensure(h->al, 16, s, true))
+    return bail(fail(GS_ERR_OUT_OF_MEMORY, "hetero union workspace"));
+  gs_status st = GS_OK;
+  for (int l = 0; l < num_layers && st == GS_OK; ++l) {
+    for (int r = 0; r < num_relations && st == GS_OK; ++r) {
+      const int k = fanouts[l * num_relations + r];
+      const int dt = dst_type[r];
+      const int64_t nf = h->nfr[(size_t)l * num_node_types + dt];
+      if (k == 0 || nf == 0) continue;
+      gs_matrix* M = nullptr;
+      st = gs_matrix_slice_columns(graphs[r], (const int32_t*)h->fr[(size_t)l * num_node_types + dt].ptr, nf, s, &M);
+      if (st == GS_OK)
+        st = gs_matrix_individual_sample(M, k, 0, 0, relation_key(rng_key, r), l, 0, s,
+                                         &h->blocks[(size_t)l * num_relations + r]);
+      gs_matrix_destroy(M);
+    }
+    for (int t = 0; t < num_node_types && st == GS_OK; ++t) {
+      const int64_t nw = (num_nodes[t] + 31) / 32;
+      DevBuf& o = h->fr[(size_t)(l + 1) * num_node_types + t];
+      if (!o.ensure(h->al, (size_t)std::max<int64_t>(num_nodes[t], 1) * 4, s)) {
+        st = fail(GS_ERR_OUT_OF_MEMORY, "hetero frontier");
+        break;
+      }
+      if (nw == 0) continue;
+      if (cudaMemsetAsync(bm.ptr, 0, (size_t)nw * 4, s) != cudaSuccess) {
+        st = fail(GS_ERR_CUDA, "hetero union memset");
+        break;
+      }
+      for (int r = 0; r < num_relations; ++r) {
+        const gs_matrix* B = h->blocks[(size_t)l * num_relations + r];
+        if (src_type[r] != t || !B || B->nnz == 0) continue;
+        mark_rows_kernel<<<grid_for(B->nnz, 256), 256, 0, s>>>((const int32_t*)B->b_row.ptr, B->nnz, num_nodes[t],
+                                                               (uint32_t*)bm.ptr, (int*)err.ptr);
+        count_launch();
+      }
+      word_count_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (int64_t*)cnt.ptr);
+      count_launch();
+      if ((st = scan_inclusive((int64_t*)cnt.ptr, nw, h->al, s))) break;
+      emit_rows_kernel<<<grid_for(nw, 256), 256, 0, s>>>((const uint32_t*)bm.ptr, nw, (const int64_t*)cnt.ptr,
+                                                         (int32_t*)o.ptr);
+      count_launch();
+      int64_t n = 0;
+      if (cudaMemcpyAsync(&n, (int64_t*)cnt.ptr + nw - 1, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+          cudaStreamSynchronize(s) != cudaSuccess) {
+        st = fail(GS_ERR_CUDA, "hetero frontier count read-back");
+        break;
+      }
+      h->nfr[(size_t)(l + 1) * num_node_types + t] = n;
+    }
+  }
+  if (st == GS_OK) st = check_err((int*)err.ptr, s);
+  bm.reset(h->al, s);
+  cnt.reset(h->al, s);
+  err.reset(h->al, s);
+  if (st) return bail(st);
+  *out = h;
+  return GS_OK;
+}
+
+gs_status gs_hetero_block(const gs_hetero* h, int layer, int relation, const gs_matrix** out) {
+  if (!h || !out || layer < 0 || layer >= h->L || relation < 0 || relation >= h->R)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_hetero_block: bad layer / relation");
+  *out = h->blocks[(size_t)layer * h->R + relation];
+  return GS_OK;
+}
+
+gs_status gs_hetero_frontier(const gs_hetero* h, int layer, int node_type, const int32_t** ids, int64_t* n) {
+  if (!h || !ids || !n || layer < 0 || layer > h->L || node_type < 0 || node_type >= h->T)
+    return fail(GS_ERR_INVALID_ARGUMENT, "gs_hetero_frontier: bad layer / node type");
+  *ids = (const int32_t*)h->fr[(size_t)layer * h->T + node_type].ptr;
+  *n = h->nfr[(size_t)layer * h->T + node_type];
+  return GS_OK;
+}

@@ -40,7 +40,8 @@ EXPORTS = ["gs_last_error", "gs_status_string", "gs_version", "gs_kernel_launche
            "gs_matrix_sum", "gs_matrix_broadcast", "gs_matrix_elementwise", "gs_matrix_row_ids",
            "gs_matrix_get_view", "gs_matrix_destroy", "gs_matrix_individual_sample",
            "gs_matrix_collective_sample", "gs_matrix_map_reduce", "gs_matrix_asgcn_bias", "gs_pass_attention", "gs_graph_set_weights",
-           "gs_graph_cache_hot"]
+           "gs_graph_cache_hot", "gs_sample_neighbors_hetero", "gs_hetero_block",
+           "gs_hetero_frontier", "gs_hetero_destroy"]
 OP_ADD, OP_SUB, OP_MUL, OP_DIV, OP_POW = 0, 1, 2, 3, 4
 
 
@@ -145,6 +146,12 @@ def load_library(path: str = LIB_PATH):
     L.gs_pass_attention.argtypes = [vp, vp, i32, vp, vp, i32, vp, vp, vp]
     L.gs_graph_set_weights.argtypes = [vp, vp, ctypes.c_uint32, vp]
     L.gs_graph_cache_hot.argtypes = [vp, i64, vp]
+    L.gs_sample_neighbors_hetero.argtypes = [vp, vp, vp, i32, i32, vp, vp, vp, vp, i32, u64, vp,
+                                             ctypes.POINTER(vp)]
+    L.gs_hetero_block.argtypes = [vp, i32, i32, ctypes.POINTER(vp)]
+    L.gs_hetero_frontier.argtypes = [vp, i32, i32, ctypes.POINTER(vp), ctypes.POINTER(ctypes.c_int64)]
+    L.gs_hetero_destroy.argtypes = [vp]
+    L.gs_hetero_destroy.restype = None
     L.gs_matrix_slice_columns.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_slice_rows.argtypes = [vp, vp, i64, vp, ctypes.POINTER(vp)]
     L.gs_matrix_sum.argtypes = [vp, i32, vp, vp]
@@ -723,3 +730,66 @@ def blocks_profile(b: "Blocks") -> list:
         res.append((name.value.decode(), ms.value))
         i += 1
     return res
+
+
+class HeteroSample:
+    """Result of sample_neighbors_hetero: blocks[l][r] (Matrix views, None when
+    skipped) and frontiers[l][t] (device int32), l = 0 .. num_layers."""
+
+    def __init__(self, h, L, R, T, keep):
+        self._h = h
+        self._keep = keep
+        self.blocks, self.frontiers = [], []
+        for l in range(L):
+            row = []
+            for r in range(R):
+                m = ctypes.c_void_p()
+                _check(_lib.gs_hetero_block(h, l, r, ctypes.byref(m)), "gs_hetero_block")
+                row.append(self._view(m) if m.value else None)
+            self.blocks.append(row)
+        for l in range(L + 1):
+            fl = []
+            for t in range(T):
+                p, n = ctypes.c_void_p(), ctypes.c_int64()
+                _check(_lib.gs_hetero_frontier(h, l, t, ctypes.byref(p), ctypes.byref(n)), "gs_hetero_frontier")
+                fl.append(_dev_tensor(p.value, n.value, torch.int32, self))
+            self.frontiers.append(fl)
+
+    def _view(self, m):  # a borrowed gs_matrix (owned by the gs_hetero)
+        v = _MatrixView()
+        _check(_lib.gs_matrix_get_view(m, ctypes.byref(v)), "gs_matrix_get_view")
+        return {"num_nodes": v.num_nodes,
+                "cols": _dev_tensor(v.cols, v.n_cols, torch.int32, self),
+                "indptr": _dev_tensor(v.indptr, v.n_cols + 1, torch.int64, self),
+                "row": _dev_tensor(v.row, v.nnz, torch.int32, self),
+                "eid": _dev_tensor(v.eid, v.nnz, torch.int64, self)}
+
+    def __del__(self):
+        try:
+            if getattr(self, "_h", None) and _alive():
+                _lib.gs_hetero_destroy(self._h)
+                self._h = None
+        except TypeError:
+            pass
+
+
+def sample_neighbors_hetero(relations, num_nodes, seeds, fanouts, rng_key=0, stream=None) -> HeteroSample:
+    """Heterogeneous node-wise sampling (gs_sample_neighbors_hetero).
+    relations: list of (src_type, dst_type, Graph); num_nodes[t]; seeds[t]
+    (device int32, possibly empty); fanouts[l][r]."""
+    L = load_library()
+    _drain()
+    R, T, NL = len(relations), len(num_nodes), len(fanouts)
+    garr = (ctypes.c_void_p * R)(*[g.handle.value for _, _, g in relations])
+    st = torch.tensor([s for s, _, _ in relations], dtype=torch.int32)
+    dt = torch.tensor([d for _, d, _ in relations], dtype=torch.int32)
+    nn = torch.tensor(list(num_nodes), dtype=torch.int64)
+    sd = [s.to(torch.int32).contiguous() for s in seeds]
+    sarr = (ctypes.c_void_p * T)(*[(s.data_ptr() if s.numel() else None) for s in sd])
+    ns = torch.tensor([s.numel() for s in sd], dtype=torch.int64)
+    fo = torch.tensor([int(k) for fl in fanouts for k in fl], dtype=torch.int32)
+    h = ctypes.c_void_p()
+    _check(L.gs_sample_neighbors_hetero(garr, _ptr(st), _ptr(dt), R, T, _ptr(nn), sarr, _ptr(ns), _ptr(fo), NL,
+                                        ctypes.c_uint64(rng_key), _stream_ptr(stream), ctypes.byref(h)),
+           "gs_sample_neighbors_hetero")
+    return HeteroSample(h, NL, R, T, (relations, sd))
