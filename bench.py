@@ -634,7 +634,72 @@ def run_gpu(args, wl, world, rank, device):
                     if k2 != "totals"} for pk in packs]
     e2e_times, d2h_all = [], []
     copy_side = torch.cuda.Stream()
-    for i in range(max(2, min(args.steps, 5))):
+    # node-wise: the epoch's batches in E2E_CHUNKS contiguous chunks (each its
+    # own call with batch_index_base = its first global batch, so the union is
+    # the same epoch), every chunk's host copies issued on two copy streams as
+    # soon as its sizes are known while the next chunks sample: the link, not
+    # the sampler, bounds the step
+    chunked = kind == "nodewise" and inputs.numel() > 0
+    if chunked:
+        nbat = (inputs.numel() + bs - 1) // bs
+        nch = max(1, min(E2E_CHUNKS, nbat))
+        cb = [nbat * c // nch for c in range(nch + 1)]
+        souts = [gs.Blocks() for _ in range(nch)]
+        cstreams = (torch.cuda.Stream(), torch.cuda.Stream())
+
+        def step_chunk(i, c, x):
+            key = base_key + 7919 * i
+            lo, hi = cb[c] * bs, min(cb[c + 1] * bs, x.numel())
+            gs.sample_neighbors(G, x[lo:hi], wl["fanouts"], batch_size=bs, batch_index_base=wbase + cb[c],
+                                replace=wl["replace"], bias_mode=wl["bias"], rng_key=key,
+                                stream=stream, out=souts[c])
+
+        for c in range(nch):  # sizes the chunk results before the pack buffers
+            step_chunk(args.warmup, c, inputs)
+        torch.cuda.synchronize()
+        cpacks = [[so.pack(l, narrow=narrow) for l in range(L)] for so in souts]
+        cmeta = [so.device_meta() for so in souts]
+        chost_meta = [torch.empty(m.shape, dtype=m.dtype).pin_memory() for m in cmeta]
+        chost_tot = [torch.empty((L, 3), dtype=torch.int64).pin_memory() for _ in range(nch)]
+        chost_pk = [[{k2: torch.empty(v.shape, dtype=v.dtype).pin_memory() for k2, v in pk.items()
+                      if k2 != "totals"} for pk in cp] for cp in cpacks]
+    for i in range(max(2, min(args.steps, 5)) + (1 if chunked else 0)):
+        if chunked:
+            flush.zero_()
+            torch.cuda.synchronize()
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            dev_in.copy_(host_in, non_blocking=True)
+            ready = []
+            for c in range(nch):
+                step_chunk(args.warmup + i, c, dev_in)
+                for l in range(L):
+                    souts[c].pack(l, cpacks[c][l], stream=stream, narrow=narrow)
+                    chost_tot[c][l].copy_(cpacks[c][l]["totals"], non_blocking=True)
+                chost_meta[c].copy_(cmeta[c], non_blocking=True)
+                e = torch.cuda.Event()
+                e.record(stream)
+                ready.append(e)
+            d2h = 0
+            for c in range(nch):
+                ready[c].synchronize()  # this chunk's sizes (the later chunks keep sampling)
+                d2h += chost_tot[c].numel() * 8 + chost_meta[c].numel() * 8
+                for cs_ in cstreams:
+                    cs_.wait_event(ready[c])
+                for l in range(L):
+                    ne, ni, nr = (int(x) for x in chost_tot[c][l])
+                    for k2, n in (("row_local", ne), ("eid", ne), ("indptr", ni), ("row_map", nr)):
+                        with torch.cuda.stream(cstreams[1] if k2 == "eid" else cstreams[0]):
+                            chost_pk[c][l][k2][:n].copy_(cpacks[c][l][k2][:n], non_blocking=True)
+                        d2h += n * cpacks[c][l][k2].element_size()
+            for cs_ in cstreams:
+                stream.wait_stream(cs_)
+            ev1.record(stream)
+            ev1.synchronize()
+            if i > 0:  # the first pass warms the chunked path
+                e2e_times.append(ev0.elapsed_time(ev1))
+                d2h_all.append(d2h)
+            continue
         flush.zero_()
         torch.cuda.synchronize()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -732,6 +797,8 @@ def run_gpu(args, wl, world, rank, device):
             "launches_per_step": launches_per_step}
 
 
+E2E_CHUNKS = 4  # node-wise e2e: the epoch sampled and copied back in this many pipelined chunks
+
 KERNEL_OF = {"nodewise": "node-wise engine (nodewise_hop.cu: nprep / select / rows / relabel / clear per hop)",
              "shadow": "gsb::shadow_induce_kernel",
              "saint": "gsb::shadow_induce_kernel", "pinsage": "gsb::pinsage_kernel",
@@ -828,7 +895,10 @@ def main():
                     "d2h_gbs_over_step": r["d2h"] / (r["e2e_ms"] / 1000.0) / 1e9,
                     "note": "host copies (pinned) inside the timed region; sampled blocks packed densely "
                             "(int32 ids when the graph has < 2^31 entries) so exactly the sampled data "
-                            "crosses the host link, which bounds this number"},
+                            "crosses the host link, which bounds this number"
+                            + (f"; node-wise: the epoch in {E2E_CHUNKS} pipelined chunks (public calls with "
+                               "batch_index_base = the chunk's first batch), each chunk's copies on two copy "
+                               "streams while the next chunks sample" if kind == "nodewise" else "")},
             "gpu_launches": args.steps * r["launches_per_step"],
             "clocks": r["clocks"],
         }

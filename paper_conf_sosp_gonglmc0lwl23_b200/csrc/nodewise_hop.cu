@@ -79,7 +79,8 @@ struct HopParams {
   // workspace
   int64_t* coff;             // per frontier column: indptr[v] (column region of the hop)
   int32_t* dcol;             // per frontier column: in-degree (0 if the id is invalid)
-  unsigned long long* bm;    // [group slot][nwp] row bitmap: bits of 32 nodes (low) | rank (high)
+  uint32_t* bm;              // [group slot][nwp] row bitmap: one bit per node, 32-bit words
+  int32_t* rank4;            // [group slot][nwp / 4] rank of the first row of every non-empty 4-word group
   uint32_t* summ;            // [group slot][nsw] bit w set iff bitmap word w is non-empty
   int64_t nw, nwp, nsw;      // words used / allocated per batch, summary words
   int sel_nq, sel_claim;     // select: claim queues, chunks per claim
@@ -87,7 +88,6 @@ struct HopParams {
   int ares_split;            // A-Res columns with d > 64: 1 hop_ares_big_kernel, 0 in select
   int ares_tau;              // hop_ares_big_kernel's first threshold: 0 normal, 1 too tight,
                              // 2 too loose (tests: every widen / narrow step runs)
-  int wsh;                   // bitmap word index shift: 1 = 64-bit words (global finalize), 0 = 32-bit (cluster)
 };
 
 // Per-launch scan bookkeeping of nprep / rows (zeroed before the launch):
@@ -593,7 +593,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
     const int pre = warp_excl(cnt, &total);
     // gather (16 loads in flight per lane), bitmap bits, slot-major staging
     const int64_t slot = b - b0;
-    uint32_t* bits = (uint32_t*)(P.bm + slot * P.nwp);  // 32-bit words or the low halves of 64-bit ones
+    uint32_t* bits = P.bm + slot * P.nwp;
     uint32_t* summ = P.summ + slot * P.nsw;
 #pragma unroll
     for (int h = 0; h < KCAP; h += 16) {
@@ -626,7 +626,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
               C.sv[pre + i] = w / csum;
             }
           }
-          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + ((u[q] >> 5) << P.wsh)), "r"(1u << (u[q] & 31))
+          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + (u[q] >> 5)), "r"(1u << (u[q] & 31))
                        : "memory");
           if (use_sum)
             asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (u[q] >> 10)), "r"(1u << ((u[q] >> 5) & 31))
@@ -731,7 +731,7 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
     const int32_t v = active ? __ldcg(F + jcol) : -1;
     const int64_t off = active ? __ldcg(P.coff + cb + jcol) : 0;
     const int64_t slot = b - b0;
-    uint32_t* bits = (uint32_t*)(P.bm + slot * P.nwp);
+    uint32_t* bits = P.bm + slot * P.nwp;
     uint32_t* summ = P.summ + slot * P.nsw;
     const int use_sum = P.use_sum[l];
     // per-column a0 values and output offsets, loaded for all heavy columns
@@ -916,7 +916,7 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
           const float w = wts ? __ldg(wts + e) : 1.0f;
           sth(P.val[l] + rb + ce + o, w / W, pf);
         }
-        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + ((u >> 5) << P.wsh)), "r"(1u << (u & 31)) : "memory");
+        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + (u >> 5)), "r"(1u << (u & 31)) : "memory");
         if (use_sum)
           asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (u >> 10)), "r"(1u << ((u >> 5) & 31)) : "memory");
       }
@@ -946,7 +946,8 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
   const int64_t j = c / ntile;
   const int t = (int)(c - j * ntile);
   const int64_t b = b0 + j;
-  unsigned long long* bm = P.bm + j * P.nwp;
+  const uint32_t* bm = P.bm + j * P.nwp;
+  int32_t* rank4 = P.rank4 + j * (P.nwp >> 2);
   const uint32_t* summ = P.summ + j * P.nsw;
   const bool sparse = P.use_sum[l];
   uint32_t wlo[WPT];
@@ -956,10 +957,12 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
   if (!sparse) {
     w0 = (int64_t)t * ROWS_TILE + (int64_t)threadIdx.x * WPT;
 #pragma unroll
-    for (int q = 0; q < WPT / 2; ++q) {
-      const ulonglong2 x = __ldcg((const ulonglong2*)(bm + w0) + q);
-      wlo[2 * q] = (uint32_t)x.x;
-      wlo[2 * q + 1] = (uint32_t)x.y;
+    for (int q = 0; q < WPT / 4; ++q) {
+      const uint4 x = __ldcg((const uint4*)(bm + w0) + q);
+      wlo[4 * q] = x.x;
+      wlo[4 * q + 1] = x.y;
+      wlo[4 * q + 2] = x.z;
+      wlo[4 * q + 3] = x.w;
     }
 #pragma unroll
     for (int q = 0; q < WPT; ++q) r += __popc(wlo[q]);
@@ -975,7 +978,7 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
       while (x) {
         const int bit = __ffs(x) - 1;
         x &= x - 1u;
-        r += __popc((uint32_t)__ldcg(bm + ((w0 + q) << 5) + bit));
+        r += __popc(__ldcg(bm + ((w0 + q) << 5) + bit));
       }
     }
   }
@@ -991,8 +994,13 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
   int32_t* row_map = P.row_map[l] + rb + tbase;
   const bool staged = tot <= ROW_STAGE;
   long long q0 = ex;  // rank of the thread's next row inside the tile
+  int64_t last_g = -1;  // a thread's words ascend and its range holds whole 4-word groups:
+                        // a group's first non-empty word starts the group's rank
   auto emit_word = [&](int64_t wi, uint32_t bits) {
-    bm[wi] = ((unsigned long long)(uint32_t)(tbase + q0) << 32) | bits;
+    if ((wi >> 2) != last_g) {
+      last_g = wi >> 2;
+      rank4[last_g] = (int32_t)(tbase + q0);
+    }
     while (bits) {
       const int bit = __ffs(bits) - 1;
       bits &= bits - 1u;
@@ -1013,7 +1021,7 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
         const int bit = __ffs(x) - 1;
         x &= x - 1u;
         const int64_t wi = ((w0 + q) << 5) + bit;
-        emit_word(wi, (uint32_t)__ldcg(bm + wi));
+        emit_word(wi, __ldcg(bm + wi));
       }
     }
   }
@@ -1036,7 +1044,8 @@ __global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, in
   const long long E = __ldcg((const long long*)P.meta + (b * P.L + l) * 8 + 2);
   const long long e0 = (long long)blockIdx.x * RL_TILE;
   if (e0 >= E) return;
-  const unsigned long long* bm = P.bm + j * P.nwp;
+  const uint4* bm4 = (const uint4*)(P.bm + j * P.nwp);
+  const int32_t* rank4 = P.rank4 + j * (P.nwp >> 2);
   int32_t* rl = P.row_local[l] + __ldg(P.bptr + b) * P.K[l];
   uint32_t u[RL_ILP];
 #pragma unroll
@@ -1044,16 +1053,27 @@ __global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, in
     const long long e = e0 + i * HB_THREADS + threadIdx.x;
     u[i] = e < E ? (uint32_t)__ldcs(rl + e) : 0u;
   }
-  unsigned long long w[RL_ILP];
+  // rank = the group's rank + set bits of the group before u: one 16-byte
+  // word group and one rank per edge (5 bytes per 32 nodes in all)
+  uint4 w[RL_ILP];
+  int32_t g[RL_ILP];
 #pragma unroll
   for (int i = 0; i < RL_ILP; ++i) {
     const long long e = e0 + i * HB_THREADS + threadIdx.x;
-    w[i] = e < E ? __ldcg(bm + (u[i] >> 5)) : 0ull;
+    w[i] = e < E ? __ldcg(bm4 + (u[i] >> 7)) : make_uint4(0, 0, 0, 0);
+    g[i] = e < E ? __ldcg(rank4 + (u[i] >> 7)) : 0;
   }
 #pragma unroll
   for (int i = 0; i < RL_ILP; ++i) {
     const long long e = e0 + i * HB_THREADS + threadIdx.x;
-    if (e < E) __stcs(rl + e, (int32_t)(w[i] >> 32) + __popc((uint32_t)w[i] & ((1u << (u[i] & 31)) - 1u)));
+    const int wq = (int)((u[i] >> 5) & 3);
+    const uint32_t below = (1u << (u[i] & 31)) - 1u;
+    int r = g[i];
+    r += wq > 0 ? __popc(w[i].x) : __popc(w[i].x & below);
+    if (wq >= 1) r += wq > 1 ? __popc(w[i].y) : __popc(w[i].y & below);
+    if (wq >= 2) r += wq > 2 ? __popc(w[i].z) : __popc(w[i].z & below);
+    if (wq == 3) r += __popc(w[i].w & below);
+    if (e < E) __stcs(rl + e, r);
   }
 }
 
@@ -1063,14 +1083,14 @@ __global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, in
 __global__ void __launch_bounds__(HB_THREADS) hop_clear_kernel(HopParams P, int l, int64_t b0) {
   const int64_t j = blockIdx.y;
   const int64_t b = b0 + j;
-  unsigned long long* bm = P.bm + j * P.nwp;
+  uint32_t* bm = P.bm + j * P.nwp;
   uint32_t* summ = P.summ + j * P.nsw;
   if (!P.use_sum[l]) {
     const int64_t t0 = (int64_t)blockIdx.x * CLEAR_TILE;
     if (t0 >= P.nw) return;
-    for (int q = 0; q < CLEAR_TILE / (2 * HB_THREADS); ++q) {
-      const int64_t w = t0 + ((int64_t)q * HB_THREADS + threadIdx.x) * 2;
-      *(ulonglong2*)(bm + w) = make_ulonglong2(0ull, 0ull);
+    for (int q = 0; q < CLEAR_TILE / (4 * HB_THREADS); ++q) {
+      const int64_t w = t0 + ((int64_t)q * HB_THREADS + threadIdx.x) * 4;
+      *(uint4*)(bm + w) = make_uint4(0, 0, 0, 0);
     }
     return;
   }
@@ -1078,7 +1098,7 @@ __global__ void __launch_bounds__(HB_THREADS) hop_clear_kernel(HopParams P, int 
   const int32_t* rows = P.row_map[l] + __ldg(P.bptr + b) * P.K[l];
   for (long long i = (long long)blockIdx.x * HB_THREADS + threadIdx.x; i < R; i += (long long)gridDim.x * HB_THREADS) {
     const uint32_t u = (uint32_t)__ldcg(rows + i);
-    bm[u >> 5] = 0ull;
+    bm[u >> 5] = 0u;
     summ[u >> 10] = 0u;
   }
 }
@@ -1156,7 +1176,6 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.nw = (g->num_nodes + 31) / 32;
   P.nwp = (P.nw + SPARSE_TILE - 1) / SPARSE_TILE * SPARSE_TILE;
   P.nsw = P.nwp / 32;
-  P.wsh = 1;
   P.sel_nq = 32;
   P.sel_claim = 2;
   P.sel_ld = 0;
@@ -1175,7 +1194,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     if (getenv("GS_HOP_DENSE")) P.use_sum[l] = 0;
     const int64_t tile = P.use_sum[l] ? SPARSE_TILE : ROWS_TILE;
     ntile[l] = (int)((P.nw + tile - 1) / tile);
-    foot = std::max(foot, P.use_sum[l] ? std::min(P.nw * 8, slots * 64) + P.nsw * 4 : P.nw * 8);
+    foot = std::max(foot, P.use_sum[l] ? std::min(P.nw * 5, slots * 48) + P.nsw * 4 : P.nw * 5);
   }
   blk->kind = gs_blocks::NODEWISE;
   blk->num_batches = nbatch;
@@ -1190,7 +1209,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   int64_t WB = std::max<int64_t>(1, budget / std::max<int64_t>(foot, 1));
   int64_t minwb = 64;
   if (const char* e = getenv("GS_HOP_MINWB")) minwb = std::max<int64_t>(1, atoll(e));
-  WB = std::max<int64_t>(WB, std::min<int64_t>(minwb, (int64_t(8) << 30) / std::max<int64_t>(P.nwp * 8, 1)));
+  WB = std::max<int64_t>(WB, std::min<int64_t>(minwb, (int64_t(8) << 30) / std::max<int64_t>(P.nwp * 5, 1)));
   WB = std::min<int64_t>(WB, MAX_GROUP);
   WB = std::min<int64_t>(WB, std::max<int64_t>(nbatch, 1));
   const int64_t G = nbatch > 0 ? (nbatch + WB - 1) / WB : 0;
@@ -1233,20 +1252,22 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   if (g_profiling || getenv("GS_HOP_TIMING")) NS = 1;
   // workspace: bitmaps + summaries (kept clear between calls), column staging
   const int64_t o_bm = 0;
-  const int64_t o_summ = a256h(o_bm + NS * WB * P.nwp * 8);
+  const int64_t o_summ = a256h(o_bm + NS * WB * P.nwp * 4);
   const int64_t o_coff = a256h(o_summ + NS * WB * P.nsw * 4);
   const int64_t o_dcol = a256h(o_coff + (maxcols + 64) * 8);
-  const int64_t ws_bytes = a256h(o_dcol + (maxcols + 64) * 4);
+  const int64_t o_rank = a256h(o_dcol + (maxcols + 64) * 4);  // not cleared: written before read
+  const int64_t ws_bytes = a256h(o_rank + NS * WB * (P.nwp / 4) * 4);
   const int64_t layout = o_coff;  // the cleared part
-  const bool fresh = blk->b_ws.bytes < (size_t)ws_bytes || blk->ws_kind_prev != 11 ||
+  const bool fresh = blk->b_ws.bytes < (size_t)ws_bytes || blk->ws_kind_prev != 12 ||
                      blk->ws_stride_prev != layout;
   if (!blk->b_ws.ensure(al, (size_t)ws_bytes, stream))
     return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (workspace)");
   if (fresh) GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, (size_t)layout, stream));
-  blk->ws_kind_prev = 11;
+  blk->ws_kind_prev = 12;
   blk->ws_stride_prev = layout;
   char* ws = (char*)blk->b_ws.ptr;
-  P.bm = (unsigned long long*)(ws + o_bm);
+  P.bm = (uint32_t*)(ws + o_bm);
+  P.rank4 = (int32_t*)(ws + o_rank);
   P.summ = (uint32_t*)(ws + o_summ);
   P.coff = (int64_t*)(ws + o_coff);
   P.dcol = (int32_t*)(ws + o_dcol);
@@ -1323,6 +1344,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     const int si = (int)(gi % NS);
     cudaStream_t stream = streams[si];
     P.bm = P0.bm + si * WB * P.nwp;
+    P.rank4 = P0.rank4 + si * WB * (P.nwp / 4);
     P.summ = P0.summ + si * WB * P.nsw;
     for (int l = 0; l < L; ++l) {
       unsigned int* c4 = ctr + (gi * L + l) * 4;
