@@ -79,8 +79,11 @@ struct HopParams {
   // workspace
   int64_t* coff;             // per frontier column: indptr[v] (column region of the hop)
   int32_t* dcol;             // per frontier column: in-degree (0 if the id is invalid)
-  uint32_t* bm;              // [group slot][nwp] row bitmap: one bit per node, 32-bit words
-  int32_t* rank4;            // [group slot][nwp / 4] rank of the first row of every non-empty 4-word group
+  uint32_t* bm;              // [group slot][nwp] row bitmap, 32-bit words in 4-word groups; lay 1: node
+                             // groups of 96 (hb_word), word 0 = the rank of the group's first row (row()),
+                             // words 1..3 = bits; lay 0: 128 nodes per group, bits only, ranks in rank4
+  int32_t* rank4;            // lay 0: [group slot][nwp / 4] rank of every non-empty group's first row
+  int lay;                   // bitmap layout (1: rank inside the group -- one load per relabelled edge)
   uint32_t* summ;            // [group slot][nsw] bit w set iff bitmap word w is non-empty
   int64_t nw, nwp, nsw;      // words used / allocated per batch, summary words
   int sel_nq, sel_claim;     // select: claim queues, chunks per claim
@@ -89,6 +92,19 @@ struct HopParams {
   int ares_tau;              // hop_ares_big_kernel's first threshold: 0 normal, 1 too tight,
                              // 2 too loose (tests: every widen / narrow step runs)
 };
+
+// Row bitmap layout: node u lives in 16-byte group g = u / 96, bit word
+// 1 + (u % 96) / 32 of it; word 0 of the group holds the rank of the group's
+// first row once row() ran, so relabel reads one 16-byte group per edge.
+constexpr uint32_t HB_GNODES = 96;
+__device__ __forceinline__ uint32_t hb_word(uint32_t u) {
+  const uint32_t g = u / HB_GNODES;
+  return g * 4u + 1u + ((u - g * HB_GNODES) >> 5);
+}
+__device__ __forceinline__ uint32_t hb_bit(uint32_t u) { return 1u << ((u - (u / HB_GNODES) * HB_GNODES) & 31); }
+// the word and bit of node u in either layout
+__device__ __forceinline__ uint32_t hb_wd(int lay, uint32_t u) { return lay ? hb_word(u) : (u >> 5); }
+__device__ __forceinline__ uint32_t hb_bt(int lay, uint32_t u) { return lay ? hb_bit(u) : 1u << (u & 31); }
 
 // Per-launch scan bookkeeping of nprep / rows (zeroed before the launch):
 // ticket counter + one look-back status word per (batch, segment).
@@ -626,11 +642,10 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
               C.sv[pre + i] = w / csum;
             }
           }
-          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + (u[q] >> 5)), "r"(1u << (u[q] & 31))
-                       : "memory");
+          const uint32_t wd = hb_wd(P.lay, u[q]);
+          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + wd), "r"(hb_bt(P.lay, u[q])) : "memory");
           if (use_sum)
-            asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (u[q] >> 10)), "r"(1u << ((u[q] >> 5) & 31))
-                         : "memory");
+            asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (wd >> 5)), "r"(1u << (wd & 31)) : "memory");
         }
       }
     }
@@ -916,9 +931,10 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
           const float w = wts ? __ldg(wts + e) : 1.0f;
           sth(P.val[l] + rb + ce + o, w / W, pf);
         }
-        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + (u >> 5)), "r"(1u << (u & 31)) : "memory");
+        const uint32_t wd = hb_wd(P.lay, u);
+        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + wd), "r"(hb_bt(P.lay, u)) : "memory");
         if (use_sum)
-          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (u >> 10)), "r"(1u << ((u >> 5) & 31)) : "memory");
+          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (wd >> 5)), "r"(1u << (wd & 31)) : "memory");
       }
     }
   }
@@ -946,8 +962,9 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
   const int64_t j = c / ntile;
   const int t = (int)(c - j * ntile);
   const int64_t b = b0 + j;
-  const uint32_t* bm = P.bm + j * P.nwp;
+  uint32_t* bm = P.bm + j * P.nwp;
   int32_t* rank4 = P.rank4 + j * (P.nwp >> 2);
+  const int lay = P.lay;
   const uint32_t* summ = P.summ + j * P.nsw;
   const bool sparse = P.use_sum[l];
   uint32_t wlo[WPT];
@@ -964,6 +981,9 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
       wlo[4 * q + 2] = x.z;
       wlo[4 * q + 3] = x.w;
     }
+#pragma unroll
+    for (int q = 0; q < WPT; q += 4)
+      if (lay) wlo[q] = 0u;  // the groups' rank words (a thread owns whole groups)
 #pragma unroll
     for (int q = 0; q < WPT; ++q) r += __popc(wlo[q]);
   } else {
@@ -994,17 +1014,19 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
   int32_t* row_map = P.row_map[l] + rb + tbase;
   const bool staged = tot <= ROW_STAGE;
   long long q0 = ex;  // rank of the thread's next row inside the tile
-  int64_t last_g = -1;  // a thread's words ascend and its range holds whole 4-word groups:
+  int64_t last_g = -1;  // a thread's words ascend and its range holds whole groups:
                         // a group's first non-empty word starts the group's rank
   auto emit_word = [&](int64_t wi, uint32_t bits) {
     if ((wi >> 2) != last_g) {
       last_g = wi >> 2;
-      rank4[last_g] = (int32_t)(tbase + q0);
+      if (lay) bm[last_g << 2] = (uint32_t)(tbase + q0);
+      else rank4[last_g] = (int32_t)(tbase + q0);
     }
     while (bits) {
       const int bit = __ffs(bits) - 1;
       bits &= bits - 1u;
-      const uint32_t u = (uint32_t)((wi << 5) + bit);
+      const uint32_t u = lay ? (uint32_t)((wi >> 2) * HB_GNODES + (((wi & 3) - 1) << 5) + bit)
+                             : (uint32_t)((wi << 5) + bit);
       if (staged) stage[q0] = u;
       else row_map[q0] = (int32_t)u;
       ++q0;
@@ -1046,6 +1068,7 @@ __global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, in
   if (e0 >= E) return;
   const uint4* bm4 = (const uint4*)(P.bm + j * P.nwp);
   const int32_t* rank4 = P.rank4 + j * (P.nwp >> 2);
+  const int lay = P.lay;
   int32_t* rl = P.row_local[l] + __ldg(P.bptr + b) * P.K[l];
   uint32_t u[RL_ILP];
 #pragma unroll
@@ -1053,8 +1076,30 @@ __global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, in
     const long long e = e0 + i * HB_THREADS + threadIdx.x;
     u[i] = e < E ? (uint32_t)__ldcs(rl + e) : 0u;
   }
-  // rank = the group's rank + set bits of the group before u: one 16-byte
-  // word group and one rank per edge (5 bytes per 32 nodes in all)
+  // rank = the group's rank word + the set bits of the group before u: one
+  // 16-byte load per edge (16 bytes per 96 nodes in all)
+  // (lay 0: the group's 128 nodes' bits + a separate rank load)
+  if (lay) {
+    uint4 w[RL_ILP];
+#pragma unroll
+    for (int i = 0; i < RL_ILP; ++i) {
+      const long long e = e0 + i * HB_THREADS + threadIdx.x;
+      w[i] = e < E ? __ldcg(bm4 + u[i] / HB_GNODES) : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int i = 0; i < RL_ILP; ++i) {
+      const long long e = e0 + i * HB_THREADS + threadIdx.x;
+      const uint32_t o = u[i] - (u[i] / HB_GNODES) * HB_GNODES;  // offset in the group
+      const int wq = (int)(o >> 5);
+      const uint32_t below = (1u << (o & 31)) - 1u;
+      int r = (int)w[i].x;
+      r += wq > 0 ? __popc(w[i].y) : __popc(w[i].y & below);
+      if (wq >= 1) r += wq > 1 ? __popc(w[i].z) : __popc(w[i].z & below);
+      if (wq == 2) r += __popc(w[i].w & below);
+      if (e < E) __stcs(rl + e, r);
+    }
+    return;
+  }
   uint4 w[RL_ILP];
   int32_t g[RL_ILP];
 #pragma unroll
@@ -1098,8 +1143,9 @@ __global__ void __launch_bounds__(HB_THREADS) hop_clear_kernel(HopParams P, int 
   const int32_t* rows = P.row_map[l] + __ldg(P.bptr + b) * P.K[l];
   for (long long i = (long long)blockIdx.x * HB_THREADS + threadIdx.x; i < R; i += (long long)gridDim.x * HB_THREADS) {
     const uint32_t u = (uint32_t)__ldcg(rows + i);
-    bm[u >> 5] = 0u;
-    summ[u >> 10] = 0u;
+    const uint32_t wd = hb_wd(P.lay, u);
+    bm[wd] = 0u;
+    summ[wd >> 5] = 0u;
   }
 }
 
@@ -1173,7 +1219,13 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   }
   // bitmap geometry: nwp words per batch slot (whole summary-mode tiles); a
   // hop is sparse (summary mode) when its slots are few against the words
-  P.nw = (g->num_nodes + 31) / 32;
+  // layout 1 (rank inside each 96-node group: one load per relabelled edge)
+  // for graphs whose per-batch bitmaps stay small; layout 0 (bits only, a
+  // rank per 128 nodes beside them) above 2^24 nodes, where sparse row()
+  // measured 5x slower in layout 1 (PP hop 2: 78 vs 14.6 ms)
+  P.lay = g->num_nodes <= (int64_t(1) << 24) ? 1 : 0;
+  if (const char* e = getenv("GS_HOP_LAYOUT")) P.lay = atoi(e) ? 1 : 0;
+  P.nw = P.lay ? (g->num_nodes + HB_GNODES - 1) / HB_GNODES * 4 : (g->num_nodes + 31) / 32;
   P.nwp = (P.nw + SPARSE_TILE - 1) / SPARSE_TILE * SPARSE_TILE;
   P.nsw = P.nwp / 32;
   P.sel_nq = 32;
@@ -1194,7 +1246,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     if (getenv("GS_HOP_DENSE")) P.use_sum[l] = 0;
     const int64_t tile = P.use_sum[l] ? SPARSE_TILE : ROWS_TILE;
     ntile[l] = (int)((P.nw + tile - 1) / tile);
-    foot = std::max(foot, P.use_sum[l] ? std::min(P.nw * 5, slots * 48) + P.nsw * 4 : P.nw * 5);
+    foot = std::max(foot, P.use_sum[l] ? std::min(P.nw * 5, slots * 48) + P.nsw * 4 : P.nw * (P.lay ? 4 : 5));
   }
   blk->kind = gs_blocks::NODEWISE;
   blk->num_batches = nbatch;
@@ -1256,14 +1308,14 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   const int64_t o_coff = a256h(o_summ + NS * WB * P.nsw * 4);
   const int64_t o_dcol = a256h(o_coff + (maxcols + 64) * 8);
   const int64_t o_rank = a256h(o_dcol + (maxcols + 64) * 4);  // not cleared: written before read
-  const int64_t ws_bytes = a256h(o_rank + NS * WB * (P.nwp / 4) * 4);
+  const int64_t ws_bytes = a256h(o_rank + (P.lay ? 256 : NS * WB * (P.nwp / 4) * 4));
   const int64_t layout = o_coff;  // the cleared part
-  const bool fresh = blk->b_ws.bytes < (size_t)ws_bytes || blk->ws_kind_prev != 12 ||
+  const bool fresh = blk->b_ws.bytes < (size_t)ws_bytes || blk->ws_kind_prev != 15 + P.lay ||
                      blk->ws_stride_prev != layout;
   if (!blk->b_ws.ensure(al, (size_t)ws_bytes, stream))
     return fail(GS_ERR_OUT_OF_MEMORY, "device allocation failed (workspace)");
   if (fresh) GS_CUDA_TRY(cudaMemsetAsync(blk->b_ws.ptr, 0, (size_t)layout, stream));
-  blk->ws_kind_prev = 12;
+  blk->ws_kind_prev = 15 + P.lay;
   blk->ws_stride_prev = layout;
   char* ws = (char*)blk->b_ws.ptr;
   P.bm = (uint32_t*)(ws + o_bm);
@@ -1344,7 +1396,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
     const int si = (int)(gi % NS);
     cudaStream_t stream = streams[si];
     P.bm = P0.bm + si * WB * P.nwp;
-    P.rank4 = P0.rank4 + si * WB * (P.nwp / 4);
+    if (!P.lay) P.rank4 = P0.rank4 + si * WB * (P.nwp / 4);
     P.summ = P0.summ + si * WB * P.nsw;
     for (int l = 0; l < L; ++l) {
       unsigned int* c4 = ctr + (gi * L + l) * 4;

@@ -179,3 +179,19 @@ def test_pack_matches_views(gs, medium, kind, narrow):
             assert torch.equal(pk["row_map"][r:r + nr], v["row_map"])
             e, i, r = e + ne, i + nc, r + nr
         assert tot == [e, i, r]
+
+
+@pytest.mark.parametrize("layout", ["0", "1"])
+@pytest.mark.parametrize("fan", [[25, 10], [15, 10, 5]])
+def test_row_bitmap_layouts(gs, oracle_lib, medium, fan, layout, monkeypatch):
+    """Both row-bitmap layouts of the node-wise engine (GS_HOP_LAYOUT: 1 = the
+    rank inside each 96-node group, the default below 2^24 nodes; 0 = bits
+    only with a rank per 128 nodes beside them, the default above), uniform and
+    weighted, against the oracle."""
+    monkeypatch.setenv("GS_HOP_LAYOUT", layout)
+    g, G, O = medium
+    seeds = synth.make_seeds(synth.GraphSpec("m", g["indptr"].numel() - 1, 1, True, None, 31), 3000)
+    for bias in (0, 1):
+        out = gs.sample_neighbors(G, seeds.cuda(), fan, batch_size=512, bias_mode=bias, rng_key=12).to_host()
+        ref = oracle_lib.sample_neighbors(O, seeds.numpy(), fan, batch_size=512, bias_mode=bias, rng_key=12)
+        compare_all(out, ref, f"layout {layout} bias {bias} fan {fan}")
