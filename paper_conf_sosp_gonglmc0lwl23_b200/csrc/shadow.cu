@@ -399,6 +399,13 @@ static gs_status induce_envelope(int64_t N, int* CS_out, int64_t* bpc_out) {
   if (CS > SH_MAX_CS)
     return fail(GS_ERR_NOT_SUPPORTED, "induce: N = %lld exceeds the shared-memory bitmap envelope (%lld nodes)",
                 (long long)N, (long long)(SH_MAX_CS * (SH_SMEM_CAP * 64 / 11)));
+  if (const char* e = getenv("GS_SH_CS")) {  // tests: a larger cluster than the graph needs
+    const int want = atoi(e);
+    while (CS < want && CS < SH_MAX_CS) {
+      CS *= 2;
+      bpc = ((N + CS - 1) / CS + 255) / 256 * 256;
+    }
+  }
   *CS_out = CS;
   *bpc_out = bpc;
   return GS_OK;

@@ -135,13 +135,17 @@ def test_shard_invariance(gs, medium):
         compare_all(part, full[lo // 500: hi // 500 + (1 if hi % 500 else 0)], "shard")
 
 
+@pytest.mark.parametrize("cs", [None, "2", "4"])
 @pytest.mark.parametrize("wcap", [None, "40"])
 @pytest.mark.parametrize("mode", [0, 1])
-def test_shadow(gs, oracle_lib, medium, mode, wcap, monkeypatch):
+def test_shadow(gs, oracle_lib, medium, mode, wcap, cs, monkeypatch):
     """ShaDow vs the oracle; wcap = 40 shrinks the induce kernel's per-warp
-    staging so that most columns take the re-stream path."""
+    staging so that most columns take the re-stream path; cs forces a 2- or
+    4-CTA cluster (the U bitmap split across peers' shared memory)."""
     if wcap:
         monkeypatch.setenv("GS_SH_WCAP", wcap)
+    if cs:
+        monkeypatch.setenv("GS_SH_CS", cs)
     g, G, O = medium
     seeds = synth.make_seeds(synth.GraphSpec("m", 200_000, 1, True, None, 6), 1000)
     out = gs.sample_shadow(G, seeds.cuda(), [10, 5], batch_size=256, bias_mode=mode,

@@ -55,12 +55,15 @@ def test_saint_dead_end_roots(gs, oracle_lib, tiny):
     compare_all(out, [[r] for r in ref], "saint dead ends")
 
 
+@pytest.mark.parametrize("cs", [None, "2"])
 @pytest.mark.parametrize("wcap", [None, "40"])
-def test_saint_medium(gs, oracle_lib, medium, wcap, monkeypatch):
+def test_saint_medium(gs, oracle_lib, medium, wcap, cs, monkeypatch):
     """wcap = 40 shrinks the induce kernel's per-warp staging so that most
-    columns take the re-stream path."""
+    columns take the re-stream path; cs = 2 forces a 2-CTA cluster."""
     if wcap:
         monkeypatch.setenv("GS_SH_WCAP", wcap)
+    if cs:
+        monkeypatch.setenv("GS_SH_CS", cs)
     g, G, O = medium
     roots = synth.make_seeds(synth.GraphSpec("m", 200_000, 1, True, None, 6), 7000)
     out = gs.sample_saint_rw(G, roots.cuda(), 3, batch_size=3000, rng_key=23).to_host()
