@@ -172,3 +172,19 @@ def test_ladies_hub_frontiers(gs, oracle_lib, hubby, lw_path):
     ref = oracle_lib.sample_layerwise(O, seeds.numpy(), [512, 256, 512], batch_size=512, prob_mode=0,
                                       rng_key=8)
     compare_all(out.to_host(), ref, "ladies hub frontiers")
+
+
+def test_ladies_zero_weights(gs, oracle_lib, ljlike):
+    """A third of the edge weights set to zero: rows whose b(u) = sum w^2 is 0
+    are ineligible (R6, R24), rows mixing zero and non-zero edges keep their
+    positive b -- every kernel against the oracle."""
+    g, G, O = ljlike
+    w = g["weights"].clone()
+    w[torch.arange(w.numel(), device=w.device) % 3 == 0] = 0.0
+    Gz = gs.Graph(g["indptr"], g["indices"], w)
+    Oz = oracle_lib.Graph(g["indptr"].cpu().numpy(), g["indices"].cpu().numpy(), w.cpu().numpy())
+    seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 41), 2500)
+    for K in (64, 512):
+        out = gs.sample_layerwise(Gz, seeds.cuda(), [K, K], batch_size=500, prob_mode=0, rng_key=K + 1)
+        ref = oracle_lib.sample_layerwise(Oz, seeds.numpy(), [K, K], batch_size=500, prob_mode=0, rng_key=K + 1)
+        compare_all(out.to_host(), ref, f"ladies zero weights K={K}")
