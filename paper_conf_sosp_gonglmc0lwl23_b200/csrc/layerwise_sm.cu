@@ -224,21 +224,10 @@ __device__ __forceinline__ void ls_tau_from_hist(const int32_t* hist, int target
 
 // Flat edge e -> its frontier column: the column of e's 2^gsh-edge block's
 // first edge, then a binary search up to the next block's.
-__device__ __forceinline__ int ls_col2(const int32_t* cstart, const int16_t* colblk, int gsh, int nblk, int T,
+__device__ __forceinline__ int ls_col(const int32_t* cstart, const int16_t* colblk, int gsh, int nblk, int T,
                                        int e) {
   const int bk = e >> gsh;
   int lo = colblk[bk], hi = bk + 1 < nblk ? colblk[bk + 1] : T - 1;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (cstart[mid] <= e) lo = mid;
-    else hi = mid - 1;
-  }
-  return lo;
-}
-
-// Flat edge e -> its frontier column (binary search of the column starts).
-__device__ __forceinline__ int ls_col(const int32_t* cstart, int T, int e) {
-  int lo = 0, hi = T - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
     if (cstart[mid] <= e) lo = mid;
@@ -380,7 +369,7 @@ __global__ void __launch_bounds__(LS_THREADS, 1) layerwise_sm_kernel(LSParams P)
           u[q] = LS_EMPTY;
           w2[q] = 0.0f;
           if (e < nflat) {
-            const int c = ls_col2(sm.cstart, sm.colblk, gsh, nblk, T, e);
+            const int c = ls_col(sm.cstart, sm.colblk, gsh, nblk, T, e);
             const int64_t pos = sm.off[c] + (e - sm.cstart[c]);
             u[q] = (uint32_t)__ldg(P.indices + pos);
             if (ladies && wts) {
@@ -630,7 +619,7 @@ __global__ void __launch_bounds__(LS_THREADS, 1) layerwise_sm_kernel(LSParams P)
           const int lid = ls_find_s(sm.key, u[q]);
           if (lid < 0) continue;
           const int e = ci * LS_CH + q * LS_THREADS + t;
-          const int c = ls_col2(sm.cstart, sm.colblk, gsh, nblk, T, e);
+          const int c = ls_col(sm.cstart, sm.colblk, gsh, nblk, T, e);
           const int64_t pos = sm.off[c] + (e - sm.cstart[c]);
           const float w = wts ? __ldg(P.weights + pos) : 1.0f;
           const float a = __fdiv_rn(w, sm.sp[lid]);
@@ -697,7 +686,7 @@ __global__ void __launch_bounds__(LS_THREADS, 1) layerwise_sm_kernel(LSParams P)
           if (!kq) continue;
           const long long o = ebase + run + sm.wpre[q * LS_WARPS + warp] + __popc(bal & ((1u << lane) - 1u));
           const int e = ci * LS_CH + q * LS_THREADS + t;
-          const int c = ls_col2(sm.cstart, sm.colblk, gsh, nblk, T, e);
+          const int c = ls_col(sm.cstart, sm.colblk, gsh, nblk, T, e);
           P.row_local[l][o] = (int32_t)u[q];
           P.eid[l][o] = sm.off[c] + (e - sm.cstart[c]);
           P.val[l][o] = __fdiv_rn(w2[q], (float)sm.cs[c]);
