@@ -117,7 +117,7 @@ struct LSSmem {
   float sp[LS_MAXK];
   int32_t wpre[LS_CHMAX / 32];
   int16_t colblk[LS_NBLK];
-  double scr[40];
+  double scr[72];
   long long misc[8];
   int imisc[8];
   float ftau;
@@ -234,6 +234,29 @@ __device__ __forceinline__ int ls_col(const int32_t* cstart, const int16_t* colb
     else hi = mid - 1;
   }
   return lo;
+}
+
+// Block-wide sums of two doubles in one pass (scratch >= 66 doubles).
+__device__ __forceinline__ void ls_reduce2(double& a, double& b, double* scr) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    a += __shfl_xor_sync(0xffffffffu, a, o);
+    b += __shfl_xor_sync(0xffffffffu, b, o);
+  }
+  if (lane == 0) {
+    scr[wid] = a;
+    scr[32 + wid] = b;
+  }
+  __syncthreads();
+  double sa = 0.0, sb = 0.0;
+  for (int w = 0; w < nw; ++w) {  // every thread sums the warps' partials in the same order
+    sa += scr[w];
+    sb += scr[32 + w];
+  }
+  __syncthreads();
+  a = sa;
+  b = sb;
 }
 
 // Counting-sort rank of n <= LS_SCAP items (bin(i) monotone in the order,
@@ -511,8 +534,10 @@ __global__ void __launch_bounds__(LS_THREADS, 1) layerwise_sm_kernel(LSParams P)
         }
         const bool ovf = sm.imisc[2] != 0;
         if (build && !ovf && !haveB) {
-          Btot = block_reduce_sum<double>(bsum, sm.scr);
-          nelig = (int)block_reduce_sum<long long>((long long)elig, scrl);
+          double e2 = (double)elig;  // B and the eligible count in one reduction
+          ls_reduce2(bsum, e2, sm.scr);
+          Btot = bsum;
+          nelig = (int)e2;
           haveB = true;
         }
         ncand = sm.imisc[0];
@@ -556,14 +581,19 @@ __global__ void __launch_bounds__(LS_THREADS, 1) layerwise_sm_kernel(LSParams P)
       // ---- D: the K smallest (key, u) of the survivors, then S ascending ----
       if (done && nsel > 0) {
         if (nsel < ncand) {
-          double km = 0.0;
-          for (int i = t; i < ncand; i += LS_THREADS) km = fmax(km, sm.skey[i]);
-          for (int o = 16; o > 0; o >>= 1) km = fmax(km, __shfl_xor_sync(0xffffffffu, km, o));
-          if (lane == 0) sm.scr[warp] = km;
-          __syncthreads();
-          double kmax = 0.0;
-          for (int w = 0; w < LS_WARPS; ++w) kmax = fmax(kmax, sm.scr[w]);
-          __syncthreads();
+          // the survivors' keys lie below tau (the key bins' range); without a
+          // threshold, below their maximum
+          double kmax = (double)tau;
+          if (!(tau > 0.0f)) {
+            double km = 0.0;
+            for (int i = t; i < ncand; i += LS_THREADS) km = fmax(km, sm.skey[i]);
+            for (int o = 16; o > 0; o >>= 1) km = fmax(km, __shfl_xor_sync(0xffffffffu, km, o));
+            if (lane == 0) sm.scr[warp] = km;
+            __syncthreads();
+            kmax = 0.0;
+            for (int w = 0; w < LS_WARPS; ++w) kmax = fmax(kmax, sm.scr[w]);
+            __syncthreads();
+          }
           const double scale = kmax > 0.0 ? (double)(LS_NB - 1) / kmax : 0.0;
           ls_rank<LS_THREADS>(
               ncand, d_hist, d_fill, d_ord, d_rank,
