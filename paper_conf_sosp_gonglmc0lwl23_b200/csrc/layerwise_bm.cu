@@ -52,6 +52,7 @@ constexpr int LB_ILP = 4;           // flat edges per thread in flight
 constexpr int LB_ILP5 = 8;          // ... in the finalize re-stream (L5a)
 constexpr int LB_MAX_K = 4096;
 constexpr int LB_SCAP = 512;        // kept edges a warp stages in L5a (more: L5b streams again)
+constexpr int LB_CCAP = 512;        // FastGCN: candidate-row edges a warp stages in L1 (more: L5a streams again)
 
 struct LBParams {
   const int64_t* indptr;
@@ -88,6 +89,10 @@ struct LBParams {
   int32_t* stg_col;
   float* stg_a;
   int scap;                         // staged kept edges per warp (<= LB_SCAP)
+  int64_t* cnd_pos;                 // [CTA][warp][LB_CCAP] FastGCN: L1's edges whose row's key is below
+  int32_t* cnd_u;                   //   the previous batch's threshold: position, row, column
+  int32_t* cnd_col;
+  int ccap;
   int gw_log;                       // log2 words per rank group (>= 2)
   int ng;                           // rank groups per bitmap
   int maxT;
@@ -100,6 +105,8 @@ struct LBShared {
   unsigned long long u64[4];
   double tau_est[MAX_LAYERS];       // FastGCN: select threshold estimate per layer (previous batch)
   int wtot[LB_WARPS];
+  int cfill[LB_WARPS];              // FastGCN: candidate-row edges each warp staged in L1
+  int cstage_ovf;
 };
 
 __device__ __forceinline__ int lb_col(const int32_t* fstart, int T, int64_t e) {
@@ -426,22 +433,35 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       const double tau_est = degree ? sh.tau_est[l] : 0.0;
       const float tau_f = (float)tau_est;
       const bool l1_deg = degree && P.degsrc != nullptr;
+      // FastGCN with a threshold: every edge whose row's key is below it is
+      // staged (position, row, column) in its warp's region, in flat order, so
+      // the finalize filters those (~0.5% of the edges) instead of streaming
+      // A[:, F] again (the selected rows all have keys below the threshold)
+      const bool cstage = l1_deg && tau_est > 0.0 && P.ccap > 0;
       unsigned long long l1_b = 0, l1_e = 0;
-      if (threadIdx.x == 0) sh.misc[6] = 0;
+      int cfill = 0;
+      const int64_t creg = ((int64_t)blockIdx.x * LB_WARPS + (threadIdx.x >> 5)) * LB_CCAP;
+      if (threadIdx.x == 0) {
+        sh.misc[6] = 0;
+        sh.cstage_ovf = 0;
+      }
       __syncthreads();
       {
         LBStream st(nflat);
         for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
           uint32_t u[LB_ILP];
           int32_t dg[LB_ILP];
+          int cc[LB_ILP];
 #pragma unroll
           for (int q = 0; q < LB_ILP; ++q) {
             const int64_t e = e0 + 32 * q + lane;
             u[q] = 0xFFFFFFFFu;
             dg[q] = 0;
+            cc[q] = 0;
             if (e < st.end) {
               const int c = st.col(s_fstart, Ti, e);
               const int64_t pos = s_off[c] + (e - s_fstart[c]);
+              cc[q] = c;
               u[q] = (uint32_t)__ldg(P.indices + pos);
               if (l1_deg) dg[q] = __ldg(P.degsrc + pos);
             }
@@ -449,30 +469,61 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
 #pragma unroll
           for (int q = 0; q < LB_ILP; ++q) {
             const uint32_t peers = __match_any_sync(0xffffffffu, u[q]);
-            if (u[q] == 0xFFFFFFFFu || (__ffs(peers) - 1) != lane) continue;
+            const int leader = __ffs(peers) - 1;
+            const bool valid = u[q] != 0xFFFFFFFFu;
             const uint32_t bit = 1u << (u[q] & 31);
-            if (!l1_deg) {
-              atomicOr(bm + (u[q] >> 5), bit);
-              continue;
+            bool cand = false;
+            if (valid && leader == lane) {
+              if (!l1_deg) {
+                atomicOr(bm + (u[q] >> 5), bit);
+              } else {
+                const bool is_new = !(atomicOr(bm + (u[q] >> 5), bit) & bit);
+                if (is_new) {
+                  l1_b += (unsigned long long)dg[q];
+                  l1_e += dg[q] > 0 ? 1 : 0;
+                }
+                // the row's key against the threshold: new rows join the fused
+                // pool; every row's edges are staged when it is below
+                if (dg[q] > 0 && tau_est > 0.0 && (is_new || cstage)) {
+                  const float bb = (float)dg[q];
+                  const uint32_t R = philox_k(u[q], 0u, ctr2(l, TAG_ARES_LAYER), gb, P.pk).x;
+                  if (ares_maybe_below(R, __fmul_rn(__fmul_rn(tau_f, bb), 1.01f))) {
+                    const double kk = ares_key(R, (double)bb);
+                    if (kk < tau_est) {
+                      cand = true;
+                      if (is_new) {
+                        const int slot = atomicAdd(&sh.misc[6], 1);
+                        if (slot < LB_CAP) {
+                          s_bk[slot] = (unsigned long long)__double_as_longlong(kk);
+                          s_bu[slot] = u[q];
+                          s_bb[slot] = bb;
+                        }
+                      }
+                    }
+                  }
+                }
+              }
             }
-            if (atomicOr(bm + (u[q] >> 5), bit) & bit) continue;  // not new
-            l1_b += (unsigned long long)dg[q];
-            if (dg[q] <= 0) continue;
-            ++l1_e;
-            if (!(tau_est > 0.0)) continue;
-            const float bb = (float)dg[q];
-            const uint32_t R = philox_k(u[q], 0u, ctr2(l, TAG_ARES_LAYER), gb, P.pk).x;
-            if (!ares_maybe_below(R, __fmul_rn(__fmul_rn(tau_f, bb), 1.01f))) continue;
-            const double kk = ares_key(R, (double)bb);
-            if (!(kk < tau_est)) continue;
-            const int slot = atomicAdd(&sh.misc[6], 1);
-            if (slot < LB_CAP) {
-              s_bk[slot] = (unsigned long long)__double_as_longlong(kk);
-              s_bu[slot] = u[q];
-              s_bb[slot] = bb;
+            if (cstage) {
+              cand = __shfl_sync(0xffffffffu, cand, leader) && valid;  // the row's verdict, for every edge of it
+              const unsigned bal = __ballot_sync(0xffffffffu, cand);
+              if (bal) {
+                const int idx = cfill + __popc(bal & ((1u << lane) - 1u));
+                if (cand && idx < P.ccap) {
+                  const int64_t e = e0 + 32 * q + lane;
+                  P.cnd_pos[creg + idx] = s_off[cc[q]] + (e - s_fstart[cc[q]]);
+                  P.cnd_u[creg + idx] = (int32_t)u[q];
+                  P.cnd_col[creg + idx] = cc[q];
+                }
+                cfill += __popc(bal);
+              }
             }
           }
         }
+      }
+      if (cstage && lane == 0) {
+        sh.cfill[threadIdx.x >> 5] = cfill;
+        if (cfill > P.ccap) sh.cstage_ovf = 1;
       }
       __syncthreads();
 
@@ -683,7 +734,32 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       float* stg_a = P.stg_a + sreg;
       if (threadIdx.x == 0) sh.misc[7] = 0;
       __syncthreads();
-      {
+      if (cstage && skip_ranks && !sh.cstage_ovf) {
+        // the kept edges are among L1's staged candidate-row edges (flat order)
+        const int n = sh.cfill[threadIdx.x >> 5];
+        for (int i0 = 0; i0 < n && nsel > 0; i0 += 32) {
+          const int i = i0 + lane;
+          const uint32_t uu = i < n ? (uint32_t)P.cnd_u[creg + i] : 0xFFFFFFFFu;
+          const int lid = uu == 0xFFFFFFFFu ? -1 : lb_lookup(s_hk, s_hv, uu);
+          const unsigned bal = __ballot_sync(0xffffffffu, lid >= 0);
+          if (lid >= 0) {
+            const int64_t pos = P.cnd_pos[creg + i];
+            const int c = P.cnd_col[creg + i];
+            const float w = P.weights ? __ldg(P.weights + pos) : 1.0f;
+            const float a = __fdiv_rn(w, __uint_as_float((uint32_t)s_sel[lid]));
+            atomicAdd(&s_cnt[c], 1);
+            atomicAdd(&s_cs[c], (double)a);
+            const int idx = wkept + __popc(bal & ((1u << lane) - 1u));
+            if (idx < P.scap) {
+              stg_pos[idx] = pos;
+              stg_lid[idx] = lid;
+              stg_col[idx] = c;
+              stg_a[idx] = a;
+            }
+          }
+          wkept += __popc(bal);
+        }
+      } else {
         LBStream st(nflat);
         for (int64_t e0 = st.beg; e0 < st.end && nsel > 0; e0 += 32 * LB_ILP5) {
           uint32_t u[LB_ILP5];
@@ -934,7 +1010,8 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.acc_cap = prob_mode == GS_PROB_DEGREE ? 0 : std::max<int64_t>(int64_t(1) << 15, blk->lw_tab_hint);
   const int64_t bm_bytes = a256(n4 * 16);
   const int64_t acc_bytes = a256(P.acc_cap * 8);
-  const int64_t stg_bytes = a256((int64_t)LB_WARPS * LB_SCAP * (8 + 4 + 4 + 4));
+  const int64_t stg_bytes = a256((int64_t)LB_WARPS * LB_SCAP * (8 + 4 + 4 + 4)) +
+                            a256((int64_t)LB_WARPS * LB_CCAP * (8 + 4 + 4));
   const int64_t stride = bm_bytes + acc_bytes + stg_bytes;
   const size_t ws_bytes = (size_t)stride * nctas;
   const bool grow = blk->b_ws.bytes < ws_bytes;
@@ -956,7 +1033,14 @@ gs_status run_layerwise_bm(const gs_graph* g, const int32_t* seeds, int64_t num_
     P.stg_lid = (int32_t*)(sb + ne * 8);
     P.stg_col = (int32_t*)(sb + ne * 12);
     P.stg_a = (float*)(sb + ne * 16);
+    char* cb = sb + a256(ne * 20);
+    const int64_t nc = (int64_t)nctas * LB_WARPS * LB_CCAP;
+    P.cnd_pos = (int64_t*)cb;
+    P.cnd_u = (int32_t*)(cb + nc * 8);
+    P.cnd_col = (int32_t*)(cb + nc * 12);
   }
+  P.ccap = prob_mode == GS_PROB_DEGREE ? LB_CCAP : 0;
+  if (const char* e = getenv("GS_LW_CCAP")) P.ccap = std::max(0, std::min(atoi(e), LB_CCAP));  // tests
   P.col0 = (int32_t*)blk->b_col[0].ptr;
   for (int l = 0; l < L; ++l) {
     P.row_map[l] = (int32_t*)blk->b_row[l].ptr;

@@ -104,13 +104,18 @@ def test_ladies_bias_capacity_retry(gs, oracle_lib, ljlike):
     compare_all(out.to_host(), ref, "ladies big")
 
 
-def test_fastgcn_threshold_reuse(gs, oracle_lib, ljlike, monkeypatch, lw_path):
+@pytest.mark.parametrize("ccap", [None, "3", "0"])
+def test_fastgcn_threshold_reuse(gs, oracle_lib, ljlike, monkeypatch, lw_path, ccap):
     """One CTA walks every batch, so from the second batch on the bitmap
-    kernel's rank pass filters against the previous batch's threshold (the
-    fused select); the result must not depend on it."""
+    kernel's extract filters against the previous batch's threshold (the
+    fused select) and stages the candidate rows' edges for the finalize; the
+    result must not depend on it (ccap 3: most warps overflow their staging and
+    stream A[:, F] again; 0: no staging)."""
     if lw_path != "bm":
         pytest.skip("bitmap-kernel path")
     monkeypatch.setenv("GS_LW_CTAS", "1")
+    if ccap is not None:
+        monkeypatch.setenv("GS_LW_CCAP", ccap)
     g, G, O = ljlike
     seeds = synth.make_seeds(synth.GraphSpec("lj", 300_000, 1, False, None, 11), 512 * 12)
     for K in (64, 512):
