@@ -1,7 +1,7 @@
 # Round-2 evidence (second session): full GPU tests, smoke, the default bench
 # line (+ reference arm), a sweep of every workload, the launch list and ncu
 # --set full captures of the re-written layer-wise kernels.
-O=gpurun_out/ev4; mkdir -p $O
+O=gpurun_out/ev5; mkdir -p $O
 timeout 2400 python -m pytest tests -m gpu -q -rf > $O/pytest_gpu.log 2>&1; echo "rc=$?" >> $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log
 timeout 600 python bench.py > $O/bench_default.log 2>&1; echo "rc=$?" >> $O/bench_default.log
@@ -12,4 +12,4 @@ done
 timeout 600 ncu --kernel-name-base demangled -k regex:"hop_|bptr_" --metrics gpu__time_duration.sum --clock-control none -c 60 --csv --log-file $O/launches_graphsage_pd.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-graph > $O/b_ncu1.log 2>&1
 
 
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:"hop_select|hop_rows|hop_relabel" --launch-skip 8 --launch-count 6 -o $O/ncu_graphsage_pd python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-graph > $O/b_ncu2.log 2>&1
+timeout 1500 ncu --set full --import-source on --clock-control none -k regex:layerwise_bm --launch-skip 1 --launch-count 1 -o $O/ncu_fastgcn python bench.py --workload fastgcn_lj --steps 1 --warmup 1 --no-cpu-baseline --no-graph > $O/b_ncu3.log 2>&1
