@@ -447,6 +447,9 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
       }
       __syncthreads();
       {
+        // the streamed columns are hinted evict-first: the 148 CTAs' candidate
+        // bitmaps (the atomics' lines) should keep their place in L2
+        const uint64_t pf1 = pol_first(), pl1 = pol_last();
         LBStream st(nflat);
         for (int64_t e0 = st.beg; e0 < st.end; e0 += 32 * LB_ILP) {
           uint32_t u[LB_ILP];
@@ -462,8 +465,8 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
               const int c = st.col(s_fstart, Ti, e);
               const int64_t pos = s_off[c] + (e - s_fstart[c]);
               cc[q] = c;
-              u[q] = (uint32_t)__ldg(P.indices + pos);
-              if (l1_deg) dg[q] = __ldg(P.degsrc + pos);
+              u[q] = (uint32_t)ldg_h(P.indices + pos, pf1);
+              if (l1_deg) dg[q] = ldg_h(P.degsrc + pos, pf1);
             }
           }
 #pragma unroll
@@ -477,7 +480,10 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
               if (!l1_deg) {
                 atomicOr(bm + (u[q] >> 5), bit);
               } else {
-                const bool is_new = !(atomicOr(bm + (u[q] >> 5), bit) & bit);
+                uint32_t old;
+                asm volatile("atom.global.or.L2::cache_hint.b32 %0, [%1], %2, %3;"
+                             : "=r"(old) : "l"(bm + (u[q] >> 5)), "r"(bit), "l"(pl1) : "memory");
+                const bool is_new = !(old & bit);
                 if (is_new) {
                   l1_b += (unsigned long long)dg[q];
                   l1_e += dg[q] > 0 ? 1 : 0;
@@ -715,7 +721,12 @@ __global__ void __launch_bounds__(LB_THREADS, 1) layerwise_bm_kernel(LBParams P)
         s_hv[h] = i;
       }
       // clear C for the next batch-layer (bitmap, b(u))
-      for (int64_t i = threadIdx.x; i < P.n4; i += blockDim.x) ((uint4*)bm)[i] = make_uint4(0, 0, 0, 0);
+      {
+        const uint64_t pl2 = pol_last();  // the cleared lines are the next batch-layer's atomics' lines
+        for (int64_t i = threadIdx.x; i < P.n4; i += blockDim.x)
+          asm volatile("st.global.L2::cache_hint.v4.b32 [%0], {%1, %1, %1, %1}, %2;" ::"l"((uint4*)bm + i), "r"(0u),
+                       "l"(pl2) : "memory");
+      }
       if (!degree && acc_ok)
         for (int64_t r = threadIdx.x; r < nc; r += blockDim.x) acc[r] = 0.0;
       for (int j = threadIdx.x; j < Ti; j += blockDim.x) {
