@@ -84,6 +84,7 @@ struct HopParams {
                              // words 1..3 = bits; lay 0: 128 nodes per group, bits only, ranks in rank4
   int32_t* rank4;            // lay 0: [group slot][nwp / 4] rank of every non-empty group's first row
   int lay;                   // bitmap layout (1: rank inside the group -- one load per relabelled edge)
+  int bm_keep;               // a group's bitmaps fit L2: their row bits are set with an evict-last hint
   uint32_t* summ;            // [group slot][nsw] bit w set iff bitmap word w is non-empty
   int64_t nw, nwp, nsw;      // words used / allocated per batch, summary words
   int sel_nq, sel_claim;     // select: claim queues, chunks per claim
@@ -102,6 +103,15 @@ __device__ __forceinline__ uint32_t hb_word(uint32_t u) {
   return g * 4u + 1u + ((u - g * HB_GNODES) >> 5);
 }
 __device__ __forceinline__ uint32_t hb_bit(uint32_t u) { return 1u << ((u - (u / HB_GNODES) * HB_GNODES) & 31); }
+// A row bit set fire-and-forget; bm_keep (the group's bitmaps fit L2): with an
+// evict-last hint, so the gathers streaming through L2 do not push the bitmap
+// out before row() / relabel / clear read it.
+__device__ __forceinline__ void bm_or(uint32_t* w, uint32_t bit, int keep, uint64_t pk) {
+  if (keep)
+    asm volatile("red.global.or.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(w), "r"(bit), "l"(pk) : "memory");
+  else
+    asm volatile("red.global.or.b32 [%0], %1;" ::"l"(w), "r"(bit) : "memory");
+}
 // the word and bit of node u in either layout
 __device__ __forceinline__ uint32_t hb_wd(int lay, uint32_t u) { return lay ? hb_word(u) : (u >> 5); }
 __device__ __forceinline__ uint32_t hb_bt(int lay, uint32_t u) { return lay ? hb_bit(u) : 1u << (u & 31); }
@@ -347,7 +357,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
   const long long nchunks = sm.cpre[nbg];
   HChunk<KCAP, WEIGHTED>& C = sm.ch[warp];
   const int k = P.k[l];
-  const uint64_t pf = pol_first();
+  const uint64_t pf = pol_first(), pk = pol_last();
   const int use_sum = P.use_sum[l];
   // chunks are claimed from NQ queues (contiguous chunk ranges, counters
   // 128 B apart): a warp drains its home queue, then steals from the next
@@ -643,9 +653,8 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
             }
           }
           const uint32_t wd = hb_wd(P.lay, u[q]);
-          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + wd), "r"(hb_bt(P.lay, u[q])) : "memory");
-          if (use_sum)
-            asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (wd >> 5)), "r"(1u << (wd & 31)) : "memory");
+          bm_or(bits + wd, hb_bt(P.lay, u[q]), P.bm_keep, pk);
+          if (use_sum) bm_or(summ + (wd >> 5), 1u << (wd & 31), P.bm_keep, pk);
         }
       }
     }
@@ -711,7 +720,7 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
   }
   const long long nchunks = cpre[nbg];
   const int k = P.k[l];
-  const uint64_t pf = pol_first();
+  const uint64_t pf = pol_first(), pk = pol_last();
   const float* wts = P.core.weights;
   uint32_t* pos = cpos[warp];
   uint32_t* rnd = crnd[warp];
@@ -932,9 +941,8 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
           sth(P.val[l] + rb + ce + o, w / W, pf);
         }
         const uint32_t wd = hb_wd(P.lay, u);
-        asm volatile("red.global.or.b32 [%0], %1;" ::"l"(bits + wd), "r"(hb_bt(P.lay, u)) : "memory");
-        if (use_sum)
-          asm volatile("red.global.or.b32 [%0], %1;" ::"l"(summ + (wd >> 5)), "r"(1u << (wd & 31)) : "memory");
+        bm_or(bits + wd, hb_bt(P.lay, u), P.bm_keep, pk);
+        if (use_sum) bm_or(summ + (wd >> 5), 1u << (wd & 31), P.bm_keep, pk);
       }
     }
   }
@@ -1265,6 +1273,8 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   WB = std::min<int64_t>(WB, MAX_GROUP);
   WB = std::min<int64_t>(WB, std::max<int64_t>(nbatch, 1));
   const int64_t G = nbatch > 0 ? (nbatch + WB - 1) / WB : 0;
+  P.bm_keep = WB * foot <= budget ? 1 : 0;
+  if (const char* e = getenv("GS_HOP_BMKEEP")) P.bm_keep = atoi(e) ? 1 : 0;
   WB = G > 0 ? (nbatch + G - 1) / G : WB;  // balanced groups
   if (getenv("GS_VERBOSE"))
     fprintf(stderr, "nodewise_hop: %lld groups of %lld batches, footprint %lld KB/batch, sparse hops:%s%s%s\n",
