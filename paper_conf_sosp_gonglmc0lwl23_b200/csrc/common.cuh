@@ -260,6 +260,11 @@ __device__ __forceinline__ int32_t ldg_h(const int32_t* a, uint64_t p) {
   asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(p));
   return v;
 }
+__device__ __forceinline__ int64_t ldg_h64(const int64_t* a, uint64_t p) {
+  int64_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(p));
+  return v;
+}
 __device__ __forceinline__ float ldg_h(const float* a, uint64_t p) {
   float v;
   asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(a), "l"(p));

@@ -84,6 +84,9 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
   __shared__ long long scr64[40];
   __shared__ unsigned long long wstage[PS_WARPS * 32];  // per-warp top-k staging
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // L2 policies: the walks' random reads evict-first, the CTA's row bitmap
+  // (148 x N/8 bytes) evict-last
+  const uint64_t pfw = pol_first(), pkw = pol_last();
   const int HCAP = 1 << P.hlog;
   const int C = P.chunk;
   int32_t* hkey = ps_smem;             // [C][HCAP]
@@ -145,15 +148,15 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
             for (int a = 0; a < PS_ILP; ++a) {
               r[a] = philox((uint32_t)wv[a], (uint32_t)(ww[a] * T + t - 1), ctr2(l, TAG_PINSAGE), gb, P.key);
               if ((float)(r[a].z >> 8) * 0x1p-24f < P.restart) alive[a] = false;  // restart at v (R27)
-              off[a] = alive[a] ? __ldg(P.indptr + wx[a]) : 0;
-              d[a] = alive[a] ? __ldg(P.indptr + wx[a] + 1) : 0;
+              off[a] = alive[a] ? ldg_h64(P.indptr + wx[a], pfw) : 0;
+              d[a] = alive[a] ? ldg_h64(P.indptr + wx[a] + 1, pfw) : 0;
             }
             bool any = false;
 #pragma unroll
             for (int a = 0; a < PS_ILP; ++a) {
               d[a] -= off[a];
               if (d[a] == 0) alive[a] = false;            // dead end (R13)
-              if (alive[a]) wx[a] = __ldg(P.indices + off[a] + (int64_t)draw_below((uint64_t)d[a], r[a].x, r[a].y));
+              if (alive[a]) wx[a] = ldg_h(P.indices + off[a] + (int64_t)draw_below((uint64_t)d[a], r[a].x, r[a].y), pfw);
               any |= alive[a];
             }
             if (!any) break;
@@ -213,7 +216,8 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
               const unsigned long long kv = ~key;
               const int32_t id = 0x7FFFFFFF - (int32_t)(uint32_t)kv;
               scratch[j * k + lane] = ((int64_t)(kv >> 32) << 32) | (uint32_t)id;
-              atomicOr(bm + (id >> 5), 1u << (id & 31));
+              asm volatile("red.global.or.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(bm + (id >> 5)),
+                           "r"(1u << (id & 31)), "l"(pkw) : "memory");
             }
           }
           __syncwarp();
@@ -244,7 +248,8 @@ __global__ void __launch_bounds__(PS_THREADS) pinsage_kernel(PSParams P) {
               const int32_t id = tk[bpos];
               scratch[j * k + taken] = ((int64_t)(uint32_t)tc[bpos] << 32) | (uint32_t)id;
               tc[bpos] = 0;
-              atomicOr(bm + (id >> 5), 1u << (id & 31));
+              asm volatile("red.global.or.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(bm + (id >> 5)),
+                           "r"(1u << (id & 31)), "l"(pkw) : "memory");
             }
             __syncwarp();
           }
