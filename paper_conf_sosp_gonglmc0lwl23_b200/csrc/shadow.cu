@@ -76,6 +76,7 @@ struct SHParams {
   int64_t wcap;
   int64_t bpc;                      // bitmap bits per CTA (multiple of 256)
   uint32_t inv;                     // floor(2^32 / bpc)
+  int load_first;                   // U column loads evict-first (else evict-normal)
 };
 
 struct SHShared {                   // static part; the bitmap + prefix are dynamic
@@ -137,7 +138,9 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
   int32_t* gp = (int32_t*)(smem_raw + (size_t)nwords * 4);
   uint8_t* off8 = (uint8_t*)(gp + ngroups);
   const uint32_t bpc32 = (uint32_t)bpc, inv = P.inv;
-  const uint64_t pf = pol_first();
+  // the output stores stream (evict-first); the U columns' index loads: evict-normal
+  // (hub columns recur in the other batches' U) unless P.load_first
+  const uint64_t pf = pol_first(), pg = P.load_first ? pol_first() : pol_normal();
   while (true) {
     if (rank == 0 && tid == 0) ss.b = (long long)atomicAdd(P.claim, 1u);
     cl.sync();
@@ -260,7 +263,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
 #pragma unroll
         for (int q = 0; q < SH_ILP; ++q) {
           const int64_t i = i0 + q * 32 + lane;
-          u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
+          u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pg) : 0xFFFFFFFFu;
         }
         bool m[SH_ILP];
 #pragma unroll
@@ -366,7 +369,7 @@ __global__ void __launch_bounds__(SH_THREADS, 1) shadow_induce_kernel(SHParams P
 #pragma unroll
           for (int q = 0; q < SH_ILP; ++q) {
             const int64_t i = i0 + q * 32 + lane;
-            u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pf) : 0xFFFFFFFFu;
+            u[q] = i < d ? (uint32_t)ldg_h(P.indices + o + i, pg) : 0xFFFFFFFFu;
           }
 #pragma unroll
           for (int q = 0; q < SH_ILP; ++q) m[q] = u[q] != 0xFFFFFFFFu && sh_member(cl, bm, bpc32, inv, u[q]);
@@ -462,6 +465,7 @@ static gs_status launch_induce(const gs_graph* g, SHParams P, int CS, int64_t bp
   P.claim = (unsigned int*)((char*)blk->b_ctr.ptr + 8 * (MAX_LAYERS + 1));
   P.bpc = bpc;
   P.inv = (uint32_t)((uint64_t(1) << 32) / (uint64_t)bpc);
+  P.load_first = getenv("GS_SH_LOAD_FIRST") ? 1 : 0;
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_err.ptr, 0, 16, stream));
   GS_CUDA_TRY(cudaMemsetAsync(blk->b_ctr.ptr, 0, 8 * (MAX_LAYERS + 2), stream));
   if (nbatch == 0) return GS_OK;
