@@ -1170,7 +1170,7 @@ static int64_t a256h(int64_t x) { return (x + 255) & ~int64_t(255); }
 
 template <bool W, int KCAP>
 static gs_status launch_select(const HopParams& P, int l, int64_t b0, int nbg, unsigned int* claim,
-                               cudaStream_t stream) {
+                               int64_t chunks_ub, cudaStream_t stream) {
   const size_t smem = sizeof(HSmem<W, KCAP>) + (W ? sizeof(HWarpA) * HS_WARPS : 0);
   auto kfn = hop_select_kernel<W, KCAP>;
   static int grid = 0;
@@ -1187,7 +1187,14 @@ static gs_status launch_select(const HopParams& P, int l, int64_t b0, int nbg, u
     if (getenv("GS_VERBOSE"))
       fprintf(stderr, "hop_select<%d,%d>: smem %zu B, %d CTAs/SM\n", (int)W, KCAP, smem, per_sm);
   }
-  kfn<<<grid, HS_THREADS, smem, stream>>>(P, l, b0, nbg, claim); count_launch();
+  // small groups (hop 0, per-rank shards of a strong-scaled epoch): no more
+  // CTAs than the group has chunks for -- the surplus warps otherwise walk
+  // every claim queue with an atomic each and find nothing
+  static int64_t cpw = -1;
+  if (cpw < 0) { cpw = 1; if (const char* e = getenv("GS_SEL_CPW")) cpw = std::max(0, atoi(e)); }
+  int g = grid;
+  if (cpw > 0) g = (int)std::max<int64_t>(1, std::min<int64_t>(grid, (chunks_ub + cpw * HS_WARPS - 1) / (cpw * HS_WARPS)));
+  kfn<<<g, HS_THREADS, smem, stream>>>(P, l, b0, nbg, claim); count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
 }
@@ -1426,14 +1433,15 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
         mark("nprep", l);
       }
       const int k = P.k[l];
+      const int64_t cub = (int64_t)nbg * ((maxbs * (l == 0 ? 1 : P.K[l - 1]) + 31) / 32);
       gs_status rc;
       if (weighted) {
-        rc = k <= 16 ? launch_select<true, 16>(P, l, b0, nbg, cq, stream)
-                     : launch_select<true, 32>(P, l, b0, nbg, cq, stream);
+        rc = k <= 16 ? launch_select<true, 16>(P, l, b0, nbg, cq, cub, stream)
+                     : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream);
       } else {
-        rc = k <= 8 ? launch_select<false, 8>(P, l, b0, nbg, cq, stream)
-                    : (k <= 16 ? launch_select<false, 16>(P, l, b0, nbg, cq, stream)
-                               : launch_select<false, 32>(P, l, b0, nbg, cq, stream));
+        rc = k <= 8 ? launch_select<false, 8>(P, l, b0, nbg, cq, cub, stream)
+                    : (k <= 16 ? launch_select<false, 16>(P, l, b0, nbg, cq, cub, stream)
+                               : launch_select<false, 32>(P, l, b0, nbg, cq, cub, stream));
       }
       if (rc) return rc;
       mark("select", l);
