@@ -643,16 +643,23 @@ def run_gpu(args, wl, world, rank, device):
     if chunked:
         nbat = (inputs.numel() + bs - 1) // bs
         nch = max(1, min(E2E_CHUNKS, nbat))
-        cb = [nbat * c // nch for c in range(nch + 1)]
+        # a small first chunk: the link starts as early as possible, the
+        # later chunks sample while it drains
+        first = nbat // E2E_FIRST if E2E_FIRST > 0 and nch > 1 else 0
+        if first >= 1:
+            cb = [0] + [first + (nbat - first) * c // (nch - 1) for c in range(nch)]
+        else:
+            cb = [nbat * c // nch for c in range(nch + 1)]
         souts = [gs.Blocks() for _ in range(nch)]
-        cstreams = (torch.cuda.Stream(), torch.cuda.Stream())
+        cstreams = tuple(torch.cuda.Stream() for _ in range(E2E_STREAMS))
+        mstream = torch.cuda.Stream()
 
-        def step_chunk(i, c, x):
+        def step_chunk(i, c, x, st=stream):
             key = base_key + 7919 * i
             lo, hi = cb[c] * bs, min(cb[c + 1] * bs, x.numel())
             gs.sample_neighbors(G, x[lo:hi], wl["fanouts"], batch_size=bs, batch_index_base=wbase + cb[c],
                                 replace=wl["replace"], bias_mode=wl["bias"], rng_key=key,
-                                stream=stream, out=souts[c])
+                                stream=st, out=souts[c])
 
         for c in range(nch):  # sizes the chunk results before the pack buffers
             step_chunk(args.warmup, c, inputs)
@@ -663,39 +670,85 @@ def run_gpu(args, wl, world, rank, device):
         chost_tot = [torch.empty((L, 3), dtype=torch.int64).pin_memory() for _ in range(nch)]
         chost_pk = [[{k2: torch.empty(v.shape, dtype=v.dtype).pin_memory() for k2, v in pk.items()
                       if k2 != "totals"} for pk in cp] for cp in cpacks]
-    for i in range(max(2, min(args.steps, 5)) + (1 if chunked else 0)):
+    n_e2e = max(2, min(args.steps, 5)) + (1 if chunked else 0)
+    cgraphs = None
+    if chunked and args.graph and E2E_GRAPH:
+        # each chunk's public calls (sample + pack) captured once per step key,
+        # as the device-timed epoch is: one launch per chunk instead of the
+        # per-call host work between the link's chunks
+        try:
+            gcs = torch.cuda.Stream()
+            cgraphs = []
+            for i in range(n_e2e):
+                row = []
+                for c in range(nch):
+                    gr = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(gr, stream=gcs):
+                        step_chunk(args.warmup + i, c, dev_in, st=gcs)
+                        for l in range(L):
+                            souts[c].pack(l, cpacks[c][l], stream=gcs, narrow=narrow)
+                    row.append(gr)
+                cgraphs.append(row)
+            torch.cuda.synchronize()
+        except Exception as e:
+            print(f"# e2e chunk capture failed ({e}); eager chunks", file=sys.stderr)
+            cgraphs = None
+            torch.cuda.synchronize()
+    for i in range(n_e2e):
         if chunked:
             flush.zero_()
             torch.cuda.synchronize()
             ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             ev0.record(stream)
             dev_in.copy_(host_in, non_blocking=True)
-            ready = []
+            ready, packs_ev = [], []
             for c in range(nch):
-                step_chunk(args.warmup + i, c, dev_in)
-                for l in range(L):
-                    souts[c].pack(l, cpacks[c][l], stream=stream, narrow=narrow)
-                    chost_tot[c][l].copy_(cpacks[c][l]["totals"], non_blocking=True)
-                chost_meta[c].copy_(cmeta[c], non_blocking=True)
-                e = torch.cuda.Event()
-                e.record(stream)
+                if cgraphs is not None:
+                    cgraphs[i][c].replay()
+                else:
+                    step_chunk(args.warmup + i, c, dev_in)
+                    for l in range(L):
+                        souts[c].pack(l, cpacks[c][l], stream=stream, narrow=narrow)
+                # the chunk's sizes and batch offsets come back on a stream of
+                # their own: a D2H copy on the sampling stream would queue
+                # behind the previous chunks' bulk copies in the copy engine
+                # and hold the next chunk's sampling back until they drain
+                packed = torch.cuda.Event(enable_timing=E2E_DEBUG)
+                packed.record(stream)
+                packs_ev.append(packed)
+                mstream.wait_event(packed)
+                with torch.cuda.stream(mstream):
+                    for l in range(L):
+                        chost_tot[c][l].copy_(cpacks[c][l]["totals"], non_blocking=True)
+                    chost_meta[c].copy_(cmeta[c], non_blocking=True)
+                e = torch.cuda.Event(enable_timing=E2E_DEBUG)
+                e.record(mstream)
                 ready.append(e)
             d2h = 0
+            queued = [0] * len(cstreams)  # bytes queued per copy stream (greedy balance)
             for c in range(nch):
                 ready[c].synchronize()  # this chunk's sizes (the later chunks keep sampling)
                 d2h += chost_tot[c].numel() * 8 + chost_meta[c].numel() * 8
                 for cs_ in cstreams:
                     cs_.wait_event(ready[c])
+                tot = chost_tot[c].tolist()
                 for l in range(L):
-                    ne, ni, nr = (int(x) for x in chost_tot[c][l])
+                    ne, ni, nr = tot[l]
                     for k2, n in (("row_local", ne), ("eid", ne), ("indptr", ni), ("row_map", nr)):
-                        with torch.cuda.stream(cstreams[1] if k2 == "eid" else cstreams[0]):
+                        nb = n * cpacks[c][l][k2].element_size()
+                        si = min(range(len(cstreams)), key=lambda j: queued[j])
+                        queued[si] += nb
+                        with torch.cuda.stream(cstreams[si]):
                             chost_pk[c][l][k2][:n].copy_(cpacks[c][l][k2][:n], non_blocking=True)
-                        d2h += n * cpacks[c][l][k2].element_size()
-            for cs_ in cstreams:
+                        d2h += nb
+            for cs_ in cstreams + (mstream,):
                 stream.wait_stream(cs_)
             ev1.record(stream)
             ev1.synchronize()
+            if E2E_DEBUG:
+                print(f"e2e step {i}: chunks packed at " + ", ".join(f"{ev0.elapsed_time(r):.3f}" for r in packs_ev)
+                      + "; ready at " + ", ".join(f"{ev0.elapsed_time(r):.3f}" for r in ready)
+                      + f" ms, end {ev0.elapsed_time(ev1):.3f} ms, {d2h / 1e6:.1f} MB", file=sys.stderr)
             if i > 0:  # the first pass warms the chunked path
                 e2e_times.append(ev0.elapsed_time(ev1))
                 d2h_all.append(d2h)
@@ -797,7 +850,11 @@ def run_gpu(args, wl, world, rank, device):
             "launches_per_step": launches_per_step}
 
 
-E2E_CHUNKS = 4  # node-wise e2e: the epoch sampled and copied back in this many pipelined chunks
+E2E_CHUNKS = int(os.environ.get("GS_E2E_CHUNKS", 4))  # node-wise e2e: the epoch sampled and copied back in this many pipelined chunks
+E2E_FIRST = int(os.environ.get("GS_E2E_FIRST", 16))  # the first chunk holds 1/E2E_FIRST of the batches (0: even chunks)
+E2E_GRAPH = int(os.environ.get("GS_E2E_GRAPH", 1))  # chunk calls replayed from CUDA graphs
+E2E_DEBUG = bool(os.environ.get("GS_E2E_DEBUG"))
+E2E_STREAMS = int(os.environ.get("GS_E2E_STREAMS", 2))  # copy streams, bytes balanced greedily
 
 KERNEL_OF = {"nodewise": "node-wise engine (nodewise_hop.cu: nprep / select / rows / relabel / clear per hop)",
              "shadow": "gsb::shadow_induce_kernel",
@@ -897,7 +954,10 @@ def main():
                             "(int32 ids when the graph has < 2^31 entries) so exactly the sampled data "
                             "crosses the host link, which bounds this number"
                             + (f"; node-wise: the epoch in {E2E_CHUNKS} pipelined chunks (public calls with "
-                               "batch_index_base = the chunk's first batch), each chunk's copies on two copy "
+                               "batch_index_base = the chunk's first batch; the first chunk "
+                               f"1/{E2E_FIRST} of the batches; each chunk's sample + pack calls replayed "
+                               "from a CUDA graph per step key when graphs are on), each chunk's sizes "
+                               f"read back on a stream of their own and its arrays on {E2E_STREAMS} copy "
                                "streams while the next chunks sample" if kind == "nodewise" else "")},
             "gpu_launches": args.steps * r["launches_per_step"],
             "clocks": r["clocks"],

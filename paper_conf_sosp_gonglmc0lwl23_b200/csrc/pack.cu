@@ -3,7 +3,8 @@
 // blocks (the sampling kernels write each batch into a fixed, padded region,
 // DESIGN.md section 5).  Two kernels on the caller's stream, no host sync:
 // an exclusive scan of the per-batch counts over batches (one CTA), then a
-// grid-stride copy, one mini-batch per CTA at a time.
+// grid-stride copy: CTA (x, y) copies slice y of every gridDim.x-th
+// mini-batch (a few batches still spread over the whole GPU).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -64,6 +65,7 @@ struct PackParams {
 
 template <bool NARROW>
 __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
+  const int64_t t0 = (int64_t)blockIdx.y * PK_THREADS + threadIdx.x, ts = (int64_t)gridDim.y * PK_THREADS;
   for (int64_t b = blockIdx.x; b < P.nb; b += gridDim.x) {
     const int64_t* m = P.meta + (b * P.L + P.layer) * GS_META_FIELDS;
     // clamped to the layer buffers: a block recorded past them is never read
@@ -72,18 +74,18 @@ __global__ void __launch_bounds__(PK_THREADS) pack_copy_kernel(PackParams P) {
     const int64_t R = min(m[1], max(P.row_cap - m[4], (int64_t)0));
     const int64_t* o = P.off + b * 3;
     const int64_t eo = o[0], io = o[1], ro = o[2];
-    for (int64_t i = threadIdx.x; i < E; i += PK_THREADS) {
+    for (int64_t i = t0; i < E; i += ts) {
       P.row_local[eo + i] = __ldcs(P.row_local_in + m[6] + i);
       const int64_t e = __ldcs(P.eid_in + m[6] + i);
       if (NARROW) ((int32_t*)P.eid)[eo + i] = (int32_t)e;
       else ((int64_t*)P.eid)[eo + i] = e;
     }
-    for (int64_t i = threadIdx.x; i <= T; i += PK_THREADS) {
+    for (int64_t i = t0; i <= T; i += ts) {
       const int64_t x = __ldcs(P.indptr_in + m[5] + i);
       if (NARROW) ((int32_t*)P.indptr)[io + i] = (int32_t)x;  // block-relative (<= 2^25)
       else ((int64_t*)P.indptr)[io + i] = x;
     }
-    for (int64_t i = threadIdx.x; i < R; i += PK_THREADS) P.row_map[ro + i] = __ldcs(P.row_map_in + m[4] + i);
+    for (int64_t i = t0; i < R; i += ts) P.row_map[ro + i] = __ldcs(P.row_map_in + m[4] + i);
   }
 }
 
@@ -127,9 +129,11 @@ static gs_status pack_impl(const gs_blocks* b, int layer, int32_t* row_local, vo
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const int64_t grid = std::min<int64_t>(nb, (int64_t)sms * 4);
-  if (narrow) pack_copy_kernel<true><<<(unsigned)grid, PK_THREADS, 0, stream>>>(P);
-  else pack_copy_kernel<false><<<(unsigned)grid, PK_THREADS, 0, stream>>>(P);
+  const int64_t gx = std::min<int64_t>(nb, (int64_t)sms * 4);
+  const int64_t gy = std::max<int64_t>(1, std::min<int64_t>(64, ((int64_t)sms * 8 + gx - 1) / gx));
+  const dim3 grid((unsigned)gx, (unsigned)gy);
+  if (narrow) pack_copy_kernel<true><<<grid, PK_THREADS, 0, stream>>>(P);
+  else pack_copy_kernel<false><<<grid, PK_THREADS, 0, stream>>>(P);
   count_launch();
   GS_CUDA_TRY(cudaGetLastError());
   return GS_OK;
