@@ -48,7 +48,31 @@ constexpr int SPARSE_TILE = HB_THREADS * WPT * 32; // bitmap words per summary-m
 constexpr int CLEAR_TILE = 8192;            // words per dense clear CTA
 constexpr int NP_CPT = 8;                   // nprep: columns per thread
 constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
-constexpr int RL_ILP = 8;                   // relabel: edges per thread in flight
+#ifndef RL_ILP
+#define RL_ILP 4                            // relabel: edges per thread in flight (4 at 8 CTAs/SM: relabel1 0.130 vs 0.137 ms at 8 x 4 CTAs)
+#endif
+#ifndef RL_MINB
+#define RL_MINB 8
+#endif
+// row() at 8 CTAs/SM (32 registers, 32 B of spills): rows0 / rows1 0.085 /
+// 0.104 vs 0.099 / 0.119 ms at 40 registers (6 CTAs/SM); nprep at 4 CTAs/SM
+// (64 registers): nprep1 0.083 vs 0.087 ms
+#ifndef ROWS_MINB
+#define ROWS_MINB 8
+#endif
+#ifndef NP_MINB
+#define NP_MINB 4
+#endif
+#if ROWS_MINB > 0
+#define ROWS_LB __launch_bounds__(HB_THREADS, ROWS_MINB)
+#else
+#define ROWS_LB __launch_bounds__(HB_THREADS)
+#endif
+#if NP_MINB > 0
+#define NP_LB __launch_bounds__(HB_THREADS, NP_MINB)
+#else
+#define NP_LB __launch_bounds__(HB_THREADS)
+#endif
 constexpr int RL_TILE = HB_THREADS * RL_ILP;
 constexpr int MAX_GROUP = 512;              // batches per group (claim directories in smem)
 #ifndef SEL_MINB
@@ -216,7 +240,7 @@ __device__ __forceinline__ int dir_find(const long long* dir, int nbg, long long
 // nprep: hop l's column side, one 2048-column segment per CTA (tickets over
 // the group's (batch, segment) pairs in batch order).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(HB_THREADS) hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, Scan S) {
+__global__ void NP_LB hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, Scan S) {
   __shared__ long long dir[MAX_GROUP + 1];
   __shared__ long long scr[40];
   __shared__ long long sh[2];
@@ -959,7 +983,7 @@ __global__ void __launch_bounds__(AB_THREADS, AB_MINB) hop_ares_big_kernel(HopPa
 // (Measured and not kept: the next hop's column side fused in here -- its
 // degree loads delay every tile's look-back: 0.24 vs 0.09 + 0.085 ms.)
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l, int64_t b0, int nbg, int ntile,
+__global__ void ROWS_LB hop_rows_kernel(HopParams P, int l, int64_t b0, int nbg, int ntile,
                                                               Scan S) {
   __shared__ long long scr[40];
   __shared__ long long sh[2];
@@ -1069,7 +1093,7 @@ __global__ void __launch_bounds__(HB_THREADS) hop_rows_kernel(HopParams P, int l
 // ---------------------------------------------------------------------------
 // relabel: row id -> rank in place (grid: edge tiles x batches of the group).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(HB_THREADS) hop_relabel_kernel(HopParams P, int l, int64_t b0) {
+__global__ void __launch_bounds__(HB_THREADS, RL_MINB) hop_relabel_kernel(HopParams P, int l, int64_t b0) {
   const int64_t j = blockIdx.y;
   const int64_t b = b0 + j;
   const long long E = __ldcg((const long long*)P.meta + (b * P.L + l) * 8 + 2);
