@@ -265,6 +265,20 @@ __device__ __forceinline__ int32_t ldg_h(const int32_t* a, uint64_t p) {
   asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(p));
   return v;
 }
+// predicated form (v unchanged when !on): no branch around the load, so a
+// run of them stays in flight together -- a load inside an if() becomes a
+// branch + reconvergence, and the compiler then waits on the loads' shared
+// scoreboard before the next one is issued
+__device__ __forceinline__ uint32_t ldg_h_if(bool on, const int32_t* a, uint64_t p, uint32_t v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.L2::cache_hint.b32 %0, [%1], %3; }"
+               : "+r"(v) : "l"(a), "r"((int)on), "l"(p));
+  return v;
+}
+__device__ __forceinline__ float ldg_h_if(bool on, const float* a, uint64_t p, float v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.L2::cache_hint.f32 %0, [%1], %3; }"
+               : "+f"(v) : "l"(a), "r"((int)on), "l"(p));
+  return v;
+}
 __device__ __forceinline__ int64_t ldg_h64(const int64_t* a, uint64_t p) {
   int64_t v;
   asm volatile("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(p));

@@ -113,7 +113,6 @@ struct HopParams {
   uint32_t* summ;            // [group slot][nsw] bit w set iff bitmap word w is non-empty
   int64_t nw, nwp, nsw;      // words used / allocated per batch, summary words
   int sel_nq, sel_claim;     // select: claim queues, chunks per claim
-  int sel_ld;                // select: gather load flavour (0 nc, 1 cg, 2 nc no-L1-allocate)
   int ares_split;            // A-Res columns with d > 64: 1 hop_ares_big_kernel, 0 in select
   int ares_tau;              // hop_ares_big_kernel's first threshold: 0 normal, 1 too tight,
                              // 2 too loose (tests: every widen / narrow step runs)
@@ -653,14 +652,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
       for (int q = 0; q < 16 && h + q < KCAP; ++q) {
         const int i = h + q;
         const uint32_t ps = all ? (uint32_t)i : a[i];
-        u[q] = 0u;
-        if (i < cnt && !defer) {
-          const int32_t* ap = P.core.indices + off + ps;
-          if (P.sel_ld == 1) u[q] = (uint32_t)ldh(ap, pf);  // L2 only
-          else if (P.sel_ld == 2)
-            asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(u[q]) : "l"(ap), "l"(pf));
-          else u[q] = (uint32_t)ldg_h(ap, pf);
-        }
+        u[q] = ldg_h_if(i < cnt && !defer, P.core.indices + off + ps, pf, 0u);
       }
 #pragma unroll
       for (int q = 0; q < 16 && h + q < KCAP; ++q) {
@@ -1270,8 +1262,6 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   P.nsw = P.nwp / 32;
   P.sel_nq = 32;
   P.sel_claim = 2;
-  P.sel_ld = 0;
-  if (const char* e = getenv("GS_SEL_LD")) P.sel_ld = atoi(e);
   P.ares_split = 1;
   if (const char* e = getenv("GS_ARES_SPLIT")) P.ares_split = atoi(e);
   P.ares_tau = 0;
