@@ -279,6 +279,26 @@ __device__ __forceinline__ float ldg_h_if(bool on, const float* a, uint64_t p, f
                : "+f"(v) : "l"(a), "r"((int)on), "l"(p));
   return v;
 }
+__device__ __forceinline__ int32_t ldcg_if(bool on, const int32_t* a, int32_t v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.cg.b32 %0, [%1]; }"
+               : "+r"(v) : "l"(a), "r"((int)on));
+  return v;
+}
+__device__ __forceinline__ int64_t ldg_if(bool on, const int64_t* a, int64_t v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.b64 %0, [%1]; }"
+               : "+l"(v) : "l"(a), "r"((int)on));
+  return v;
+}
+__device__ __forceinline__ float ldg_if(bool on, const float* a, float v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.f32 %0, [%1]; }"
+               : "+f"(v) : "l"(a), "r"((int)on));
+  return v;
+}
+__device__ __forceinline__ int32_t ldg_if(bool on, const int32_t* a, int32_t v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.b32 %0, [%1]; }"
+               : "+r"(v) : "l"(a), "r"((int)on));
+  return v;
+}
 __device__ __forceinline__ int64_t ldg_h64(const int64_t* a, uint64_t p) {
   int64_t v;
   asm volatile("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(p));

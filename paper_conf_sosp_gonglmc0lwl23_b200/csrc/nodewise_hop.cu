@@ -262,19 +262,30 @@ __global__ void NP_LB hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, 
   long long sum = 0;
   int32_t v[NP_CPT];
 #pragma unroll
-  for (int q = 0; q < NP_CPT; ++q) v[q] = j0 + q < T ? __ldcg(F + j0 + q) : -1;
+  for (int q = 0; q < NP_CPT; ++q) v[q] = ldcg_if(j0 + q < T, F + j0 + q, -1);
+  // predicated loads (no branch between them: all 16 in flight at once), the
+  // range check's error flag after them
   int64_t off[NP_CPT], d[NP_CPT];
+  bool bad = false;
 #pragma unroll
   for (int q = 0; q < NP_CPT; ++q) {
     const bool act = j0 + q < T;
     const bool valid = act && v[q] >= 0 && (int64_t)v[q] < P.core.N;
-    if (act && !valid) atomicOr(P.core.err, ERR_SEED_RANGE);
-    off[q] = valid ? __ldg(P.core.indptr + v[q]) : 0;
-    d[q] = valid ? __ldg(P.core.indptr + v[q] + 1) - off[q] : 0;
+    bad |= act && !valid;
+    off[q] = ldg_if(valid, P.core.indptr + v[q], (int64_t)0);
+    d[q] = ldg_if(valid, P.core.indptr + v[q] + 1, (int64_t)0);
   }
 #pragma unroll
+  for (int q = 0; q < NP_CPT; ++q) d[q] -= off[q];
+  if (bad) atomicOr(P.core.err, ERR_SEED_RANGE);
+  // weighted (A-Res): the a0 positive-weight counts, all in flight together
+  int pc[NP_CPT];
+  const bool use_pc = !P.core.replace && P.poscnt != nullptr;
+#pragma unroll
+  for (int q = 0; q < NP_CPT; ++q) pc[q] = ldg_if(use_pc && d[q] > 0, P.poscnt + v[q], 0);
+#pragma unroll
   for (int q = 0; q < NP_CPT; ++q) {
-    cnt[q] = hp_count(P, l, v[q], d[q]);
+    cnt[q] = use_pc ? (d[q] > 0 ? min(P.k[l], pc[q]) : 0) : hp_count(P, l, v[q], d[q]);  // = hp_count
     sum += cnt[q];
   }
   const long long agg = block_reduce_sum<long long>(sum, scr);
