@@ -209,6 +209,33 @@ __device__ long long lookback(unsigned long long* st, int s, long long agg) {
   return ex;
 }
 
+// Block-wide exclusive scan chained across a segment chain by the look-back
+// above, in two barriers (a reduce, the look-back and a scan back to back
+// took seven): returns this thread's exclusive prefix over the whole chain,
+// *base the CTA's own prefix and *total its aggregate.  scr >= 34 entries.
+__device__ __forceinline__ long long block_scan_chain(long long v, long long* scr, unsigned long long* status,
+                                                      int seg, long long* base, long long* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const long long inc = warp_inclusive_scan(v);
+  if (lane == 31) scr[wid] = inc;
+  __syncthreads();
+  if (wid == 0) {
+    const long long s = lane < nw ? scr[lane] : 0ll;
+    const long long si = warp_inclusive_scan(s);
+    const long long agg = __shfl_sync(0xffffffffu, si, nw - 1);
+    const long long b = lookback(status, seg, agg);
+    if (lane < nw) scr[lane] = b + si - s;
+    if (lane == 0) {
+      scr[32] = b;
+      scr[33] = agg;
+    }
+  }
+  __syncthreads();
+  *base = scr[32];
+  *total = scr[33];
+  return inc - v + scr[wid];
+}
+
 // Directory of a group: dir[i] = segments of the group's batches before i;
 // ticket -> (batch slot, segment).  All threads; ends synchronised.
 template <class NSEG>
@@ -288,13 +315,8 @@ __global__ void NP_LB hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, 
     cnt[q] = use_pc ? (d[q] > 0 ? min(P.k[l], pc[q]) : 0) : hp_count(P, l, v[q], d[q]);  // = hp_count
     sum += cnt[q];
   }
-  const long long agg = block_reduce_sum<long long>(sum, scr);
-  if (threadIdx.x < 32) {
-    const long long ex0 = lookback(S.status + (c - seg), seg, agg);
-    if (threadIdx.x == 0) sh[1] = ex0;
-  }
-  long long tot;
-  long long ex = block_exclusive_scan<long long>(sum, scr, &tot) + sh[1];  // syncs: sh[1] visible
+  long long sbase, tot;
+  long long ex = block_scan_chain(sum, scr, S.status + (c - seg), seg, &sbase, &tot);
 #pragma unroll
   for (int q = 0; q < NP_CPT; ++q) {
     const long long jj = j0 + q;

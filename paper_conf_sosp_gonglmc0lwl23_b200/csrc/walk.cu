@@ -92,7 +92,10 @@ __device__ __forceinline__ int32_t walk_pick(const WalkParams& P, int64_t pos, i
   return __ldg(P.indices + pos);
 }
 
-__global__ void __launch_bounds__(256) walk_kernel(WalkParams P) {
+#ifndef WALK_MINB
+#define WALK_MINB 4
+#endif
+__global__ void __launch_bounds__(256, WALK_MINB) walk_kernel(WalkParams P) {
   const int64_t L1 = (int64_t)P.length + 1;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P.num_walkers;
        i += (int64_t)gridDim.x * blockDim.x) {
