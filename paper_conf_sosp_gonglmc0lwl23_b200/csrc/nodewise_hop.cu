@@ -78,6 +78,9 @@ constexpr int MAX_GROUP = 512;              // batches per group (claim director
 #ifndef SEL_MINB
 #define SEL_MINB 3
 #endif
+#ifndef SEL_MINB32
+#define SEL_MINB32 2
+#endif
 constexpr int HW_CAP = 128;                 // A-Res candidates per warp
 constexpr int ROW_STAGE = 4096;             // rows of a tile staged in smem for coalesced writes
 
@@ -391,7 +394,7 @@ struct HSmem {
 // the lane's sampled rows gathered 16 at a time, bitmap bits set, edge id / row
 // id staged slot-major in shared memory, then written out coalesced.
 template <bool WEIGHTED, int KCAP>
-__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_MINB : 2))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
+__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_MINB : SEL_MINB32))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
                                                                  unsigned int* claim) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = HSmem<WEIGHTED, KCAP>;
