@@ -1308,8 +1308,14 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
   int64_t foot = 0;  // L2 footprint of one batch slot (bytes)
   for (int l = 0; l < L; ++l) {
     const int64_t slots = maxbs * P.K[l];
-    P.use_sum[l] = slots * 4 < P.nw ? 1 : 0;
+    // summary (sparse) row() only when rows are far fewer than bitmap words:
+    // in the 96-node-group layout the rows of a batch touch a large share of
+    // the groups, and the dense scan of an L2-resident bitmap is cheaper
+    // (PD hop 0 with k = 10: 0.086 vs 0.229 ms; PP's 111 M-node layout-0
+    // bitmaps keep the summary at 4 slots per word: dense 16.2 vs 1.1 ms)
+    P.use_sum[l] = slots * (P.lay ? 32 : 4) < P.nw ? 1 : 0;
     if (getenv("GS_HOP_DENSE")) P.use_sum[l] = 0;
+    if (getenv("GS_HOP_SPARSE")) P.use_sum[l] = 1;  // tests: the summary path at any density
     const int64_t tile = P.use_sum[l] ? SPARSE_TILE : ROWS_TILE;
     ntile[l] = (int)((P.nw + tile - 1) / tile);
     foot = std::max(foot, P.use_sum[l] ? std::min(P.nw * 5, slots * 48) + P.nsw * 4 : P.nw * (P.lay ? 4 : 5));

@@ -185,14 +185,18 @@ def test_pack_matches_views(gs, medium, kind, narrow):
         assert tot == [e, i, r]
 
 
+@pytest.mark.parametrize("rowmode", ["auto", "GS_HOP_SPARSE", "GS_HOP_DENSE"])
 @pytest.mark.parametrize("layout", ["0", "1"])
 @pytest.mark.parametrize("fan", [[25, 10], [15, 10, 5]])
-def test_row_bitmap_layouts(gs, oracle_lib, medium, fan, layout, monkeypatch):
+def test_row_bitmap_layouts(gs, oracle_lib, medium, fan, layout, rowmode, monkeypatch):
     """Both row-bitmap layouts of the node-wise engine (GS_HOP_LAYOUT: 1 = the
     rank inside each 96-node group, the default below 2^24 nodes; 0 = bits
-    only with a rank per 128 nodes beside them, the default above), uniform and
-    weighted, against the oracle."""
+    only with a rank per 128 nodes beside them, the default above), each with
+    row() chosen by density or forced to the summary (sparse) or dense scan,
+    uniform and weighted, against the oracle."""
     monkeypatch.setenv("GS_HOP_LAYOUT", layout)
+    if rowmode != "auto":
+        monkeypatch.setenv(rowmode, "1")
     g, G, O = medium
     seeds = synth.make_seeds(synth.GraphSpec("m", g["indptr"].numel() - 1, 1, True, None, 31), 3000)
     for bias in (0, 1):
