@@ -60,6 +60,9 @@ constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
 #ifndef ROWS_MINB
 #define ROWS_MINB 8
 #endif
+#ifndef SP_B
+#define SP_B 4                              // summary-mode row(): non-empty words loaded together
+#endif
 #ifndef NP_MINB
 #define NP_MINB 4
 #endif
@@ -1054,12 +1057,20 @@ __global__ void ROWS_LB hop_rows_kernel(HopParams P, int l, int64_t b0, int nbg,
       const uint4 x = __ldcg((const uint4*)(summ + w0) + q);
       sw[4 * q] = x.x; sw[4 * q + 1] = x.y; sw[4 * q + 2] = x.z; sw[4 * q + 3] = x.w;
     }
+    // the non-empty words, RL_B at a time: their loads are issued together
+    // (one at a time, each popcount waited for its own load)
     for (int q = 0; q < WPT; ++q) {
       uint32_t x = sw[q];
       while (x) {
-        const int bit = __ffs(x) - 1;
-        x &= x - 1u;
-        r += __popc(__ldcg(bm + ((w0 + q) << 5) + bit));
+        uint32_t v[SP_B];
+#pragma unroll
+        for (int j = 0; j < SP_B; ++j) {
+          const int bit = x ? __ffs(x) - 1 : 0;
+          v[j] = (uint32_t)ldcg_if(x != 0u, (const int32_t*)bm + ((w0 + q) << 5) + bit, 0);
+          x &= x - 1u;
+        }
+#pragma unroll
+        for (int j = 0; j < SP_B; ++j) r += __popc(v[j]);
       }
     }
   }
@@ -1101,10 +1112,18 @@ __global__ void ROWS_LB hop_rows_kernel(HopParams P, int l, int64_t b0, int nbg,
     for (int q = 0; q < WPT; ++q) {
       uint32_t x = sw[q];
       while (x) {
-        const int bit = __ffs(x) - 1;
-        x &= x - 1u;
-        const int64_t wi = ((w0 + q) << 5) + bit;
-        emit_word(wi, __ldcg(bm + wi));
+        uint32_t v[SP_B];
+        int64_t wi[SP_B];
+#pragma unroll
+        for (int j = 0; j < SP_B; ++j) {
+          const int bit = x ? __ffs(x) - 1 : 0;
+          wi[j] = x ? ((w0 + q) << 5) + bit : -1;
+          v[j] = (uint32_t)ldcg_if(x != 0u, (const int32_t*)bm + ((w0 + q) << 5) + bit, 0);
+          x &= x - 1u;
+        }
+#pragma unroll
+        for (int j = 0; j < SP_B; ++j)
+          if (wi[j] >= 0) emit_word(wi[j], v[j]);
       }
     }
   }
