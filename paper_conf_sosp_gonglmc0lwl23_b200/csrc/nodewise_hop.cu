@@ -421,6 +421,10 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
   HChunk<KCAP, WEIGHTED>& C = sm.ch[warp];
   const int k = P.k[l];
   const uint64_t pf = P.gather_normal ? pol_normal() : pol_first(), pk = pol_last();
+#ifndef SEL_EID_FIRST
+#define SEL_EID_FIRST 1
+#endif
+  const uint64_t pe = SEL_EID_FIRST ? pol_first() : pf;
   const int use_sum = P.use_sum[l];
   // chunks are claimed from NQ queues (contiguous chunk ranges, counters
   // 128 B apart): a warp drains its home queue, then steals from the next
@@ -720,7 +724,7 @@ __global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_
     float* val_out = P.val[l] ? P.val[l] + rb + ebase : nullptr;
     for (int f = lane; f < total; f += 32) {
       if (WEIGHTED && C.se[f] == ~0ull) continue;
-      sth(eid_out + f, (int64_t)C.se[f], pf);
+      sth(eid_out + f, (int64_t)C.se[f], pe);  // edge ids: never read again on the device
       sth(rl_out + f, (int32_t)C.su[f], pf);
       if constexpr (WEIGHTED) {
         if (val_out) sth(val_out + f, C.sv[f], pf);
