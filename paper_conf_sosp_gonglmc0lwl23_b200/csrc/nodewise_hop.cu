@@ -43,8 +43,11 @@ constexpr int HB_THREADS = 256;             // nprep / rows / relabel / clear
 constexpr int HS_THREADS = 256;             // select
 constexpr int HS_WARPS = HS_THREADS / 32;
 constexpr int WPT = 8;                      // bitmap (dense) or summary (sparse) words per thread
-constexpr int ROWS_TILE = HB_THREADS * WPT;        // bitmap words per dense rows tile
-constexpr int SPARSE_TILE = HB_THREADS * WPT * 32; // bitmap words per summary-mode tile
+#ifndef RW_THREADS
+#define RW_THREADS 512                      // row(): threads per tile (512: hop-0 row() 0.078 vs 0.083 ms at 256)
+#endif
+constexpr int ROWS_TILE = RW_THREADS * WPT;        // bitmap words per dense rows tile
+constexpr int SPARSE_TILE = RW_THREADS * WPT * 32; // bitmap words per summary-mode tile
 constexpr int CLEAR_TILE = 8192;            // words per dense clear CTA
 constexpr int NP_CPT = 8;                   // nprep: columns per thread
 constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
@@ -58,7 +61,7 @@ constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
 // 0.104 vs 0.099 / 0.119 ms at 40 registers (6 CTAs/SM); nprep at 4 CTAs/SM
 // (64 registers): nprep1 0.083 vs 0.087 ms
 #ifndef ROWS_MINB
-#define ROWS_MINB 8
+#define ROWS_MINB (2048 / RW_THREADS)
 #endif
 #ifndef SP_B
 #define SP_B 4                              // summary-mode row(): non-empty words loaded together
@@ -67,9 +70,9 @@ constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
 #define NP_MINB 4
 #endif
 #if ROWS_MINB > 0
-#define ROWS_LB __launch_bounds__(HB_THREADS, ROWS_MINB)
+#define ROWS_LB __launch_bounds__(RW_THREADS, ROWS_MINB)
 #else
-#define ROWS_LB __launch_bounds__(HB_THREADS)
+#define ROWS_LB __launch_bounds__(RW_THREADS)
 #endif
 #if NP_MINB > 0
 #define NP_LB __launch_bounds__(HB_THREADS, NP_MINB)
@@ -85,7 +88,7 @@ constexpr int MAX_GROUP = 512;              // batches per group (claim director
 #define SEL_MINB32 2
 #endif
 constexpr int HW_CAP = 128;                 // A-Res candidates per warp
-constexpr int ROW_STAGE = 4096;             // rows of a tile staged in smem for coalesced writes
+constexpr int ROW_STAGE = 16 * RW_THREADS;  // rows of a tile staged in smem for coalesced writes
 
 struct HopParams {
   NWCore core;
@@ -1133,7 +1136,7 @@ __global__ void ROWS_LB hop_rows_kernel(HopParams P, int l, int64_t b0, int nbg,
   }
   if (staged) {
     __syncthreads();
-    for (int i = threadIdx.x; i < (int)tot; i += HB_THREADS) row_map[i] = (int32_t)stage[i];
+    for (int i = threadIdx.x; i < (int)tot; i += RW_THREADS) row_map[i] = (int32_t)stage[i];
   }
   if (t == ntile - 1 && threadIdx.x == 0) {  // the batch's row count
     long long* m = (long long*)(P.meta + (b * P.L + l) * 8);
@@ -1538,7 +1541,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
         GS_CUDA_TRY(cudaGetLastError());
         mark("ares", l);
       }
-      hop_rows_kernel<<<(unsigned)(nbg * ntile[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, ntile[l], srow); count_launch();
+      hop_rows_kernel<<<(unsigned)(nbg * ntile[l]), RW_THREADS, 0, stream>>>(P, l, b0, nbg, ntile[l], srow); count_launch();
       GS_CUDA_TRY(cudaGetLastError());
       mark("rows", l);
       const int64_t tiles = (maxbs * P.K[l] + RL_TILE - 1) / RL_TILE;
