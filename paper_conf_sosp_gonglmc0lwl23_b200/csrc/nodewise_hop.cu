@@ -50,7 +50,10 @@ constexpr int ROWS_TILE = RW_THREADS * WPT;        // bitmap words per dense row
 constexpr int SPARSE_TILE = RW_THREADS * WPT * 32; // bitmap words per summary-mode tile
 constexpr int CLEAR_TILE = 8192;            // words per dense clear CTA
 constexpr int NP_CPT = 8;                   // nprep: columns per thread
-constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
+#ifndef NP_THREADS
+#define NP_THREADS 256                      // nprep: threads per segment
+#endif
+constexpr int NP_SEG = NP_THREADS * NP_CPT; // columns per nprep segment
 #ifndef RL_ILP
 #define RL_ILP 4                            // relabel: edges per thread in flight (4 at 8 CTAs/SM: relabel1 0.130 vs 0.137 ms at 8 x 4 CTAs)
 #endif
@@ -67,7 +70,7 @@ constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
 #define SP_B 4                              // summary-mode row(): non-empty words loaded together
 #endif
 #ifndef NP_MINB
-#define NP_MINB 4
+#define NP_MINB (1024 / NP_THREADS)
 #endif
 #if ROWS_MINB > 0
 #define ROWS_LB __launch_bounds__(RW_THREADS, ROWS_MINB)
@@ -75,9 +78,9 @@ constexpr int NP_SEG = HB_THREADS * NP_CPT; // columns per nprep segment
 #define ROWS_LB __launch_bounds__(RW_THREADS)
 #endif
 #if NP_MINB > 0
-#define NP_LB __launch_bounds__(HB_THREADS, NP_MINB)
+#define NP_LB __launch_bounds__(NP_THREADS, NP_MINB)
 #else
-#define NP_LB __launch_bounds__(HB_THREADS)
+#define NP_LB __launch_bounds__(NP_THREADS)
 #endif
 constexpr int RL_TILE = HB_THREADS * RL_ILP;
 constexpr int MAX_GROUP = 512;              // batches per group (claim directories in smem)
@@ -337,7 +340,7 @@ __global__ void NP_LB hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, 
     }
     ex += cnt[q];
   }
-  if (threadIdx.x == HB_THREADS - 1 && (long long)(seg + 1) * NP_SEG >= T) {  // the batch's last segment
+  if (threadIdx.x == NP_THREADS - 1 && (long long)(seg + 1) * NP_SEG >= T) {  // the batch's last segment
     P.indptr_out[l][ib + T] = ex;
     long long* m = (long long*)(P.meta + (b * P.L + l) * 8);
     m[0] = T; m[1] = 0; m[2] = ex; m[3] = cb; m[4] = rb; m[5] = ib; m[6] = rb; m[7] = 0;
@@ -1510,7 +1513,7 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       const Scan srow{c4 + 1, st};
       st += WB * ntile[l];
       {
-        hop_nprep_kernel<<<(unsigned)(nbg * nseg_max[l]), HB_THREADS, 0, stream>>>(P, l, b0, nbg, snp); count_launch();
+        hop_nprep_kernel<<<(unsigned)(nbg * nseg_max[l]), NP_THREADS, 0, stream>>>(P, l, b0, nbg, snp); count_launch();
         GS_CUDA_TRY(cudaGetLastError());
         mark("nprep", l);
       }
