@@ -378,10 +378,10 @@ struct HChunk {
   uint32_t su[32 * KCAP];            // ... gathered row id
 };
 template <int KCAP>
-struct HChunk<KCAP, true> {
-  unsigned long long se[32 * KCAP];
-  uint32_t su[32 * KCAP];
-  float sv[32 * KCAP];               // ... PASS value
+struct HChunk<KCAP, true> {  // (>= 16 slots per lane: the k < d <= 64 group lists alias se / su / sv)
+  unsigned long long se[32 * (KCAP < 16 ? 16 : KCAP)];
+  uint32_t su[32 * (KCAP < 16 ? 16 : KCAP)];
+  float sv[32 * (KCAP < 16 ? 16 : KCAP)];  // ... PASS value
   uint32_t list[KCAP][32];           // selected positions, [rank][column lane]
 };
 
@@ -403,7 +403,10 @@ struct HSmem {
 // the lane's sampled rows gathered 16 at a time, bitmap bits set, edge id / row
 // id staged slot-major in shared memory, then written out coalesced.
 template <bool WEIGHTED, int KCAP>
-__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? 2 : (KCAP <= 16 ? SEL_MINB : SEL_MINB32))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
+#ifndef SEL_MINBW8
+#define SEL_MINBW8 2                        // weighted k <= 8 (PP hop 2): select2 20.5 ms vs 22.6 at 3 CTAs/SM, 23.0 with the 16-slot variant
+#endif
+__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? (KCAP <= 8 ? SEL_MINBW8 : 2) : (KCAP <= 16 ? SEL_MINB : SEL_MINB32))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
                                                                  unsigned int* claim) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = HSmem<WEIGHTED, KCAP>;
@@ -1521,8 +1524,9 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       const int64_t cub = (int64_t)nbg * ((maxbs * (l == 0 ? 1 : P.K[l - 1]) + 31) / 32);
       gs_status rc;
       if (weighted) {
-        rc = k <= 16 ? launch_select<true, 16>(P, l, b0, nbg, cq, cub, stream)
-                     : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream);
+        rc = k <= 8 ? launch_select<true, 8>(P, l, b0, nbg, cq, cub, stream)
+                    : (k <= 16 ? launch_select<true, 16>(P, l, b0, nbg, cq, cub, stream)
+                               : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream));
       } else {
         rc = k <= 8 ? launch_select<false, 8>(P, l, b0, nbg, cq, cub, stream)
                     : (k <= 16 ? launch_select<false, 16>(P, l, b0, nbg, cq, cub, stream)
