@@ -403,10 +403,13 @@ struct HSmem {
 // the lane's sampled rows gathered 16 at a time, bitmap bits set, edge id / row
 // id staged slot-major in shared memory, then written out coalesced.
 template <bool WEIGHTED, int KCAP>
+#ifndef SEL_MINB8
+#define SEL_MINB8 3
+#endif
 #ifndef SEL_MINBW8
 #define SEL_MINBW8 2                        // weighted k <= 8 (PP hop 2): select2 20.5 ms vs 22.6 at 3 CTAs/SM, 23.0 with the 16-slot variant
 #endif
-__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? (KCAP <= 8 ? SEL_MINBW8 : 2) : (KCAP <= 16 ? SEL_MINB : SEL_MINB32))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
+__global__ void __launch_bounds__(HS_THREADS, (WEIGHTED ? (KCAP <= 8 ? SEL_MINBW8 : 2) : (KCAP <= 8 ? SEL_MINB8 : (KCAP <= 16 ? SEL_MINB : SEL_MINB32)))) hop_select_kernel(HopParams P, int l, int64_t b0, int nbg,
                                                                  unsigned int* claim) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = HSmem<WEIGHTED, KCAP>;
