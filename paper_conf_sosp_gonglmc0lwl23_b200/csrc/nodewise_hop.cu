@@ -406,6 +406,9 @@ template <bool WEIGHTED, int KCAP>
 #ifndef SEL_MINB8
 #define SEL_MINB8 3
 #endif
+#ifndef SEL_W12
+#define SEL_W12 12                          // weighted 8 < k <= 12: a 12-slot variant
+#endif
 #ifndef SEL_MINBW8
 #define SEL_MINBW8 2                        // weighted k <= 8 (PP hop 2): select2 20.5 ms vs 22.6 at 3 CTAs/SM, 23.0 with the 16-slot variant
 #endif
@@ -1528,8 +1531,9 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
       gs_status rc;
       if (weighted) {
         rc = k <= 8 ? launch_select<true, 8>(P, l, b0, nbg, cq, cub, stream)
+                    : (k <= SEL_W12 ? launch_select<true, 12>(P, l, b0, nbg, cq, cub, stream)
                     : (k <= 16 ? launch_select<true, 16>(P, l, b0, nbg, cq, cub, stream)
-                               : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream));
+                               : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream)));
       } else {
         rc = k <= 8 ? launch_select<false, 8>(P, l, b0, nbg, cq, cub, stream)
                     : (k <= 16 ? launch_select<false, 16>(P, l, b0, nbg, cq, cub, stream)
