@@ -353,6 +353,19 @@ __global__ void NP_LB hop_nprep_kernel(HopParams P, int l, int64_t b0, int nbg, 
 // Ascending bitonic sorting network over a register array (N a power of two).
 template <int N>
 __device__ __forceinline__ void sort_net(uint32_t (&a)[N]) {
+  if constexpr ((N & (N - 1)) != 0) {
+    // N not a power of two: odd-even transposition (N rounds)
+#pragma unroll
+    for (int r = 0; r < N; ++r) {
+#pragma unroll
+      for (int i = r & 1; i + 1 < N; i += 2) {
+        const uint32_t x = a[i], y = a[i + 1];
+        a[i] = x < y ? x : y;
+        a[i + 1] = x < y ? y : x;
+      }
+    }
+    return;
+  }
 #pragma unroll
   for (int kk = 2; kk <= N; kk <<= 1) {
 #pragma unroll
@@ -405,6 +418,9 @@ struct HSmem {
 template <bool WEIGHTED, int KCAP>
 #ifndef SEL_MINB8
 #define SEL_MINB8 3
+#endif
+#ifndef SEL_U12
+#define SEL_U12 12                          // uniform 8 < k <= 12: a 12-slot variant
 #endif
 #ifndef SEL_W12
 #define SEL_W12 12                          // weighted 8 < k <= 12: a 12-slot variant
@@ -1536,8 +1552,9 @@ gs_status run_nodewise_hop(const gs_graph* g, const int32_t* seeds, int64_t num_
                                : launch_select<true, 32>(P, l, b0, nbg, cq, cub, stream)));
       } else {
         rc = k <= 8 ? launch_select<false, 8>(P, l, b0, nbg, cq, cub, stream)
+                    : (k <= SEL_U12 ? launch_select<false, 12>(P, l, b0, nbg, cq, cub, stream)
                     : (k <= 16 ? launch_select<false, 16>(P, l, b0, nbg, cq, cub, stream)
-                               : launch_select<false, 32>(P, l, b0, nbg, cq, cub, stream));
+                               : launch_select<false, 32>(P, l, b0, nbg, cq, cub, stream)));
       }
       if (rc) return rc;
       mark("select", l);
