@@ -1,7 +1,7 @@
 # Round-2 evidence (final session): full GPU tests, smoke, the default bench
 # line (+ reference arm), a sweep of every workload, the launch list and an
 # ncu --set full capture of the default workload's hop kernels.
-O=gpurun_out/ev11; mkdir -p $O
+O=gpurun_out/ev12; mkdir -p $O
 timeout 2400 python -m pytest tests -m gpu -q -rf > $O/pytest_gpu.log 2>&1; echo "rc=$?" >> $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log
 timeout 600 python bench.py > $O/bench_default.log 2>&1; echo "rc=$?" >> $O/bench_default.log
